@@ -1,0 +1,436 @@
+/*
+ * hccmf_oracle.c -- the plain, slow, serial CPU ORACLE for the HCC-MF hot path.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and bench.py's
+ * cpu_baseline / --impl reference legs may load this library.  The product path
+ * (paper_conf_icpp_huangylhbl21_b200/) never links, imports or calls it, and it
+ * shares no code, header, table or constant generator with the CUDA path: every
+ * function below is written from PAPER.md (Huang et al., ICPP '21) and from the
+ * readings recorded in DESIGN.md section 3 ("Readings of the paper").
+ *
+ * Citation convention: L<n> = /root/reference/PAPER.md line n.
+ *
+ * Arithmetic: fp64 for every floating-point quantity (the paper fixes no
+ * precision for P and Q; L1234-L1249 only mentions FP16 for transmission).
+ * Build strictly: -O2 -ffp-contract=off, no -ffast-math, no OpenMP, so each
+ * a*b+c is two IEEE roundings, exactly as written.
+ *
+ * Pins (tests/test_oracle_pins.py, -m "not gpu"): Fig. 1 worked example
+ * (L283-L403), finite-difference gradient, monotone loss at small gamma,
+ * planted rank-k recovery, full-batch O(gamma^2) limit, dense brute-force
+ * objective, Theorem-1 equalisation (L924-L954), Eq. 6 closed form, brute-force
+ * partition/sort on tiny inputs, SplitMix64 published test vectors.
+ * Parity unpinned: none of the functions below is left without a pin; the
+ * all-reduce replica mode is pinned only against its own definition
+ * (mean of per-shard replicas) -- see DESIGN.md section 3, reading R13.
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+/* ------------------------------------------------------------------------- */
+/* Counter-based hash (R8: "shuffling", L546).  SplitMix64 finaliser  */
+/* as published by Steele, Lea & Flood (2014); the CUDA side implements the     */
+/* same specification independently.                                           */
+/* ------------------------------------------------------------------------- */
+uint64_t orc_splitmix(uint64_t x)
+{
+    uint64_t z = x + 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+/* H(seed, tag, a, b) = sm(sm(sm(seed ^ (tag << 56)) ^ a) ^ b) */
+uint64_t orc_hash(uint64_t seed, uint64_t tag, uint64_t a, uint64_t b)
+{
+    uint64_t h = orc_splitmix(seed ^ (tag << 56));
+    h = orc_splitmix(h ^ a);
+    return orc_splitmix(h ^ b);
+}
+
+/* U[0,1) with 24 random bits: exact in fp32 and fp64. */
+double orc_uniform(uint64_t h) { return (double)(h >> 40) * (1.0 / 16777216.0); }
+
+/* ------------------------------------------------------------------------- */
+/* Step 1 of the preprocessing (L543-L548): shuffle = seeded ID permutation.   */
+/* perm[id] = rank of (H(seed, tag, id, 0), id) among all ids; seed 0 = identity */
+/* ------------------------------------------------------------------------- */
+typedef struct { uint64_t key; int64_t id; } orc_keyid;
+
+static int cmp_keyid(const void* a, const void* b)
+{
+    const orc_keyid* x = (const orc_keyid*)a;
+    const orc_keyid* y = (const orc_keyid*)b;
+    if (x->key != y->key) return x->key < y->key ? -1 : 1;
+    if (x->id != y->id) return x->id < y->id ? -1 : 1;
+    return 0;
+}
+
+int orc_perm(uint64_t seed, uint64_t tag, int64_t count, int32_t* perm)
+{
+    if (count < 0) return -1;
+    if (seed == 0) {
+        for (int64_t i = 0; i < count; ++i) perm[i] = (int32_t)i;
+        return 0;
+    }
+    orc_keyid* a = (orc_keyid*)malloc(sizeof(orc_keyid) * (size_t)(count ? count : 1));
+    if (!a) return -3;
+    for (int64_t i = 0; i < count; ++i) {
+        a[i].key = orc_hash(seed, tag, (uint64_t)i, 0);
+        a[i].id = i;
+    }
+    qsort(a, (size_t)count, sizeof(orc_keyid), cmp_keyid);
+    for (int64_t r = 0; r < count; ++r) perm[a[r].id] = (int32_t)r;
+    free(a);
+    return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* Data partition strategies (section 3.3).                        */
+/* ------------------------------------------------------------------------- */
+
+/* DP0, Eq. 6 (L967-L981): x_i = 1 / sum_j (T_i,e / T_j,e). */
+void orc_dp0(int32_t p, const double* t_e, double* x)
+{
+    for (int32_t i = 0; i < p; ++i) {
+        double s = 0.0;
+        for (int32_t j = 0; j < p; ++j) s += t_e[i] / t_e[j];
+        x[i] = 1.0 / s;
+    }
+}
+
+/* Theorem 1 (L924-L954) with unequal b_i: the minimiser of max_i(a_i x_i + b_i)
+ * s.t. sum x_i = 1, x_i >= 0 equalises a_i x_i + b_i over the workers that get
+ * data.  Water-filling: T* = (1 + sum b_j/a_j) / sum (1/a_j) over the active set;
+ * workers with b_i >= T* get x_i = 0 and leave the active set. */
+void orc_dp0_affine(int32_t p, const double* a, const double* b, double* x)
+{
+    int32_t* active = (int32_t*)malloc(sizeof(int32_t) * (size_t)(p ? p : 1));
+    for (int32_t i = 0; i < p; ++i) active[i] = 1;
+    for (;;) {
+        double num = 1.0, den = 0.0;
+        for (int32_t j = 0; j < p; ++j)
+            if (active[j]) { num += b[j] / a[j]; den += 1.0 / a[j]; }
+        double T = num / den;
+        int changed = 0;
+        for (int32_t j = 0; j < p; ++j)
+            if (active[j] && b[j] >= T) { active[j] = 0; changed = 1; }
+        if (!changed) {
+            for (int32_t j = 0; j < p; ++j) x[j] = active[j] ? (T - b[j]) / a[j] : 0.0;
+            break;
+        }
+    }
+    free(active);
+}
+
+/* DP1, Algorithm 1 (L1025-L1142) generalised to a GPU-only box (R11):
+ * per-shard compensation toward the mean time, renormalised, stop when
+ * max_s |t_s - Tbar| / min_s t_s <= 0.1, at most 8 rounds.  The re-measurement
+ * of line 12 (sgd_update) uses the paper's constant-bandwidth observation
+ * (L1013-L1016): t_s scales linearly with x_s.  Returns the number of rounds. */
+int32_t orc_dp1(int32_t p, const double* x_in, const double* t_in, double* x_out)
+{
+    double* x = (double*)malloc(sizeof(double) * (size_t)p);
+    double* t = (double*)malloc(sizeof(double) * (size_t)p);
+    memcpy(x, x_in, sizeof(double) * (size_t)p);
+    memcpy(t, t_in, sizeof(double) * (size_t)p);
+    int32_t it = 0;
+    for (; it < 8; ++it) {
+        double tbar = 0.0, tmin = t[0], dev = 0.0;
+        for (int32_t s = 0; s < p; ++s) tbar += t[s];
+        tbar /= (double)p;
+        for (int32_t s = 0; s < p; ++s) {
+            if (t[s] < tmin) tmin = t[s];
+            double d = fabs(t[s] - tbar);
+            if (d > dev) dev = d;
+        }
+        if (dev / tmin <= 0.1) break;
+        double sum = 0.0;
+        for (int32_t s = 0; s < p; ++s) sum += x[s] * tbar / t[s];
+        for (int32_t s = 0; s < p; ++s) {
+            double xn = (x[s] * tbar / t[s]) / sum;
+            t[s] = t[s] * xn / x[s];
+            x[s] = xn;
+        }
+    }
+    memcpy(x_out, x, sizeof(double) * (size_t)p);
+    free(x);
+    free(t);
+    return it;
+}
+
+/* DP2, Eq. 7 (L1143-L1172) (R12): the shard s_med = (p-1)/2 keeps its
+ * DP1 time T_med = t[s_med]; shard s targets T_s = T_med + (s - s_med) * T_sync so
+ * that shard s's sync hides under shard s+1's compute; x_s <- x_s * T_s / t_s
+ * (line 6 of Algorithm 1, the "similar method"), renormalised. */
+void orc_dp2(int32_t p, const double* x_in, const double* t_in, double t_sync, double* x_out)
+{
+    int32_t smed = (p - 1) / 2;
+    double tmed = t_in[smed];
+    double sum = 0.0;
+    for (int32_t s = 0; s < p; ++s) {
+        double Ts = tmed + (double)(s - smed) * t_sync;
+        if (Ts < 0.0) Ts = 0.0;
+        x_out[s] = x_in[s] * Ts / t_in[s];
+        sum += x_out[s];
+    }
+    for (int32_t s = 0; s < p; ++s) x_out[s] /= sum;
+}
+
+/* Row grid (L881-L895): per-row counts in permuted order, exclusive prefix S
+ * (S has m+1 entries), and shard boundaries b_0 = 0 <= ... <= b_G = m where b_s
+ * is the row r in [b_{s-1}, m] minimising |S[r] - llround(nnz * sum_{j<s} x_j)|,
+ * ties to the smaller r (R10).  Brute-force linear scan. */
+void orc_row_prefix(int64_t m, int64_t nnz, const int32_t* u, const int32_t* perm_row, int64_t* S)
+{
+    int64_t* cnt = (int64_t*)calloc((size_t)(m + 1), sizeof(int64_t));
+    for (int64_t i = 0; i < nnz; ++i) cnt[perm_row[u[i]]] += 1;
+    S[0] = 0;
+    for (int64_t r = 0; r < m; ++r) S[r + 1] = S[r] + cnt[r];
+    free(cnt);
+}
+
+void orc_bounds(int64_t m, int64_t nnz, const int64_t* S, int32_t G, const double* x, int32_t* b)
+{
+    double cum = 0.0;
+    b[0] = 0;
+    for (int32_t s = 1; s < G; ++s) {
+        cum += x[s - 1];
+        int64_t T = llround((double)nnz * cum);
+        int64_t best = b[s - 1];
+        for (int64_t r = b[s - 1]; r <= m; ++r) {
+            int64_t dr = S[r] - T, db = S[best] - T;
+            if (dr < 0) dr = -dr;
+            if (db < 0) db = -db;
+            if (dr < db) best = r;
+        }
+        b[s] = (int32_t)best;
+    }
+    b[G] = (int32_t)m;
+}
+
+/* ------------------------------------------------------------------------- */
+/* Blocking + stable sort (L546 "sorting", L1472-L1474 row-sorted blocks).      */
+/* Record i goes to shard s (b_s <= u' < b_{s+1}), row block                     */
+/* rb = floor((u'-b_s) * Br / (b_{s+1}-b_s)), column block cb = floor(v' * Bc / n),*/
+/* and records are ordered by (s, rb, cb, u', v', i).                            */
+/* off[((s*Br + rb)*Bc + cb)] = first record of the block; off has G*Br*Bc+1.    */
+/* ------------------------------------------------------------------------- */
+typedef struct { int64_t blk; int32_t up, vp; int64_t i; } orc_rec;
+
+static int cmp_rec(const void* a, const void* b)
+{
+    const orc_rec* x = (const orc_rec*)a;
+    const orc_rec* y = (const orc_rec*)b;
+    if (x->blk != y->blk) return x->blk < y->blk ? -1 : 1;
+    if (x->up != y->up) return x->up < y->up ? -1 : 1;
+    if (x->vp != y->vp) return x->vp < y->vp ? -1 : 1;
+    if (x->i != y->i) return x->i < y->i ? -1 : 1;
+    return 0;
+}
+
+int orc_block_sort(int64_t m, int64_t n, int64_t nnz, const int32_t* u, const int32_t* v,
+                   const float* r, int32_t G, int32_t Br, int32_t Bc, const int32_t* b,
+                   const int32_t* perm_row, const int32_t* perm_col, int32_t* out_u,
+                   int32_t* out_v, float* out_r, int64_t* off)
+{
+    int64_t nblk = (int64_t)G * Br * Bc;
+    orc_rec* a = (orc_rec*)malloc(sizeof(orc_rec) * (size_t)(nnz ? nnz : 1));
+    if (!a) return -3;
+    for (int64_t i = 0; i < nnz; ++i) {
+        int32_t up = perm_row[u[i]], vp = perm_col[v[i]];
+        int32_t s = 0;
+        while (!(b[s] <= up && up < b[s + 1])) ++s;
+        int64_t rows = (int64_t)b[s + 1] - b[s];
+        int64_t rb = ((int64_t)(up - b[s]) * Br) / rows;
+        int64_t cb = ((int64_t)vp * Bc) / n;
+        a[i].blk = ((int64_t)s * Br + rb) * Bc + cb;
+        a[i].up = up;
+        a[i].vp = vp;
+        a[i].i = i;
+    }
+    qsort(a, (size_t)nnz, sizeof(orc_rec), cmp_rec);
+    for (int64_t j = 0; j <= nblk; ++j) off[j] = 0;
+    for (int64_t j = 0; j < nnz; ++j) off[a[j].blk + 1] += 1;
+    for (int64_t j = 0; j < nblk; ++j) off[j + 1] += off[j];
+    for (int64_t j = 0; j < nnz; ++j) {
+        out_u[j] = a[j].up;
+        out_v[j] = a[j].vp;
+        out_r[j] = r[a[j].i];
+    }
+    free(a);
+    (void)m;
+    return 0;
+}
+
+/* ------------------------------------------------------------------------- */
+/* Factor initialisation (R5; the paper is silent): on ORIGINAL ids, */
+/* P[u][j] = U(H(seed,3,u,j)) * sqrt(1/k), Q[v][j] = U(H(seed,4,v,j)) * sqrt(1/k).*/
+/* Stored in permuted order: P'[perm_row[u]] = P[u].                           */
+/* ------------------------------------------------------------------------- */
+void orc_init(uint64_t seed, int64_t m, int64_t n, int32_t k, const int32_t* perm_row,
+              const int32_t* perm_col, double* P, double* Q)
+{
+    double sc = sqrt(1.0 / (double)k);
+    for (int64_t u = 0; u < m; ++u)
+        for (int32_t j = 0; j < k; ++j)
+            P[(int64_t)perm_row[u] * k + j] = orc_uniform(orc_hash(seed, 3, (uint64_t)u, (uint64_t)j)) * sc;
+    for (int64_t v = 0; v < n; ++v)
+        for (int32_t j = 0; j < k; ++j)
+            Q[(int64_t)perm_col[v] * k + j] = orc_uniform(orc_hash(seed, 4, (uint64_t)v, (uint64_t)j)) * sc;
+}
+
+/* ------------------------------------------------------------------------- */
+/* The per-rating SGD update (section 2.1, Fig. 1,          */
+/* north_star; R1 old-p reading, R2 gamma absorbs the factor 2):      */
+/*   e  = r - p.q                                                              */
+/*   p' = p + gamma (e q - lambda p)                                           */
+/*   q' = q + gamma (e p - lambda q)      (p = value before this update)       */
+/* Returns e.                                                                  */
+/* ------------------------------------------------------------------------- */
+double orc_sgd_update(int32_t k, double gamma, double lambda, double* p, double* q, double r)
+{
+    double d = 0.0;
+    for (int32_t j = 0; j < k; ++j) d += p[j] * q[j];
+    double e = r - d;
+    for (int32_t j = 0; j < k; ++j) {
+        double pj = p[j], qj = q[j];
+        p[j] = pj + gamma * (e * qj - lambda * pj);
+        q[j] = qj + gamma * (e * pj - lambda * qj);
+    }
+    return e;
+}
+
+/* Serial pass over records [lo, hi) in stored order. */
+void orc_run(int64_t lo, int64_t hi, int32_t k, double gamma, double lambda, const int32_t* ru,
+             const int32_t* rv, const float* rr, double* P, double* Q)
+{
+    for (int64_t i = lo; i < hi; ++i)
+        orc_sgd_update(k, gamma, lambda, P + (int64_t)ru[i] * k, Q + (int64_t)rv[i] * k, (double)rr[i]);
+}
+
+/* One epoch in the canonical serialisation of a schedule (R19).
+ *   sched 0 = DET (conflict-free strata, L2269-L2275), 1 = SERIAL (the record
+ *   order the Hogwild mode races through, L216-L219).
+ *   sync  0 = NONE (G == 1), 1 = RING (rotating Q column groups, L1143-L1172,
+ *   L1251-L1269), 2 = ALLREDUCE_AVG (per-shard Q replica, then the server's
+ *   multiply-add sync Q = sum_s Q_s / G, L549-L557, L783-L784).
+ * DET needs Br == Bc (NONE, ALLREDUCE) or Bc == G*Br (RING).
+ * Returns 0, or -1 for an invalid grid. */
+static void det_square(int32_t s, int32_t c, int32_t Br, int32_t Bc, int32_t col0, const int64_t* off,
+                       int32_t k, double gamma, double lambda, const int32_t* ru, const int32_t* rv,
+                       const float* rr, double* P, double* Q)
+{
+    for (int32_t t = 0; t < c; ++t)
+        for (int32_t i = 0; i < c; ++i) {
+            int64_t blk = ((int64_t)s * Br + i) * Bc + col0 + (i + t) % c;
+            orc_run(off[blk], off[blk + 1], k, gamma, lambda, ru, rv, rr, P, Q);
+        }
+}
+
+int orc_epoch(int32_t sched, int32_t sync, int32_t G, int32_t Br, int32_t Bc, const int64_t* off,
+              int64_t n, int32_t k, double gamma, double lambda, const int32_t* ru, const int32_t* rv,
+              const float* rr, double* P, double* Q)
+{
+    if (sync == 0) {
+        if (G != 1) return -1;
+        if (sched == 0) {
+            if (Br != Bc) return -1;
+            det_square(0, Br, Br, Bc, 0, off, k, gamma, lambda, ru, rv, rr, P, Q);
+        } else {
+            orc_run(0, off[(int64_t)Br * Bc], k, gamma, lambda, ru, rv, rr, P, Q);
+        }
+        return 0;
+    }
+    if (sync == 1) {
+        if (Bc % G != 0) return -1;
+        int32_t c = Bc / G;
+        if (sched == 0 && c != Br) return -1;
+        for (int32_t t = 0; t < G; ++t)
+            for (int32_t s = 0; s < G; ++s) {
+                int32_t g = (s + t) % G;
+                if (sched == 0) {
+                    det_square(s, c, Br, Bc, g * c, off, k, gamma, lambda, ru, rv, rr, P, Q);
+                } else {
+                    for (int32_t j = 0; j < c; ++j)
+                        for (int32_t rb = 0; rb < Br; ++rb) {
+                            int64_t blk = ((int64_t)s * Br + rb) * Bc + g * c + j;
+                            orc_run(off[blk], off[blk + 1], k, gamma, lambda, ru, rv, rr, P, Q);
+                        }
+                }
+            }
+        return 0;
+    }
+    if (sync == 2) {
+        if (sched == 0 && Br != Bc) return -1;
+        size_t qn = (size_t)n * (size_t)k;
+        double* Qs = (double*)malloc(sizeof(double) * qn);
+        double* Qsum = (double*)calloc(qn, sizeof(double));
+        for (int32_t s = 0; s < G; ++s) {
+            memcpy(Qs, Q, sizeof(double) * qn);
+            if (sched == 0) {
+                det_square(s, Br, Br, Bc, 0, off, k, gamma, lambda, ru, rv, rr, P, Qs);
+            } else {
+                int64_t lo = off[(int64_t)s * Br * Bc], hi = off[(int64_t)(s + 1) * Br * Bc];
+                orc_run(lo, hi, k, gamma, lambda, ru, rv, rr, P, Qs);
+            }
+            for (size_t i = 0; i < qn; ++i) Qsum[i] += Qs[i];
+        }
+        for (size_t i = 0; i < qn; ++i) Q[i] = Qsum[i] / (double)G;
+        free(Qs);
+        free(Qsum);
+        return 0;
+    }
+    return -1;
+}
+
+/* ------------------------------------------------------------------------- */
+/* Evaluation (Fig. 1 caption L405-L407; Fig. 7).                              */
+/* RMSE over a set T given in ORIGINAL ids: sqrt(sum (r - p_u.q_v)^2 / |T|).   */
+/* ------------------------------------------------------------------------- */
+double orc_rmse(int64_t nt, const int32_t* tu, const int32_t* tv, const float* tr, int32_t k,
+                const int32_t* perm_row, const int32_t* perm_col, const double* P, const double* Q)
+{
+    if (nt == 0) return 0.0;
+    double sse = 0.0;
+    for (int64_t i = 0; i < nt; ++i) {
+        const double* p = P + (int64_t)perm_row[tu[i]] * k;
+        const double* q = Q + (int64_t)perm_col[tv[i]] * k;
+        double d = 0.0;
+        for (int32_t j = 0; j < k; ++j) d += p[j] * q[j];
+        double e = (double)tr[i] - d;
+        sse += e * e;
+    }
+    return sqrt(sse / (double)nt);
+}
+
+/* Objective over the training set in ORIGINAL ids (R2, R4):
+ * L = sum_Omega [ (r - p_u.q_v)^2 + lambda (|p_u|^2 + |q_v|^2) ]. */
+double orc_objective(int64_t nnz, const int32_t* u, const int32_t* v, const float* r, int32_t k,
+                     double lambda, const int32_t* perm_row, const int32_t* perm_col, const double* P,
+                     const double* Q)
+{
+    double L = 0.0;
+    for (int64_t i = 0; i < nnz; ++i) {
+        const double* p = P + (int64_t)perm_row[u[i]] * k;
+        const double* q = Q + (int64_t)perm_col[v[i]] * k;
+        double d = 0.0, pp = 0.0, qq = 0.0;
+        for (int32_t j = 0; j < k; ++j) {
+            d += p[j] * q[j];
+            pp += p[j] * p[j];
+            qq += q[j] * q[j];
+        }
+        double e = (double)r[i] - d;
+        L += e * e + lambda * (pp + qq);
+    }
+    return L;
+}
+
+/* Export (final push, L1205-L1206): un-permute to original ids. */
+void orc_unpermute(int64_t rows, int32_t k, const int32_t* perm, const double* Xp, double* X)
+{
+    for (int64_t i = 0; i < rows; ++i)
+        memcpy(X + i * k, Xp + (int64_t)perm[i] * k, sizeof(double) * (size_t)k);
+}

@@ -1,0 +1,159 @@
+"""Pins for the oracle's partitioner (section 3.3) and blocker (L546, L1472-L1474).
+
+Brute force on tiny inputs with Python's sorted/min (textbook routines), the
+DP0 closed form (Eq. 6), Theorem 1's equalisation, and invariants.
+"""
+import math
+
+import numpy as np
+import pytest
+
+
+def _llround(x):
+    return int(math.floor(x + 0.5))  # x >= 0: round half away from zero
+
+
+def _bruteforce_partition(m, n, u, v, G, Br, Bc, x, perm_row, perm_col):
+    cnt = np.bincount(perm_row[u], minlength=m) if len(u) else np.zeros(m, int)
+    S = [0]
+    for c in cnt:
+        S.append(S[-1] + int(c))
+    b = [0]
+    cum = 0.0
+    for s in range(1, G):
+        cum += x[s - 1]
+        T = _llround(len(u) * cum)
+        b.append(min(range(b[-1], m + 1), key=lambda r_: (abs(S[r_] - T), r_)))
+    b.append(m)
+    recs = []
+    for i in range(len(u)):
+        up, vp = int(perm_row[u[i]]), int(perm_col[v[i]])
+        s = max(j for j in range(G) if b[j] <= up < b[j + 1])
+        rb = (up - b[s]) * Br // (b[s + 1] - b[s])
+        cb = vp * Bc // n
+        recs.append((((s * Br + rb) * Bc + cb), up, vp, i))
+    recs.sort()
+    off = [0] * (G * Br * Bc + 1)
+    for rec in recs:
+        off[rec[0] + 1] += 1
+    for j in range(G * Br * Bc):
+        off[j + 1] += off[j]
+    return S, b, recs, off
+
+
+def test_partition_and_sort_bruteforce(orc):
+    import synth
+    rng = np.random.default_rng(1234)
+    for trial in range(400):
+        m, n = int(rng.integers(1, 9)), int(rng.integers(1, 9))
+        nnz = int(rng.integers(0, 65))
+        G = int(rng.integers(1, min(m, 4) + 1))
+        Br, Bc = int(rng.integers(1, 5)), int(rng.integers(1, 5))
+        seed = 0 if trial % 4 == 0 else int(rng.integers(1, 2**62))
+        u, v, r = synth.tiny(m, n, nnz, seed=trial)
+        x = rng.dirichlet(np.ones(G)) if trial % 2 else np.full(G, 1.0 / G)
+        pr, pc = orc.perm(seed, 1, m), orc.perm(seed, 2, n)
+        S, b, recs, off = _bruteforce_partition(m, n, u, v, G, Br, Bc, x, pr, pc)
+        assert list(orc.row_prefix(m, u, pr)) == S
+        ob = orc.bounds(m, nnz, np.array(S, np.int64), G, x)
+        assert list(ob) == b
+        if any(b[s + 1] == b[s] for s in range(G)) and nnz:
+            # an empty shard with ratings elsewhere is fine; the blocker never
+            # divides by its zero row count because no record lands in it
+            pass
+        ou, ov, orr, ooff = orc.block_sort(m, n, u, v, r, G, Br, Bc, ob, pr, pc)
+        assert list(ooff) == off
+        assert list(ou) == [t[1] for t in recs] and list(ov) == [t[2] for t in recs]
+        assert np.array_equal(orr, r[[t[3] for t in recs]])
+
+
+def test_partition_invariants_medium(orc):
+    import synth
+    m, n, nnz = 500, 300, 20000
+    (u, v, r), _ = synth.powerlaw(m, n, nnz, seed=3, n_test=0)
+    for seed in (0, 99):
+        pr, pc = orc.perm(seed, 1, m), orc.perm(seed, 2, n)
+        assert sorted(pr) == list(range(m)) and sorted(pc) == list(range(n))
+        S = orc.row_prefix(m, u, pr)
+        cnt = np.diff(S)
+        for G in (1, 2, 3, 8):
+            x = np.full(G, 1.0 / G)
+            b = orc.bounds(m, nnz, S, G, x)
+            assert b[0] == 0 and b[-1] == m and np.all(np.diff(b) >= 0)
+            cum = np.cumsum(x)
+            for s in range(1, G):
+                assert abs(S[b[s]] - _llround(nnz * cum[s - 1])) <= cnt.max()
+            ou, ov, orr, off = orc.block_sort(m, n, u, v, r, G, 4, 5, b, pr, pc)
+            assert off[-1] == nnz
+            # multiset preserved
+            a = np.sort(np.stack([ou, ov, orr.view(np.int32)]), axis=1)
+            want = np.sort(np.stack([pr[u], pc[v], r.view(np.int32)]), axis=1)
+            assert np.array_equal(np.sort(ou), np.sort(pr[u]))
+            assert np.array_equal(np.sort(orr), np.sort(r))
+            # row-sorted within each block; every record inside its block's ranges
+            for blk in range(G * 20):
+                lo, hi = off[blk], off[blk + 1]
+                s, rem = divmod(blk, 20)
+                rb, cb = divmod(rem, 5)
+                key = ou[lo:hi].astype(np.int64) * n + ov[lo:hi]
+                assert np.all(np.diff(key) >= 0)
+                assert np.all((ou[lo:hi] >= b[s]) & (ou[lo:hi] < b[s + 1]))
+                assert np.all(ov[lo:hi] * 5 // n == cb)
+            del a, want
+
+
+def test_dp0_eq6_closed_form(orc):
+    # Eq. 6: x_i = 1 / sum_j (T_i,e / T_j,e)  ==  (1/T_i) / sum_j (1/T_j); sum = 1;
+    # Theorem 1 with equal b: a_i x_i equal for all i (L961-L964)
+    t = np.array([1.0, 2.0, 4.0, 0.5])
+    x = orc.dp0(t)
+    np.testing.assert_allclose(x, (1 / t) / np.sum(1 / t), rtol=1e-15)
+    assert x.sum() == pytest.approx(1.0, abs=1e-15)
+    np.testing.assert_allclose(t * x, (t * x)[0], rtol=1e-14)
+    # homogeneous GPUs -> 1/G
+    np.testing.assert_allclose(orc.dp0(np.full(8, 3.3)), np.full(8, 1 / 8), rtol=1e-15)
+
+
+def test_theorem1_affine_equalisation(orc):
+    # Theorem 1 (L924-L954): argmin max(a_i x_i + b_i) s.t. sum x = 1 equalises
+    # a_i x_i + b_i; checked against a brute-force grid search for p = 3
+    a = np.array([2.0, 3.0, 5.0])
+    b = np.array([0.1, 0.3, 0.2])
+    x = orc.dp0_affine(a, b)
+    assert x.sum() == pytest.approx(1.0, abs=1e-14)
+    np.testing.assert_allclose(a * x + b, (a * x + b)[0], rtol=1e-12)
+    best = min(((max(a[0] * i / 400 + b[0], a[1] * j / 400 + b[1], a[2] * (400 - i - j) / 400 + b[2]), i, j)
+                for i in range(401) for j in range(401 - i)))
+    assert max(a * x + b) <= best[0] + 1e-12
+    assert max(a * x + b) == pytest.approx(best[0], abs=0.01)
+    # a worker whose communication alone exceeds the optimum gets no data
+    x = orc.dp0_affine(np.array([1.0, 1.0]), np.array([0.0, 5.0]))
+    np.testing.assert_allclose(x, [1.0, 0.0])
+
+
+def test_dp1_compensation(orc):
+    # Algorithm 1 (L1025-L1142), GPU-only generalisation (R11):
+    # already balanced within 10% -> unchanged, zero rounds
+    x0 = np.array([0.25, 0.25, 0.25, 0.25])
+    x, it = orc.dp1(x0, np.array([1.0, 1.05, 0.97, 1.02]))
+    assert it == 0 and np.array_equal(x, x0)
+    # imbalanced: the linear-bandwidth model (L1013-L1016) balances in one round
+    t = np.array([1.0, 2.0, 1.0, 1.0])
+    x, it = orc.dp1(x0, t)
+    assert it == 1 and x.sum() == pytest.approx(1.0, abs=1e-15)
+    pred = t * x / x0  # predicted times at the new partition
+    np.testing.assert_allclose(pred, pred[0], rtol=1e-12)
+    assert x[1] < x[0]
+
+
+def test_dp2_hidden_sync_ramp(orc):
+    # Eq. 7 (L1166): T_(i+-n),c = T_i,c +- n T_i,sync around the median shard
+    x0 = np.full(5, 0.2)
+    t = np.full(5, 1.0)
+    x = orc.dp2(x0, t, 0.1)
+    assert x.sum() == pytest.approx(1.0, abs=1e-15)
+    pred = t * x / x0
+    d = np.diff(pred)
+    np.testing.assert_allclose(d, d[0], rtol=1e-12)
+    # ramp step relative to the median time equals t_sync / T_med
+    assert d[0] / pred[2] == pytest.approx(0.1, rel=1e-12)

@@ -1,0 +1,275 @@
+"""Pins for the CPU oracle against what the paper and mathematics fix (-m "not gpu").
+
+Each test pins the oracle to something other than itself: values printed in the
+paper (Fig. 1), hand-computed worked examples, closed forms, invariants,
+finite differences and brute force.  A plausible mistake in the oracle (a
+dropped term, a wrong sign or index, a transposed operand, new-p instead of
+old-p) fails at least one of them; the comment on each test says which.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import golden_io
+
+GOLDEN_MIX = 0x9E3779B97F4A7C15
+M64 = (1 << 64) - 1
+
+
+# ----------------------------------------------------------------- hash spec
+def test_splitmix64_published_vectors(orc):
+    # SplitMix64 (Steele, Lea, Flood 2014) from state 0: the first four outputs
+    # of the reference generator.  orc_splitmix(x) = mix(x + golden), so output i
+    # is orc_splitmix(i * golden).  Pins every constant and shift of the mixer.
+    want = [0xE220A8397B1DCDAF, 0x6E789E6AA1B965F4, 0x06C45D188009454F, 0xF88BB8A8724C81EC]
+    got = [orc.splitmix((i * GOLDEN_MIX) & M64) for i in range(4)]
+    assert got == want
+
+
+def test_hash_composition_and_uniform(orc):
+    # H(seed, tag, a, b) = sm(sm(sm(seed ^ tag<<56) ^ a) ^ b)  (R8)
+    for seed, tag, a, b in [(1, 1, 0, 0), (7, 3, 12345, 17), (2**63 + 5, 4, 2**31 - 1, 127)]:
+        h = orc.splitmix((seed ^ (tag << 56)) & M64)
+        h = orc.splitmix(h ^ a)
+        h = orc.splitmix(h ^ b)
+        assert orc.hash4(seed, tag, a, b) == h
+    # U = (h >> 40) * 2^-24: 0 for h < 2^40 and 1 - 2^-24 for h = 2^64 - 1
+    assert orc.uniform(0) == 0.0
+    assert orc.uniform(M64) == 1.0 - 2.0 ** -24
+    assert orc.uniform(1 << 63) == 0.5
+
+
+def test_perm_bruteforce(orc):
+    # seed 0 = identity; otherwise perm[id] = rank of (H(seed,tag,id,0), id), by Python sorted
+    assert list(orc.perm(0, 1, 9)) == list(range(9))
+    rng = np.random.default_rng(0)
+    for _ in range(50):
+        cnt = int(rng.integers(1, 40))
+        seed = int(rng.integers(1, 2**63))
+        tag = int(rng.integers(1, 3))
+        keys = [(orc.hash4(seed, tag, i, 0), i) for i in range(cnt)]
+        order = sorted(range(cnt), key=lambda i: keys[i])
+        want = np.empty(cnt, np.int32)
+        want[order] = np.arange(cnt)
+        assert np.array_equal(orc.perm(seed, tag, cnt), want)
+
+
+# ------------------------------------------------------------ Fig. 1 (paper)
+def test_fig1_prediction_matches_printed_Rp(orc):
+    # Fig. 1 (L283-L403): R_p = P x Q printed to 2 decimals, all 20 cells.  The
+    # oracle's inner product is read through sgd_update with gamma = 0, r = 0
+    # (returns e = -p.q).  Pins the dot product and the P (m x k) / Q (n x k)
+    # orientation (a transposed Q fails).
+    _, P, Q, Rp = golden_io.fig1()
+    for i in range(5):
+        for j in range(4):
+            p, q = P[i].copy(), Q[j].copy()
+            pred = -orc.sgd_update(0.0, 0.0, p, q, 0.0)
+            assert round(pred + 1e-12, 2) == pytest.approx(Rp[i, j], abs=1e-9), (i, j)
+
+
+def test_fig1_training_rmse(orc):
+    # RMSE over the 12 observed ratings of Fig. 1 with the printed P, Q, computed
+    # independently with numpy: SSE = 0.50034114, RMSE = 0.2041938.
+    (u, v, r), P, Q, _ = golden_io.fig1()
+    pr = np.arange(5, dtype=np.int32)
+    pc = np.arange(4, dtype=np.int32)
+    sse = float(np.sum((r.astype(np.float64) - np.sum(P[u] * Q[v], axis=1)) ** 2))
+    assert sse == pytest.approx(0.50034114, abs=1e-8)
+    assert orc.rmse(u, v, r, pr, pc, P, Q) == pytest.approx(math.sqrt(sse / 12), rel=1e-14)
+    assert orc.rmse(u, v, r, pr, pc, P, Q) == pytest.approx(0.2041938, abs=1e-7)
+
+
+def test_single_update_hand_computed(orc):
+    # Rating (0, 0, 5.0) of Fig. 1, p = (2.37, 0), q = (2.09, 0.69), lambda = 0.01.
+    # By hand: e = 5 - 2.37*2.09 = 0.0467.
+    #  gamma = 0.005: p0' = 2.37 + 0.005*(0.0467*2.09 - 0.01*2.37) = 2.370369515
+    #                 p1' = 0 + 0.005*(0.0467*0.69) = 0.000161115
+    #                 q0' = 2.09 + 0.005*(0.0467*2.37 - 0.01*2.09) = 2.090448895
+    #                 q1' = 0.69 + 0.005*(0 - 0.01*0.69) = 0.6899655
+    p, q = np.array([2.37, 0.0]), np.array([2.09, 0.69])
+    e = orc.sgd_update(0.005, 0.01, p, q, 5.0)
+    assert e == pytest.approx(0.0467, abs=1e-12)
+    assert p == pytest.approx([2.370369515, 0.000161115], abs=1e-12)
+    assert q == pytest.approx([2.090448895, 0.6899655], abs=1e-12)
+    # gamma = 0.1 separates the old-p reading (R1) from new-p:
+    #   q0' old-p = 2.09 + 0.1*(0.0467*2.37 - 0.0209)  = 2.0989779
+    #   q0' new-p = 2.09 + 0.1*(0.0467*2.3773903 - 0.0209) = 2.09901243...
+    p, q = np.array([2.37, 0.0]), np.array([2.09, 0.69])
+    orc.sgd_update(0.1, 0.01, p, q, 5.0)
+    assert p == pytest.approx([2.3773903, 0.0032223], abs=1e-12)
+    assert q == pytest.approx([2.0989779, 0.68931], abs=1e-12)
+    assert abs(q[0] - 2.0990124) > 3e-5
+
+
+def test_update_is_minus_gamma_finite_difference_gradient(orc):
+    # DESIGN.md R2: step = -gamma * grad f, f = 1/2[(r - p.q)^2 + lambda(|p|^2 + |q|^2)],
+    # gradient by central differences in numpy (independent of the oracle).
+    rng = np.random.default_rng(3)
+    for k in (1, 3, 8):
+        p0, q0 = rng.normal(size=k), rng.normal(size=k)
+        r, lam, gamma, h = 1.7, 0.3, 0.01, 1e-6
+
+        def f(p, q):
+            return 0.5 * ((r - p @ q) ** 2 + lam * (p @ p + q @ q))
+
+        gp = np.array([(f(p0 + h * np.eye(k)[j], q0) - f(p0 - h * np.eye(k)[j], q0)) / (2 * h) for j in range(k)])
+        gq = np.array([(f(p0, q0 + h * np.eye(k)[j]) - f(p0, q0 - h * np.eye(k)[j])) / (2 * h) for j in range(k)])
+        p, q = p0.copy(), q0.copy()
+        orc.sgd_update(gamma, lam, p, q, r)
+        np.testing.assert_allclose((p - p0) / -gamma, gp, rtol=1e-6, atol=1e-8)
+        np.testing.assert_allclose((q - q0) / -gamma, gq, rtol=1e-6, atol=1e-8)
+
+
+def test_fig1_end_to_end_epoch(orc):
+    # tests/golden/fig1_epoch.txt: partition, sort order, strata order and values.
+    g = golden_io.load("fig1_epoch.txt")
+    (u, v, r), P0, Q0, _ = golden_io.fig1()
+    pr = orc.perm(0, 1, 5)
+    S = orc.row_prefix(5, u, pr)
+    assert list(S) == [0, 3, 5, 8, 11, 12]
+    assert list(orc.bounds(5, 12, S, 2, [0.5, 0.5])) == [int(x) for x in g["bounds_G2"][0]]
+    for G, sec in ((1, "sorted_G1_B2"), (2, "sorted_G2_B2")):
+        prob = orc.Problem(5, 4, 2, 0.005, 0.01, u, v, r, G=G, Br=2, Bc=2, seed=0)
+        want = np.array(g[sec], dtype=np.int64)
+        assert np.array_equal(prob.ru, want[:, 3]) and np.array_equal(prob.rv, want[:, 4])
+        blk = ((want[:, 0] * 2 + want[:, 1]) * 2 + want[:, 2])
+        counts = np.bincount(blk, minlength=G * 4)
+        assert np.array_equal(np.diff(prob.off), counts)
+    prob = orc.Problem(5, 4, 2, 0.005, 0.01, u, v, r, G=1, Br=2, Bc=2, seed=0)
+    prob.set_factors(P0, Q0)
+    rm0 = prob.rmse(u, v, r)
+    prob.epoch("det", "none")
+    P1, Q1 = prob.factors()
+    np.testing.assert_allclose(P1, golden_io.matrix(g["P_after"]), atol=1e-10)
+    np.testing.assert_allclose(Q1, golden_io.matrix(g["Q_after"]), atol=1e-10)
+    assert [rm0, prob.rmse(u, v, r)] == pytest.approx(g["rmse"][0], abs=1e-10)
+
+
+# --------------------------------------------------- objective / convergence
+def _dense_objective(u, v, r, lam, P, Q, m, n):
+    # brute force: masked dense residual with a multiplicity mask (duplicates count)
+    M = np.zeros((m, n))
+    R = np.zeros((m, n))
+    np.add.at(M, (u, v), 1.0)
+    np.add.at(R, (u, v), r.astype(np.float64))
+    pred = P @ Q.T
+    # sum over Omega of (r - pq)^2 = sum_cells sum_dups (r_i - pred)^2
+    sq = np.zeros((m, n))
+    np.add.at(sq, (u, v), (r.astype(np.float64) - pred[u, v]) ** 2)
+    reg = lam * (M.sum(axis=1) @ (P * P).sum(axis=1) + M.sum(axis=0) @ (Q * Q).sum(axis=1))
+    return sq.sum() + reg
+
+
+def test_objective_matches_dense_bruteforce(orc):
+    import synth
+    m, n, k = 7, 6, 3
+    u, v, r = synth.tiny(m, n, 30, seed=5)
+    rng = np.random.default_rng(1)
+    P, Q = rng.normal(size=(m, k)), rng.normal(size=(n, k))
+    pr, pc = np.arange(m, dtype=np.int32), np.arange(n, dtype=np.int32)
+    got = orc.objective(u, v, r, 0.05, pr, pc, P, Q)
+    assert got == pytest.approx(_dense_objective(u, v, r, 0.05, P, Q, m, n), rel=1e-12)
+
+
+def test_monotone_loss_small_gamma(orc):
+    import synth
+    m, n, k = 20, 15, 4
+    u, v, r = synth.tiny(m, n, 120, seed=11, dup=False)
+    prob = orc.Problem(m, n, k, 1e-3, 0.01, u, v, r, G=1, Br=2, Bc=2, seed=9)
+    prob.init(4)
+    prev = None
+    for _ in range(30):
+        P, Q = prob.factors()
+        L = orc.objective(u, v, r, 0.01, np.arange(m, dtype=np.int32), np.arange(n, dtype=np.int32), P, Q)
+        if prev is not None:
+            assert L < prev
+        prev = L
+        prob.epoch("det", "none")
+
+
+def test_planted_recovery(orc):
+    # noise-free rank-4 60 x 40 at 50% density, lambda = 0: train RMSE -> 0
+    rng = np.random.default_rng(2)
+    m, n, k = 60, 40, 4
+    Ps, Qs = rng.uniform(0, 1, (m, k)), rng.uniform(0, 1, (n, k))
+    cells = rng.choice(m * n, size=m * n // 2, replace=False)
+    u, v = (cells // n).astype(np.int32), (cells % n).astype(np.int32)
+    r = np.sum(Ps[u] * Qs[v], axis=1).astype(np.float32)
+    prob = orc.Problem(m, n, k, 0.05, 0.0, u, v, r, G=1, Br=1, Bc=1, seed=3)
+    prob.init(1)
+    first = prob.rmse(u, v, r)
+    for _ in range(200):
+        prob.epoch("det", "none")
+    assert first > 0.3
+    assert prob.rmse(u, v, r) < 2e-3
+
+
+def _gd_step(u, v, r, lam, P, Q, gp, gq):
+    # one full-batch gradient step on L/2 (R2, R4): frequency-weighted reg
+    E = r.astype(np.float64) - np.sum(P[u] * Q[v], axis=1)
+    dP = np.zeros_like(P)
+    dQ = np.zeros_like(Q)
+    np.add.at(dP, u, E[:, None] * Q[v] - lam * P[u])
+    np.add.at(dQ, v, E[:, None] * P[u] - lam * Q[v])
+    return P + gp * dP, Q + gq * dQ
+
+
+@pytest.mark.parametrize("sched,sync,G,Br,Bc", [
+    ("det", "none", 1, 3, 3), ("serial", "none", 1, 2, 5), ("det", "ring", 2, 2, 4),
+    ("serial", "ring", 3, 1, 3), ("det", "allreduce", 2, 2, 2), ("serial", "allreduce", 3, 1, 1),
+])
+def test_full_batch_limit(orc, sched, sync, G, Br, Bc):
+    # Any serialisation that visits every rating exactly once differs from one
+    # full-batch GD step by O(gamma^2): halving gamma quarters the gap.  For the
+    # all-reduce mode the Q step is the mean of G replicas, so its first-order
+    # term is the GD Q-step divided by G (L549-L557 sync = average).  A dropped
+    # or doubled block, a wrong-sign term, or a wrong average fails this.
+    import synth
+    m, n, k = 9, 7, 3
+    u, v, r = synth.tiny(m, n, 40, seed=21)
+    rng = np.random.default_rng(4)
+    P0, Q0 = rng.uniform(0, 1, (m, k)), rng.uniform(0, 1, (n, k))
+    gaps = []
+    for gamma in (1e-2, 5e-3, 2.5e-3):
+        prob = orc.Problem(m, n, k, gamma, 0.1, u, v, r, G=G, Br=Br, Bc=Bc, seed=13)
+        prob.set_factors(P0, Q0)
+        prob.epoch(sched, sync)
+        P1, Q1 = prob.factors()
+        gq = gamma / G if sync == "allreduce" else gamma
+        Pg, Qg = _gd_step(u, v, r, 0.1, P0, Q0, gamma, gq)
+        first = max(np.abs(P1 - P0).max(), np.abs(Q1 - Q0).max())
+        gap = max(np.abs(P1 - Pg).max(), np.abs(Q1 - Qg).max())
+        assert gap < 0.2 * first
+        gaps.append(gap)
+    assert 0.2 < gaps[1] / gaps[0] < 0.3 and 0.2 < gaps[2] / gaps[1] < 0.3
+
+
+def test_allreduce_g1_equals_none_and_ring_g1_equals_none(orc):
+    import synth
+    m, n, k = 8, 6, 4
+    u, v, r = synth.tiny(m, n, 30, seed=8)
+    outs = []
+    for sync in ("none", "ring", "allreduce"):
+        prob = orc.Problem(m, n, k, 0.05, 0.02, u, v, r, G=1, Br=3, Bc=3, seed=2)
+        prob.init(6)
+        prob.epoch("det", sync)
+        outs.append(prob.factors())
+    for P, Q in outs[1:]:
+        assert np.array_equal(P, outs[0][0]) and np.array_equal(Q, outs[0][1])
+
+
+def test_init_range_and_scale(orc):
+    m, n, k = 300, 200, 16
+    P, Q = orc.init(5, m, n, k, np.arange(m, dtype=np.int32), np.arange(n, dtype=np.int32))
+    for X in (P, Q):
+        assert X.min() >= 0.0 and X.max() < math.sqrt(1.0 / k)
+        assert X.mean() == pytest.approx(0.5 * math.sqrt(1.0 / k), rel=0.02)
+        # 24-bit grid: every value is an integer multiple of 2^-24 * sqrt(1/k)
+        q = X / (math.sqrt(1.0 / k) * 2.0 ** -24)
+        assert np.allclose(q, np.rint(q), atol=1e-6)
+    # permuted storage: perm_row maps original id -> stored row
+    pr = orc.perm(3, 1, m)
+    P2, _ = orc.init(5, m, n, k, pr, np.arange(n, dtype=np.int32))
+    assert np.array_equal(P2[pr], P)
