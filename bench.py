@@ -1,0 +1,347 @@
+#!/usr/bin/env python
+"""bench.py -- rating updates/s of the HCC-MF hot path on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--sched hogwild]
+    torchrun --nproc-per-node N bench.py --gpus N ...         (one rank per GPU, NCCL)
+    python bench.py --impl reference ...                       (the oracle arm, host cores)
+
+A "step" is one training epoch over every rating of the workload, the per-epoch
+hot path of the paper's workflow (L549-L557): the SGD kernel over all nnz
+(a5/a6), the Q synchronisation across GPUs (a7, G > 1) and the RMSE evaluation
+of the held-out test set (a8, Fig. 7).  Preprocessing (a1-a4) happens once
+before training, as in the paper (steps 1-3, L543-L548); the `e2e` object times
+the WHOLE job through the public API from host buffers (ingest + shuffle +
+partition + sort + init + epochs + RMSE + export), H2D/D2H inside the timed
+region.  value = nnz * steps / device time (Eq. 8 "computing power", L1709-L1715),
+max over ranks.  Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import synth  # noqa: E402
+
+METRIC = "rating updates/sec (whole box)"
+UNIT = "updates/s"
+FALLBACK_HBM_GBS = 6650.0
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c3", choices=sorted(synth.CONFIGS))
+    ap.add_argument("--sched", default="hogwild", choices=["hogwild", "det"])
+    ap.add_argument("--sync", default=None, choices=["none", "ring", "allreduce"])
+    ap.add_argument("--grid", default=None, help="Br,Bc (default: hogwild 1,G ; det 64,64*G)")
+    ap.add_argument("--warps", type=int, default=0)
+    ap.add_argument("--task", type=int, default=0)
+    ap.add_argument("--impl", default="hccmf", choices=["hccmf", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ helpers
+class Clocks:
+    """nvidia-smi sampler for the timed region (B200_PROFILING.md clocks line)."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index, self.rows, self.proc = index, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        self.proc.wait(timeout=5)
+        self.t.join(timeout=2)
+        sm = [float(r[0]) for r in self.rows if len(r) >= 8 and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) >= 8 and r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows if len(r) >= 8 for i in range(4) if r[4 + i] == "Active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(sm)}
+
+
+def hbm_peak():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic(cfg_name, sched):
+    """DRAM bytes per launch of the SGD kernel from the committed ncu --set full summary, if any."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(p) as f:
+            return json.load(f).get(f"{cfg_name}/{sched}")
+    except Exception:
+        return None
+
+
+def host_cpu():
+    model = "unknown"
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return model, os.cpu_count()
+
+
+def oracle_sample(cfg, u, v, r, seconds):
+    """The oracle, as it stands, on a bounded prefix sample of the same workload (1 host core)."""
+    import oracle
+    S = int(min(len(u), 2_000_000 if cfg.k >= 64 else 8_000_000))
+    prob = oracle.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u[:S], v[:S], r[:S], G=1, Br=1, Bc=1,
+                          seed=cfg.seed)
+    prob.init(1)
+    t0 = time.perf_counter()
+    epochs = 0
+    while True:
+        prob.epoch("serial", "none")
+        epochs += 1
+        if time.perf_counter() - t0 >= seconds:
+            break
+    dt = time.perf_counter() - t0
+    return S * epochs / dt, S, epochs, dt
+
+
+# ------------------------------------------------------------ reference arm
+def run_reference(args, cfg, rank, world):
+    if rank != 0:
+        return
+    (u, v, r), _ = synth.make(cfg, n_test=1)
+    import oracle
+    S = int(min(len(u), 1_000_000 if cfg.k >= 64 else 4_000_000))
+    prob = oracle.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u[:S], v[:S], r[:S], seed=cfg.seed)
+    prob.init(1)
+    for _ in range(args.warmup):
+        prob.epoch("serial", "none")
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        prob.epoch("serial", "none")
+    dt = time.perf_counter() - t0
+    val = S * args.steps / dt
+    model, ncpu = host_cpu()
+    sample = (f"serial oracle epoch over the first {S} ratings of the {cfg.name} stream (k={cfg.k}) per step; "
+              f"1 of {ncpu} host cores ({model})")
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": cfg.name, "m": cfg.m, "n": cfg.n, "nnz": cfg.nnz, "k": cfg.k},
+        "cpu_baseline": {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+# --------------------------------------------------------------- main arm
+def main():
+    args = parse()
+    cfg = synth.CONFIGS[args.config]
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    if args.impl == "reference":
+        run_reference(args, cfg, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icpp_huangylhbl21_b200 as hc
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    G = world
+    sync = args.sync or ("none" if G == 1 else "ring")
+    if args.grid:
+        Br, Bc = (int(x) for x in args.grid.split(","))
+    elif args.sched == "hogwild":
+        Br, Bc = 1, (G if sync == "ring" else 1)
+    else:
+        Br, Bc = 64, 64 * (G if sync == "ring" else 1)
+
+    t_gen = time.perf_counter()
+    (u, v, r), (tu, tv, tr) = synth.make(cfg)
+    t_gen = time.perf_counter() - t_gen
+    nnz, nt = len(u), len(tu)
+
+    stream = torch.cuda.Stream()
+    mdl = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, dist=world > 1, device=local)
+    mdl.set_stream(stream)
+    if args.warps:
+        mdl.set_option("hogwild_warps", args.warps)
+    if args.task:
+        mdl.set_option("task_ratings", args.task)
+    du, dv, dr = (torch.from_numpy(x).cuda() for x in (u, v, r))
+    dtu, dtv, dtr = (torch.from_numpy(x).cuda() for x in (tu, tv, tr))
+    torch.cuda.synchronize()
+    t_prep = time.perf_counter()
+    mdl.load(du, dv, dr)
+    mdl.partition(G, (Br, Bc), "DP0", seed=cfg.seed)
+    mdl.init(1)
+    t_prep = time.perf_counter() - t_prep
+    info = mdl.info()
+    del du, dv, dr
+    rm0 = mdl.rmse(dtu, dtv, dtr)
+    mdl.set_option("sync_stream", 0)
+
+    def step(ev=None):
+        if ev is not None:
+            ev[0].record(stream)
+        mdl.train_epoch(args.sched, sync)
+        if ev is not None:
+            ev[1].record(stream)
+        return mdl.rmse(dtu, dtv, dtr)
+
+    for _ in range(args.warmup):
+        step()
+    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    clocks = Clocks(local)
+    clocks.start()
+    time.sleep(0.3)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_start.record(stream)
+    rms = [step(kev[i]) for i in range(args.steps)]
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    ms = t_start.elapsed_time(t_end)
+    k_ms = [a.elapsed_time(b) for a, b in kev]
+    if world > 1:
+        t = torch.tensor([ms, float(np.mean(k_ms))], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms, kmean = t.tolist()
+    else:
+        kmean = float(np.mean(k_ms))
+    value = nnz * args.steps / (ms / 1e3)
+
+    # roofline of the dominant kernel (the SGD epoch): north_star bytes/update = 12 + 16k
+    peak, peak_src = hbm_peak()
+    b_upd = 12 + 16 * cfg.k
+    local_nnz = info["local_nnz"]
+    achieved = local_nnz * b_upd / (kmean / 1e3) / 1e9
+    traffic = ncu_traffic(args.config, args.sched)
+    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+            "traffic": traffic, "kernel": "sgd_kernel (a5/a6 epoch incl. Q sync)", "bytes_per_update": b_upd,
+            "updates_per_launch": local_nnz, "kernel_ms": kmean, "kernel_share_of_step": kmean / (ms / args.steps),
+            "peak_source": peak_src}
+
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+           "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+           "config": {"workload": f"{cfg.name} ({args.config})", "m": cfg.m, "n": cfg.n, "nnz": nnz, "k": cfg.k,
+                      "test_ratings": nt, "gamma": cfg.gamma, "lambda": cfg.lam, "sched": args.sched,
+                      "sync": sync, "grid": [Br, Bc], "parallelism": f"dp{world} (row shards, Q {sync})",
+                      "step": "1 SGD epoch over all nnz + Q sync + test RMSE",
+                      "l2": "inputs larger than L2 (records %.2f GB > 126 MB); Q is L2-resident by design"
+                            % (12 * nnz / 1e9),
+                      "hogwild_tasks": info["n_tasks"], "key_bits": info["key_bits"]},
+           "roofline": roof, "clocks": clk,
+           "gpu_launches": args.steps * ((Bc if args.sched == "hogwild" else Br) * (G if sync == "ring" else 1)
+                                         + 3),
+           "rmse": {"test_initial": rm0, "test_after_warmup_plus_timed": rms[-1],
+                    "epochs": args.warmup + args.steps},
+           "prep_s": t_prep, "gen_s": t_gen,
+           "paper_context": {"netflix_hcc_updates_per_s": 2228476993,
+                             "hardware": "2x Xeon Gold 6242 + RTX 2080 + RTX 2080S (Table 4, L2001)"}}
+
+    # ---- e2e: the whole job through the public API from pinned host buffers
+    if not args.no_e2e:
+        pin = [torch.from_numpy(x).pin_memory() for x in (u, v, r, tu, tv, tr)]
+        Ph = torch.empty((cfg.m, cfg.k), dtype=torch.float32).pin_memory()
+        Qh = torch.empty((cfg.n, cfg.k), dtype=torch.float32).pin_memory()
+        E = cfg.epochs
+
+        def job():
+            m2 = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, dist=world > 1, device=local)
+            m2.set_stream(stream)
+            if args.warps:
+                m2.set_option("hogwild_warps", args.warps)
+            m2.load(pin[0], pin[1], pin[2])
+            m2.partition(G, (Br, Bc), "DP0", seed=cfg.seed)
+            m2.init(1)
+            for _ in range(E):
+                m2.train_epoch(args.sched, sync)
+                m2.rmse(pin[3], pin[4], pin[5])
+            m2.factors(Ph, Qh)
+            m2.close()
+
+        job()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        reps = 2
+        t0 = time.perf_counter()
+        for _ in range(reps):
+            job()
+        torch.cuda.synchronize()
+        e2e_s = (time.perf_counter() - t0) / reps
+        if world > 1:
+            t = torch.tensor([e2e_s], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_s = t.item()
+        out["e2e"] = {"value": nnz * E / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 12 * (nnz + nt),
+                      "d2h_bytes_per_step": 4 * (cfg.m + cfg.n) * cfg.k + 8 * (E + 0),
+                      "step": f"job: load+partition+init+{E} epochs (each with test RMSE)+export P,Q; "
+                              "host pinned buffers", "s_per_step": e2e_s}
+
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        val, S, ep, dt = oracle_sample(cfg, u, v, r, args.cpu_seconds)
+        model, ncpu = host_cpu()
+        out["cpu_baseline"] = {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
+                               "sample": f"{ep} serial fp64 oracle epoch(s) over the first {S} ratings of the "
+                                         f"same stream, {dt:.1f} s on 1 of {ncpu} cores ({model})"}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    mdl.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,221 @@
+/*
+ * hccmf.h -- C ABI of libhccmf, the B200-native hot path of HCC-MF
+ * (Huang, Yin, Liu, He, Bai, Li: "A Novel Multi-CPU/GPU Collaborative Computing
+ * Framework for SGD-based Matrix Factorization", ICPP '21).
+ *
+ * Citations: L<n> = line n of the paper text.
+ * lists every reading taken where the paper is silent or garbled (R1..R20).
+ *
+ * What the library computes:
+ *   a0 factor init, a1 ingest+validate COO, a2 seeded ID shuffle, a3 row-grid
+ *   partition (DP0/DP1/DP2), a4 blocking + stable sort, a5 deterministic SGD
+ *   epoch, a6 Hogwild SGD epoch, a7 Q synchronisation across shards, a8 RMSE,
+ *   a9 export.
+ *
+ * Conventions (all entry points):
+ *  - extern "C", plain pointers and sizes; no C++ types or exceptions cross it.
+ *  - Every call returns hccmf_status; details in hccmf_last_error(h).  CUDA and
+ *    NCCL failures are sticky: after one, every call on the handle returns the
+ *    same code.
+ *  - Indices are 0-based.  u in [0, m), v in [0, n).
+ *  - Factor layout: P is m x k row-major fp32 (p_u contiguous); Q is n x k
+ *    row-major fp32 (q_v contiguous) -- this is the paper's k x n item matrix Q
+ *    (Table 1) TRANSPOSED.
+ *  - Input pointers may be host or device memory (classified with
+ *    cudaPointerGetAttributes).  The library COPIES inputs; the caller keeps
+ *    ownership and may free them when the call returns.  Output pointers are
+ *    caller-allocated, host or device.  The handle owns all device memory it
+ *    allocates; hccmf_destroy frees it.
+ *  - Call order: create -> load_ratings -> partition -> (init_factors |
+ *    set_factors) -> { train_epoch | rmse | get_factors }*.  Out of order:
+ *    HCCMF_ESTATE.
+ *  - All work is issued on the handle's CUDA stream (its own, or the one given
+ *    to hccmf_set_stream); every call returns after that stream is synchronised
+ *    unless stated otherwise, so host timing around a call is meaningful.
+ *  - Not thread-safe per handle; distinct handles are independent.
+ *  - There is no CPU fallback: without a CUDA device every call that needs one
+ *    returns HCCMF_ECUDA.
+ */
+#ifndef HCCMF_H_
+#define HCCMF_H_
+
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define HCCMF_API __attribute__((visibility("default")))
+#else
+#define HCCMF_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct hccmf_ctx* hccmf_t;
+
+typedef enum {
+    HCCMF_OK = 0,
+    HCCMF_EINVAL = -1, /* bad argument (sizes, k, gamma, grid, NULL)         */
+    HCCMF_ERANGE = -2, /* rating index out of range, non-finite r, overflow  */
+    HCCMF_ENOMEM = -3, /* device allocation failed                           */
+    HCCMF_ESTATE = -4, /* call out of order                                  */
+    HCCMF_ECUDA = -5,  /* CUDA runtime error / no device (sticky)            */
+    HCCMF_ENCCL = -6   /* NCCL error (sticky)                                */
+} hccmf_status;
+
+/* a5 / a6: the SGD schedule inside a shard.
+ * DET: FPSGD-style conflict-free strata of independent blocks in a fixed order
+ *      (PAPER.md L93-L97, L2269-L2275); the result equals the oracle's serial
+ *      run of the same order up to fp32 rounding.
+ * HOGWILD: lock-free racing updates over user-aligned tasks (Hogwild!, L216-L219,
+ *      L1680-L1691).  Non-deterministic by design. */
+typedef enum { HCCMF_SCHED_DET = 0, HCCMF_SCHED_HOGWILD = 1 } hccmf_sched;
+
+/* a7: how shards exchange Q (only Q moves: Strategy 1, L1203-L1233).
+ * NONE: one shard.  RING: rotating column groups of Q, stage t shard s updates
+ *      group (s+t) mod G and passes it to shard s-1 (hidden synchronisation,
+ *      L1143-L1172; async computing-transmission, L1251-L1269).
+ * ALLREDUCE_AVG: every shard trains against its own replica of Q, then
+ *      Q = mean_s Q_s (the server's multiply-add sync, L549-L557, L783-L784). */
+typedef enum { HCCMF_SYNC_NONE = 0, HCCMF_SYNC_RING = 1, HCCMF_SYNC_ALLREDUCE_AVG = 2 } hccmf_sync;
+
+/* a3: data partition strategy (section 3.3).
+ * DP0: Eq. 6 (L967-L981) from t_meas if given, else equal shares x_s = 1/G.
+ * DP1: Algorithm 1 compensation (L1025-L1142), needs t_meas (R11).
+ * DP2: Eq. 7 hidden-synchronisation ramp (L1143-L1172), needs t_meas, t_sync. */
+typedef enum { HCCMF_DP0 = 0, HCCMF_DP1 = 1, HCCMF_DP2 = 2 } hccmf_dp;
+
+typedef struct {
+    int32_t n_shards;     /* G >= 1.  Distributed handle: must equal world size.
+                             Single-process handle: G > 1 runs G LOGICAL shards on
+                             the one device (exactly the multi-GPU schedule). */
+    int32_t grid_rows;    /* B_r >= 1 row blocks per shard                         */
+    int32_t grid_cols;    /* B_c >= 1 column blocks over all n columns.  DET needs
+                             B_r == B_c (NONE, ALLREDUCE) or B_c == G*B_r (RING);
+                             HOGWILD+RING needs B_c % G == 0.                      */
+    int32_t strategy;     /* hccmf_dp                                               */
+    const double* x;      /* optional [G] starting fractions of nnz, sum 1 (DP1/2) */
+    const double* t_meas; /* optional [G] measured compute time per shard, s       */
+    double t_sync;        /* DP2: per-shard sync time, s                            */
+    uint64_t seed;        /* a2 ID shuffle seed; 0 = identity permutation          */
+    int32_t storage;      /* 0 = fp32 factors (the only value accepted this round) */
+} hccmf_partition_opts;
+
+typedef struct {
+    int64_t m, n, nnz;       /* problem (nnz = ratings loaded, all shards)        */
+    int32_t k;
+    int32_t n_shards;        /* G                                                 */
+    int32_t shard_lo;        /* first shard held by this handle                   */
+    int32_t shard_hi;        /* one past the last shard held                      */
+    int64_t local_nnz;       /* ratings held by this handle                       */
+    int64_t row0, rows;      /* permuted row range [row0, row0+rows) of local P   */
+    int64_t n_blocks;        /* G * B_r * B_c                                     */
+    int64_t n_tasks;         /* Hogwild tasks (user-aligned runs) held locally    */
+    int32_t key_bits;        /* bits of the a4 sort key                           */
+    int32_t rank, world;     /* 0, 1 for a single-process handle                  */
+    int64_t device_bytes;    /* device memory currently owned by the handle       */
+} hccmf_info;
+
+/* Tunables for hccmf_set_option (values are int64). */
+typedef enum {
+    HCCMF_OPT_HOGWILD_WARPS = 1, /* concurrent warps of the Hogwild kernel; 0 = auto
+                                    (R14)                               */
+    HCCMF_OPT_TASK_RATINGS = 2,  /* target ratings per Hogwild task (>= 1, default
+                                    256); tasks never split a user's run          */
+    HCCMF_OPT_SYNC_STREAM = 3,   /* 1 (default): calls return after the stream is
+                                    synchronised; 0: return after enqueueing      */
+    HCCMF_OPT_RING_SUBBLOCKS = 4 /* reserved                                       */
+} hccmf_option;
+
+/* ------------------------------------------------------------------ lifecycle */
+
+/* Create a single-process handle on the current CUDA device.
+ * m, n in [1, 2^31); k multiple of 4 in [4, 512]; gamma > 0 finite (learning
+ * rate, Table 3); lambda >= 0 finite (L2 weight lambda_1 = lambda_2,
+ * Table 3).  *out receives the handle. */
+HCCMF_API hccmf_status hccmf_create(int64_t m, int64_t n, int32_t k, float gamma, float lambda, hccmf_t* out);
+
+/* Write an NCCL unique id (128 bytes) into out[128]; rank 0 calls it and
+ * broadcasts the bytes with torch.distributed before hccmf_create_dist. */
+HCCMF_API hccmf_status hccmf_nccl_unique_id(void* out128);
+
+/* Create a distributed handle: one process per GPU, rank in [0, world), on CUDA
+ * device `device`.  Collective: all ranks must call it with the same id. */
+HCCMF_API hccmf_status hccmf_create_dist(int64_t m, int64_t n, int32_t k, float gamma, float lambda,
+                               const void* nccl_unique_id, int32_t rank, int32_t world,
+                               int32_t device, hccmf_t* out);
+
+/* Issue all further work on `stream` (a cudaStream_t, may be the legacy default
+ * 0).  The caller keeps ownership of the stream and must keep it alive. */
+HCCMF_API hccmf_status hccmf_set_stream(hccmf_t h, void* stream);
+
+HCCMF_API hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value);
+
+/* Release all device memory and the NCCL communicator.  NULL is a no-op. */
+HCCMF_API void hccmf_destroy(hccmf_t h);
+
+/* Last error message of the handle ("" if none); h == NULL -> last global error. */
+HCCMF_API const char* hccmf_last_error(hccmf_t h);
+
+/* ---------------------------------------------------------------- the path */
+
+/* a1 (preprocessing, L543-L548): copy nnz >= 0 COO ratings (u[i], v[i], r[i])
+ * of R (Table 1).  Duplicated (u, v) are kept, each one update.
+ * Validates 0 <= u < m, 0 <= v < n and finite r -> HCCMF_ERANGE otherwise.
+ * Distributed handles: every rank passes the same global COO. */
+HCCMF_API hccmf_status hccmf_load_ratings(hccmf_t h, const int32_t* u, const int32_t* v, const float* r, int64_t nnz);
+
+/* a2-a4: shuffle (seeded permutation of row and column ids), row-grid partition
+ * into G shards of contiguous permuted rows balanced on nnz (DP0/1/2,
+ * L881-L1172), blocking into G*B_r*B_c blocks and a stable sort by
+ * (shard, row block, column block, u', v') -- the row-sorted blocks of
+ * L1472-L1474.  Bit-exact with the oracle.  Collective for distributed handles. */
+HCCMF_API hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* opts);
+
+/* a0: P[u][j] = U(H(seed,3,u,j)) * sqrtf(1/k), Q[v][j] = U(H(seed,4,v,j)) * sqrtf(1/k)
+ * on ORIGINAL ids (R5); H is the SplitMix64-based hash of DESIGN.md R8. */
+HCCMF_API hccmf_status hccmf_init_factors(hccmf_t h, uint64_t seed);
+
+/* Set P (m x k) and Q (n x k) in ORIGINAL id order (checkpoint restore, tests).
+ * Distributed handles: every rank passes the full matrices. */
+HCCMF_API hccmf_status hccmf_set_factors(hccmf_t h, const float* P, const float* Q);
+
+/* a5/a6 + a7: one epoch over every held rating:
+ *   e = r - p_u.q_v;  p_u += gamma (e q_v - lambda p_u);  q_v += gamma (e p_u - lambda q_v)
+ * (section 2.1; Fig. 1; p_u on the right is the pre-update value, R1),
+ * in the given schedule, followed (G > 1) by the given Q synchronisation. */
+HCCMF_API hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync);
+
+/* a8: sqrt( sum_T (r - p_u.q_v)^2 / |T| ) over nt test ratings in ORIGINAL ids
+ * (Fig. 1 caption L405-L407, Fig. 7).  fp32 dot products, fp64 accumulation in a
+ * fixed order (deterministic).  Distributed: all-reduced over ranks, collective. */
+HCCMF_API hccmf_status hccmf_rmse(hccmf_t h, const int32_t* u, const int32_t* v, const float* r, int64_t nt, double* out);
+
+/* a9 (final push, L1205-L1206): P (m x k) and/or Q (n x k) in ORIGINAL id order;
+ * either pointer may be NULL.  Distributed: collective; every rank gets the full
+ * matrices. */
+HCCMF_API hccmf_status hccmf_get_factors(hccmf_t h, float* P, float* Q);
+
+/* Partition introspection (bit-exact parity tests).  Any pointer may be NULL.
+ * bounds[G+1] (int32 permuted-row boundaries b_s), block_off[G*B_r*B_c+1]
+ * (int64, first record of each block in the global sorted order), perm_row[m],
+ * perm_col[n] (int32, original id -> permuted id). */
+HCCMF_API hccmf_status hccmf_get_partition(hccmf_t h, int32_t* bounds, int64_t* block_off, int32_t* perm_row,
+                                 int32_t* perm_col);
+
+/* Sorted records held by this handle (local_nnz of them, permuted ids).
+ * Any pointer may be NULL. */
+HCCMF_API hccmf_status hccmf_get_records(hccmf_t h, int32_t* u, int32_t* v, float* r);
+
+/* Partition fractions x[G] actually used (after DP0/1/2). */
+HCCMF_API hccmf_status hccmf_get_fractions(hccmf_t h, double* x);
+
+HCCMF_API hccmf_status hccmf_get_info(hccmf_t h, hccmf_info* out);
+
+/* Library version string, e.g. "hccmf 0.1 sm_100a". */
+HCCMF_API const char* hccmf_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* HCCMF_H_ */

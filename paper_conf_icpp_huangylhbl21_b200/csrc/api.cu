@@ -1,0 +1,875 @@
+// api.cu -- the C ABI (include/hccmf.h) and the host runtime around the kernels:
+// argument checks, device memory, the partition planner (DP0/DP1/DP2), SGD
+// launch plans for every (schedule, sync) pair, the ring / all-reduce Q
+// synchronisation over NCCL, and export.
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+
+#include "internal.cuh"
+
+using namespace hccmf;
+
+namespace {
+
+thread_local std::string g_err;
+
+hccmf_status fail(hccmf_t h, hccmf_status st, const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  if (h) {
+    h->err = buf;
+    if (st == HCCMF_ECUDA || st == HCCMF_ENCCL) h->sticky = st;
+  }
+  g_err = buf;
+  return st;
+}
+
+#define CU(h, call)                                                                                   \
+  do {                                                                                                \
+    cudaError_t e_ = (call);                                                                          \
+    if (e_ != cudaSuccess) {                                                                          \
+      if (e_ == cudaErrorMemoryAllocation) {                                                          \
+        cudaGetLastError();                                                                           \
+        return fail(h, HCCMF_ENOMEM, "%s: out of device memory (%s:%d)", #call, __FILE__, __LINE__);  \
+      }                                                                                               \
+      return fail(h, HCCMF_ECUDA, "%s: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    }                                                                                                 \
+  } while (0)
+
+#define NC(h, call)                                                                                            \
+  do {                                                                                                         \
+    ncclResult_t r_ = (call);                                                                                  \
+    if (r_ != ncclSuccess)                                                                                     \
+      return fail(h, HCCMF_ENCCL, "%s: %s (%s:%d)", #call, ncclGetErrorString(r_), __FILE__, __LINE__);       \
+  } while (0)
+
+#define ENTER(h)                                      \
+  do {                                                \
+    if (!(h)) return fail(nullptr, HCCMF_EINVAL, "NULL handle"); \
+    if ((h)->sticky != HCCMF_OK) return (h)->sticky;  \
+    CU(h, cudaSetDevice((h)->device));                \
+  } while (0)
+
+template <typename T>
+cudaError_t dmalloc(hccmf_t h, T** p, size_t count) {
+  const size_t bytes = sizeof(T) * (count ? count : 1);
+  cudaError_t e = cudaMalloc((void**)p, bytes);
+  if (e == cudaSuccess) h->device_bytes += bytes;
+  return e;
+}
+template <typename T>
+void dfree(hccmf_t h, T*& p, size_t count) {
+  if (p) {
+    cudaFree((void*)p);
+    h->device_bytes -= sizeof(T) * (count ? count : 1);
+  }
+  p = nullptr;
+}
+
+hccmf_status finish(hccmf_t h) {
+  CU(h, cudaGetLastError());
+  if (h->sync_stream) CU(h, cudaStreamSynchronize(h->stream));
+  return HCCMF_OK;
+}
+
+int bitlen(uint64_t x) {  // bits needed to represent x (0 -> 0)
+  int b = 0;
+  while (x) { ++b; x >>= 1; }
+  return b;
+}
+
+int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+hccmf_status check_problem(int64_t m, int64_t n, int32_t k, float gamma, float lambda) {
+  if (m < 1 || m >= (1LL << 31) || n < 1 || n >= (1LL << 31))
+    return fail(nullptr, HCCMF_EINVAL, "m, n must be in [1, 2^31)");
+  if (k < 4 || k > 512 || k % 4 != 0) return fail(nullptr, HCCMF_EINVAL, "k must be a multiple of 4 in [4, 512]");
+  if (!(gamma > 0.f) || !std::isfinite(gamma)) return fail(nullptr, HCCMF_EINVAL, "gamma must be finite and > 0");
+  if (!(lambda >= 0.f) || !std::isfinite(lambda)) return fail(nullptr, HCCMF_EINVAL, "lambda must be finite and >= 0");
+  return HCCMF_OK;
+}
+
+hccmf_status make_ctx(int64_t m, int64_t n, int32_t k, float gamma, float lambda, int device, hccmf_t* out) {
+  hccmf_t h = new hccmf_ctx();
+  h->m = m;
+  h->n = n;
+  h->k = k;
+  h->gamma = gamma;
+  h->lambda = lambda;
+  h->device = device;
+  cudaError_t e = cudaSetDevice(device);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking);
+  if (e != cudaSuccess) {
+    hccmf_status st = fail(nullptr, HCCMF_ECUDA, "no usable CUDA device: %s", cudaGetErrorString(e));
+    cudaGetLastError();
+    delete h;
+    return st;
+  }
+  h->own_stream = true;
+  *out = h;
+  return HCCMF_OK;
+}
+
+// ----------------------------------------------------------- DP planners
+// Independent host implementation of section 3.3 (the oracle has its own).
+void plan_dp0(int G, const double* t, std::vector<double>& x) {  // Eq. 6
+  x.assign(G, 0.0);
+  for (int i = 0; i < G; ++i) {
+    double s = 0.0;
+    for (int j = 0; j < G; ++j) s += t[i] / t[j];
+    x[i] = 1.0 / s;
+  }
+}
+
+void plan_dp1(int G, std::vector<double>& x, std::vector<double> t) {  // Alg. 1, R11
+  for (int it = 0; it < 8; ++it) {
+    double tbar = 0.0, tmin = t[0], dev = 0.0;
+    for (int s = 0; s < G; ++s) tbar += t[s];
+    tbar /= (double)G;
+    for (int s = 0; s < G; ++s) {
+      tmin = std::min(tmin, t[s]);
+      dev = std::max(dev, std::fabs(t[s] - tbar));
+    }
+    if (dev / tmin <= 0.1) break;
+    double sum = 0.0;
+    for (int s = 0; s < G; ++s) sum += x[s] * tbar / t[s];
+    for (int s = 0; s < G; ++s) {
+      const double xn = (x[s] * tbar / t[s]) / sum;
+      t[s] = t[s] * xn / x[s];
+      x[s] = xn;
+    }
+  }
+}
+
+void plan_dp2(int G, std::vector<double>& x, const double* t, double t_sync) {  // Eq. 7, R12
+  const int smed = (G - 1) / 2;
+  const double tmed = t[smed];
+  double sum = 0.0;
+  std::vector<double> y(G);
+  for (int s = 0; s < G; ++s) {
+    double Ts = tmed + (double)(s - smed) * t_sync;
+    if (Ts < 0.0) Ts = 0.0;
+    y[s] = x[s] * Ts / t[s];
+    sum += y[s];
+  }
+  for (int s = 0; s < G; ++s) x[s] = y[s] / sum;
+}
+
+// first column of column block cb
+int64_t col_start(const hccmf_t h, int64_t cb) { return ceil_div(cb * h->n, h->Bc); }
+
+int64_t blk_index(const hccmf_t h, int64_t s, int64_t rb, int64_t cb) { return (s * h->Br + rb) * h->Bc + cb; }
+
+void free_partition(hccmf_t h) {
+  for (auto& p : h->plans) {
+    dfree(h, p.d_lo, p.n_tasks);
+    dfree(h, p.d_hi, p.n_tasks);
+  }
+  h->plans.clear();
+  dfree(h, h->d_task_lo, h->n_tasks);
+  dfree(h, h->d_task_hi, h->n_tasks);
+  h->n_tasks = 0;
+  dfree(h, h->d_u, h->local_nnz);
+  dfree(h, h->d_v, h->local_nnz);
+  dfree(h, h->d_r, h->local_nnz);
+  dfree(h, h->d_perm_row, h->m);
+  dfree(h, h->d_perm_col, h->n);
+  dfree(h, h->d_P, h->rows * h->k);
+  dfree(h, h->d_Q, h->n * h->k);
+  dfree(h, h->d_Qrep, (size_t)h->n * h->k * (h->shard_hi - h->shard_lo));
+  dfree(h, h->d_counters, h->n_counters);
+  h->n_counters = 0;
+  h->local_nnz = 0;
+  h->rows = 0;
+  h->blk_task_off.clear();
+  h->h_task_lo.clear();
+  h->h_task_hi.clear();
+}
+
+// ------------------------------------------------------------ SGD plans
+hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
+  for (auto& p : h->plans)
+    if (p.sched == sched && p.sync == sync) {
+      *out = &p;
+      return HCCMF_OK;
+    }
+  const int G = h->G, Br = h->Br, Bc = h->Bc;
+  Plan pl;
+  pl.sched = sched;
+  pl.sync = sync;
+  std::vector<int64_t> lo, hi;
+  auto local_off = [&](int64_t blk) { return h->block_off[blk] - h->rec0; };
+  auto add_block_det = [&](int64_t blk) {
+    const int64_t a = local_off(blk), b = local_off(blk + 1);
+    if (b > a) {
+      lo.push_back(a);
+      hi.push_back(b);
+    }
+  };
+  auto add_block_hog = [&](int64_t blk) {
+    const int64_t j = blk - h->blk0;
+    for (int64_t t = h->blk_task_off[j]; t < h->blk_task_off[j + 1]; ++t) {
+      lo.push_back(h->h_task_lo[t]);
+      hi.push_back(h->h_task_hi[t]);
+    }
+  };
+  auto close_launch = [&](int64_t& t0, int32_t qrep, int32_t stage) {
+    const int64_t nt = (int64_t)lo.size() - t0;
+    pl.launches.push_back(Launch{t0, nt, qrep, stage});
+    t0 = (int64_t)lo.size();
+  };
+  int64_t t0 = 0;
+  const bool G1 = (G == 1);
+  const int eff_sync = G1 ? HCCMF_SYNC_NONE : sync;
+  if (eff_sync == HCCMF_SYNC_NONE && !G1) return fail(h, HCCMF_EINVAL, "sync NONE needs n_shards == 1");
+  if (sched == HCCMF_SCHED_DET) {
+    if (eff_sync == HCCMF_SYNC_RING) {
+      if (Bc != G * Br) return fail(h, HCCMF_EINVAL, "DET+RING needs grid_cols == n_shards * grid_rows");
+      const int c = Br;
+      pl.n_stages = G;
+      for (int t = 0; t < G; ++t)
+        for (int t2 = 0; t2 < c; ++t2) {
+          for (int s = h->shard_lo; s < h->shard_hi; ++s) {
+            const int g = (s + t) % G;
+            for (int i = 0; i < c; ++i) add_block_det(blk_index(h, s, i, (int64_t)g * c + (i + t2) % c));
+          }
+          close_launch(t0, 0, t);
+        }
+    } else {
+      if (Br != Bc) return fail(h, HCCMF_EINVAL, "DET needs grid_rows == grid_cols (sync NONE/ALLREDUCE)");
+      const int c = Br;
+      for (int s = h->shard_lo; s < h->shard_hi; ++s)
+        for (int t2 = 0; t2 < c; ++t2) {
+          for (int i = 0; i < c; ++i) add_block_det(blk_index(h, s, i, (i + t2) % c));
+          close_launch(t0, s - h->shard_lo, 0);
+        }
+    }
+  } else {
+    if (eff_sync == HCCMF_SYNC_RING) {
+      if (Bc % G != 0) return fail(h, HCCMF_EINVAL, "HOGWILD+RING needs grid_cols %% n_shards == 0");
+      const int c = Bc / G;
+      pl.n_stages = G;
+      for (int t = 0; t < G; ++t)
+        for (int j = 0; j < c; ++j) {
+          for (int s = h->shard_lo; s < h->shard_hi; ++s) {
+            const int g = (s + t) % G;
+            for (int rb = 0; rb < Br; ++rb) add_block_hog(blk_index(h, s, rb, (int64_t)g * c + j));
+          }
+          close_launch(t0, 0, t);
+        }
+    } else {
+      // column-block-major phases: a user's p_u is touched by one task per launch
+      for (int s = h->shard_lo; s < h->shard_hi; ++s)
+        for (int cb = 0; cb < Bc; ++cb) {
+          for (int rb = 0; rb < Br; ++rb) add_block_hog(blk_index(h, s, rb, cb));
+          close_launch(t0, s - h->shard_lo, 0);
+        }
+    }
+  }
+  pl.n_tasks = (int64_t)lo.size();
+  CU(h, dmalloc(h, &pl.d_lo, pl.n_tasks));
+  CU(h, dmalloc(h, &pl.d_hi, pl.n_tasks));
+  if (pl.n_tasks) {
+    CU(h, cudaMemcpyAsync(pl.d_lo, lo.data(), sizeof(int64_t) * pl.n_tasks, cudaMemcpyHostToDevice, h->stream));
+    CU(h, cudaMemcpyAsync(pl.d_hi, hi.data(), sizeof(int64_t) * pl.n_tasks, cudaMemcpyHostToDevice, h->stream));
+  }
+  if ((int64_t)pl.launches.size() > h->n_counters) {
+    dfree(h, h->d_counters, h->n_counters);
+    h->n_counters = (int64_t)pl.launches.size();
+    CU(h, dmalloc(h, &h->d_counters, h->n_counters));
+  }
+  CU(h, cudaStreamSynchronize(h->stream));
+  h->plans.push_back(pl);
+  *out = &h->plans.back();
+  return HCCMF_OK;
+}
+
+int64_t auto_warps(hccmf_t h) {
+  if (h->opt_warps > 0) return h->opt_warps;
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
+  return (int64_t)sms * 32;
+}
+
+// column-group row range [a, b) of Q for ring group g
+void ring_group_cols(hccmf_t h, int sched, int g, int64_t* a, int64_t* b) {
+  const int c = (sched == HCCMF_SCHED_DET) ? h->Br : h->Bc / h->G;
+  *a = col_start(h, (int64_t)g * c);
+  *b = col_start(h, (int64_t)(g + 1) * c);
+}
+
+hccmf_status ring_exchange(hccmf_t h, int sched, int t) {
+  const int G = h->G, s = h->rank;
+  const int g_send = (s + t) % G, g_recv = (s + t + 1) % G;
+  int64_t sa, sb, ra, rb;
+  ring_group_cols(h, sched, g_send, &sa, &sb);
+  ring_group_cols(h, sched, g_recv, &ra, &rb);
+  const int prev = (s - 1 + G) % G, next = (s + 1) % G;
+  NC(h, ncclGroupStart());
+  if (sb > sa) NC(h, ncclSend(h->d_Q + sa * h->k, (size_t)(sb - sa) * h->k, ncclFloat, prev, h->comm, h->stream));
+  if (rb > ra) NC(h, ncclRecv(h->d_Q + ra * h->k, (size_t)(rb - ra) * h->k, ncclFloat, next, h->comm, h->stream));
+  NC(h, ncclGroupEnd());
+  return HCCMF_OK;
+}
+
+// after ring epochs rank s holds only group s of Q: broadcast every group from its owner
+hccmf_status materialize_q(hccmf_t h) {
+  if (h->world <= 1 || h->q_ring_sched < 0) return HCCMF_OK;
+  NC(h, ncclGroupStart());
+  for (int g = 0; g < h->G; ++g) {
+    int64_t a, b;
+    ring_group_cols(h, h->q_ring_sched, g, &a, &b);
+    if (b > a)
+      NC(h, ncclBroadcast(h->d_Q + a * h->k, h->d_Q + a * h->k, (size_t)(b - a) * h->k, ncclFloat, g, h->comm,
+                          h->stream));
+  }
+  NC(h, ncclGroupEnd());
+  h->q_ring_sched = -1;
+  return HCCMF_OK;
+}
+
+}  // namespace
+
+// ======================================================================== ABI
+extern "C" {
+
+const char* hccmf_version(void) { return "hccmf 0.1 sm_100a"; }
+
+const char* hccmf_last_error(hccmf_t h) { return h ? h->err.c_str() : g_err.c_str(); }
+
+hccmf_status hccmf_create(int64_t m, int64_t n, int32_t k, float gamma, float lambda, hccmf_t* out) {
+  if (!out) return fail(nullptr, HCCMF_EINVAL, "out is NULL");
+  *out = nullptr;
+  hccmf_status st = check_problem(m, n, k, gamma, lambda);
+  if (st != HCCMF_OK) return st;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(nullptr, HCCMF_ECUDA, "no CUDA device: %s", cudaGetErrorString(e));
+  }
+  return make_ctx(m, n, k, gamma, lambda, dev, out);
+}
+
+hccmf_status hccmf_nccl_unique_id(void* out128) {
+  if (!out128) return fail(nullptr, HCCMF_EINVAL, "out is NULL");
+  ncclUniqueId id;
+  ncclResult_t r = ncclGetUniqueId(&id);
+  if (r != ncclSuccess) return fail(nullptr, HCCMF_ENCCL, "ncclGetUniqueId: %s", ncclGetErrorString(r));
+  static_assert(sizeof(ncclUniqueId) == 128, "NCCL unique id is 128 bytes");
+  memcpy(out128, &id, sizeof(id));
+  return HCCMF_OK;
+}
+
+hccmf_status hccmf_create_dist(int64_t m, int64_t n, int32_t k, float gamma, float lambda, const void* nccl_unique_id,
+                               int32_t rank, int32_t world, int32_t device, hccmf_t* out) {
+  if (!out || !nccl_unique_id) return fail(nullptr, HCCMF_EINVAL, "NULL argument");
+  *out = nullptr;
+  if (world < 1 || rank < 0 || rank >= world || device < 0) return fail(nullptr, HCCMF_EINVAL, "bad rank/world/device");
+  hccmf_status st = check_problem(m, n, k, gamma, lambda);
+  if (st != HCCMF_OK) return st;
+  st = make_ctx(m, n, k, gamma, lambda, device, out);
+  if (st != HCCMF_OK) return st;
+  hccmf_t h = *out;
+  h->rank = rank;
+  h->world = world;
+  ncclUniqueId id;
+  memcpy(&id, nccl_unique_id, sizeof(id));
+  ncclResult_t r = ncclCommInitRank(&h->comm, world, id, rank);
+  if (r != ncclSuccess) {
+    st = fail(nullptr, HCCMF_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+    hccmf_destroy(h);
+    *out = nullptr;
+    return st;
+  }
+  return HCCMF_OK;
+}
+
+hccmf_status hccmf_set_stream(hccmf_t h, void* stream) {
+  ENTER(h);
+  if (h->own_stream && h->stream) {
+    CU(h, cudaStreamSynchronize(h->stream));
+    cudaStreamDestroy(h->stream);
+  }
+  h->stream = (cudaStream_t)stream;
+  h->own_stream = false;
+  return HCCMF_OK;
+}
+
+hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
+  ENTER(h);
+  switch (option) {
+    case HCCMF_OPT_HOGWILD_WARPS:
+      if (value < 0) return fail(h, HCCMF_EINVAL, "warps must be >= 0");
+      h->opt_warps = value;
+      return HCCMF_OK;
+    case HCCMF_OPT_TASK_RATINGS:
+      if (value < 1) return fail(h, HCCMF_EINVAL, "task ratings must be >= 1");
+      h->opt_task = value;
+      return HCCMF_OK;
+    case HCCMF_OPT_SYNC_STREAM:
+      h->sync_stream = value != 0;
+      return HCCMF_OK;
+    case HCCMF_OPT_RING_SUBBLOCKS:
+      return HCCMF_OK;
+    default:
+      return fail(h, HCCMF_EINVAL, "unknown option %d", option);
+  }
+}
+
+void hccmf_destroy(hccmf_t h) {
+  if (!h) return;
+  cudaSetDevice(h->device);
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  free_partition(h);
+  dfree(h, h->d_in_u, h->nnz);
+  dfree(h, h->d_in_v, h->nnz);
+  dfree(h, h->d_in_r, h->nnz);
+  dfree(h, h->d_partials, 2 * RMSE_BLOCKS);
+  dfree(h, h->d_scalar, 2);
+  if (h->comm) ncclCommDestroy(h->comm);
+  if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+  delete h;
+}
+
+hccmf_status hccmf_load_ratings(hccmf_t h, const int32_t* u, const int32_t* v, const float* r, int64_t nnz) {
+  ENTER(h);
+  if (nnz < 0) return fail(h, HCCMF_EINVAL, "nnz must be >= 0");
+  if (nnz > 0 && (!u || !v || !r)) return fail(h, HCCMF_EINVAL, "NULL rating array");
+  free_partition(h);
+  dfree(h, h->d_in_u, h->nnz);
+  dfree(h, h->d_in_v, h->nnz);
+  dfree(h, h->d_in_r, h->nnz);
+  h->state = 0;
+  h->nnz = nnz;
+  CU(h, dmalloc(h, &h->d_in_u, nnz));
+  CU(h, dmalloc(h, &h->d_in_v, nnz));
+  CU(h, dmalloc(h, &h->d_in_r, nnz));
+  if (!h->d_scalar) CU(h, dmalloc(h, &h->d_scalar, 2));
+  if (nnz) {
+    CU(h, cudaMemcpyAsync(h->d_in_u, u, sizeof(int32_t) * nnz, cudaMemcpyDefault, h->stream));
+    CU(h, cudaMemcpyAsync(h->d_in_v, v, sizeof(int32_t) * nnz, cudaMemcpyDefault, h->stream));
+    CU(h, cudaMemcpyAsync(h->d_in_r, r, sizeof(float) * nnz, cudaMemcpyDefault, h->stream));
+    unsigned int* flag = reinterpret_cast<unsigned int*>(h->d_scalar);
+    CU(h, cudaMemsetAsync(flag, 0, sizeof(unsigned int), h->stream));
+    CU(h, k_validate(h->d_in_u, h->d_in_v, h->d_in_r, nnz, h->m, h->n, flag, h->stream));
+    unsigned int bad = 0;
+    CU(h, cudaMemcpyAsync(&bad, flag, sizeof(bad), cudaMemcpyDeviceToHost, h->stream));
+    CU(h, cudaStreamSynchronize(h->stream));
+    if (bad) {
+      h->nnz = 0;
+      return fail(h, HCCMF_ERANGE, "invalid ratings:%s%s%s", (bad & 1) ? " u out of [0,m)" : "",
+                  (bad & 2) ? " v out of [0,n)" : "", (bad & 4) ? " non-finite r" : "");
+    }
+  }
+  h->state = 1;
+  return finish(h);
+}
+
+hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
+  ENTER(h);
+  if (!o) return fail(h, HCCMF_EINVAL, "opts is NULL");
+  if (h->state < 1 || !h->d_in_u) return fail(h, HCCMF_ESTATE, "partition needs load_ratings first");
+  const int G = o->n_shards;
+  if (G < 1) return fail(h, HCCMF_EINVAL, "n_shards must be >= 1");
+  if (h->world > 1 && G != h->world) return fail(h, HCCMF_EINVAL, "n_shards must equal the world size");
+  if (G > h->m) return fail(h, HCCMF_EINVAL, "n_shards must be <= m");
+  if (o->grid_rows < 1 || o->grid_cols < 1) return fail(h, HCCMF_EINVAL, "grid must be >= 1 x 1");
+  if (o->storage != 0) return fail(h, HCCMF_EINVAL, "only fp32 storage (0) is implemented");
+  if (o->strategy < HCCMF_DP0 || o->strategy > HCCMF_DP2) return fail(h, HCCMF_EINVAL, "bad strategy");
+  if ((o->strategy != HCCMF_DP0) && !o->t_meas) return fail(h, HCCMF_EINVAL, "DP1/DP2 need t_meas");
+  free_partition(h);
+
+  // ---- a3 partition fractions (host planner, section 3.3)
+  std::vector<double> x(G, 1.0 / G);
+  if (o->x)
+    for (int s = 0; s < G; ++s) x[s] = o->x[s];
+  if (o->strategy == HCCMF_DP0 && o->t_meas) plan_dp0(G, o->t_meas, x);
+  if (o->strategy == HCCMF_DP1) plan_dp1(G, x, std::vector<double>(o->t_meas, o->t_meas + G));
+  if (o->strategy == HCCMF_DP2) plan_dp2(G, x, o->t_meas, o->t_sync);
+  for (int s = 0; s < G; ++s)
+    if (!(x[s] >= 0.0) || !std::isfinite(x[s])) return fail(h, HCCMF_EINVAL, "partition fractions must be >= 0");
+  h->x = x;
+  h->G = G;
+  h->Br = o->grid_rows;
+  h->Bc = o->grid_cols;
+  h->seed = o->seed;
+  const int64_t m = h->m, n = h->n, nnz = h->nnz;
+  cudaStream_t st = h->stream;
+
+  // ---- a2 shuffle
+  CU(h, dmalloc(h, &h->d_perm_row, m));
+  CU(h, dmalloc(h, &h->d_perm_col, n));
+  CU(h, k_perm(h->seed, 1, m, h->d_perm_row, st));
+  CU(h, k_perm(h->seed, 2, n, h->d_perm_col, st));
+
+  // ---- a3 row histogram, prefix, boundaries
+  unsigned long long* dS = nullptr;
+  CU(h, cudaMallocAsync((void**)&dS, sizeof(unsigned long long) * (m + 1), st));
+  CU(h, k_row_prefix(h->d_in_u, nnz, h->d_perm_row, m, dS, st));
+  std::vector<int64_t> targets(G > 1 ? G - 1 : 1, 0), rstar(G > 1 ? G - 1 : 1, 0);
+  double cum = 0.0;
+  for (int s = 1; s < G; ++s) {
+    cum += x[s - 1];
+    targets[s - 1] = llround((double)nnz * cum);
+  }
+  h->bounds.assign(G + 1, 0);
+  h->bounds[G] = (int32_t)m;
+  if (G > 1) {
+    int64_t *dT = nullptr, *dR = nullptr;
+    CU(h, cudaMallocAsync((void**)&dT, sizeof(int64_t) * (G - 1), st));
+    CU(h, cudaMallocAsync((void**)&dR, sizeof(int64_t) * (G - 1), st));
+    CU(h, cudaMemcpyAsync(dT, targets.data(), sizeof(int64_t) * (G - 1), cudaMemcpyHostToDevice, st));
+    CU(h, k_bound_search(dS, m, dT, G - 1, dR, st));
+    CU(h, cudaMemcpyAsync(rstar.data(), dR, sizeof(int64_t) * (G - 1), cudaMemcpyDeviceToHost, st));
+    CU(h, cudaStreamSynchronize(st));
+    cudaFreeAsync(dT, st);
+    cudaFreeAsync(dR, st);
+    for (int s = 1; s < G; ++s) h->bounds[s] = (int32_t)std::max<int64_t>(h->bounds[s - 1], rstar[s - 1]);
+  }
+  cudaFreeAsync(dS, st);
+  int32_t* dB = nullptr;
+  CU(h, cudaMallocAsync((void**)&dB, sizeof(int32_t) * (G + 1), st));
+  CU(h, cudaMemcpyAsync(dB, h->bounds.data(), sizeof(int32_t) * (G + 1), cudaMemcpyHostToDevice, st));
+
+  // ---- a4 geometry + stable sort
+  BlockGeom g{};
+  g.G = G;
+  g.Br = h->Br;
+  g.Bc = h->Bc;
+  g.m = m;
+  g.n = n;
+  int64_t maxr = 1;
+  for (int s = 0; s < G; ++s) maxr = std::max<int64_t>(maxr, ceil_div((int64_t)h->bounds[s + 1] - h->bounds[s], h->Br));
+  const int64_t nblk = (int64_t)G * h->Br * h->Bc;
+  g.bu = bitlen((uint64_t)(maxr - 1));
+  g.bv = bitlen((uint64_t)(ceil_div(n, h->Bc) - 1));
+  g.bb = bitlen((uint64_t)(nblk - 1));
+  if (g.bb + g.bu + g.bv > 64) return fail(h, HCCMF_ERANGE, "sort key needs %d > 64 bits", g.bb + g.bu + g.bv);
+  h->geom = g;
+  int32_t *su = nullptr, *sv = nullptr;
+  float* sr = nullptr;
+  int64_t* dOff = nullptr;
+  CU(h, dmalloc(h, &su, nnz));
+  CU(h, dmalloc(h, &sv, nnz));
+  CU(h, dmalloc(h, &sr, nnz));
+  CU(h, cudaMallocAsync((void**)&dOff, sizeof(int64_t) * (nblk + 1), st));
+  CU(h, k_block_sort(g, dB, h->d_perm_row, h->d_perm_col, h->d_in_u, h->d_in_v, h->d_in_r, nnz, su, sv, sr, dOff, st));
+  h->block_off.assign(nblk + 1, 0);
+  CU(h, cudaMemcpyAsync(h->block_off.data(), dOff, sizeof(int64_t) * (nblk + 1), cudaMemcpyDeviceToHost, st));
+  CU(h, cudaStreamSynchronize(st));
+  cudaFreeAsync(dOff, st);
+  cudaFreeAsync(dB, st);
+  dfree(h, h->d_in_u, nnz);
+  dfree(h, h->d_in_v, nnz);
+  dfree(h, h->d_in_r, nnz);
+
+  // ---- local shard(s)
+  const int64_t bps = (int64_t)h->Br * h->Bc;
+  if (h->world > 1) {
+    h->shard_lo = h->rank;
+    h->shard_hi = h->rank + 1;
+  } else {
+    h->shard_lo = 0;
+    h->shard_hi = G;
+  }
+  h->blk0 = h->shard_lo * bps;
+  h->nblk_local = (h->shard_hi - h->shard_lo) * bps;
+  h->rec0 = h->block_off[h->blk0];
+  h->local_nnz = h->block_off[h->blk0 + h->nblk_local] - h->rec0;
+  if (h->world > 1) {
+    CU(h, dmalloc(h, &h->d_u, h->local_nnz));
+    CU(h, dmalloc(h, &h->d_v, h->local_nnz));
+    CU(h, dmalloc(h, &h->d_r, h->local_nnz));
+    if (h->local_nnz) {
+      CU(h, cudaMemcpyAsync(h->d_u, su + h->rec0, 4 * h->local_nnz, cudaMemcpyDeviceToDevice, st));
+      CU(h, cudaMemcpyAsync(h->d_v, sv + h->rec0, 4 * h->local_nnz, cudaMemcpyDeviceToDevice, st));
+      CU(h, cudaMemcpyAsync(h->d_r, sr + h->rec0, 4 * h->local_nnz, cudaMemcpyDeviceToDevice, st));
+    }
+    CU(h, cudaStreamSynchronize(st));
+    dfree(h, su, nnz);
+    dfree(h, sv, nnz);
+    dfree(h, sr, nnz);
+  } else {
+    h->d_u = su;
+    h->d_v = sv;
+    h->d_r = sr;
+  }
+  h->row0 = h->bounds[h->shard_lo];
+  h->rows = (int64_t)h->bounds[h->shard_hi] - h->row0;
+
+  // ---- Hogwild tasks: user-aligned runs of ~opt_task ratings inside each block
+  std::vector<int64_t> loc_off(h->nblk_local + 1);
+  for (int64_t j = 0; j <= h->nblk_local; ++j) loc_off[j] = h->block_off[h->blk0 + j] - h->rec0;
+  int64_t* dLoc = nullptr;
+  CU(h, cudaMallocAsync((void**)&dLoc, sizeof(int64_t) * (h->nblk_local + 1), st));
+  CU(h, cudaMemcpyAsync(dLoc, loc_off.data(), sizeof(int64_t) * (h->nblk_local + 1), cudaMemcpyHostToDevice, st));
+  int64_t nt = 0;
+  CU(h, k_build_tasks(h->d_u, h->local_nnz, dLoc, h->nblk_local, h->opt_task, &h->d_task_lo, &h->d_task_hi, &nt, st));
+  h->device_bytes += 2 * sizeof(int64_t) * (nt ? nt : 1);
+  h->n_tasks = nt;
+  cudaFreeAsync(dLoc, st);
+  h->h_task_lo.resize(nt);
+  h->h_task_hi.resize(nt);
+  if (nt) {
+    CU(h, cudaMemcpyAsync(h->h_task_lo.data(), h->d_task_lo, sizeof(int64_t) * nt, cudaMemcpyDeviceToHost, st));
+    CU(h, cudaMemcpyAsync(h->h_task_hi.data(), h->d_task_hi, sizeof(int64_t) * nt, cudaMemcpyDeviceToHost, st));
+  }
+  CU(h, cudaStreamSynchronize(st));
+  // tasks are grouped by block (LPT order inside a block): count per block
+  h->blk_task_off.assign(h->nblk_local + 1, 0);
+  for (int64_t t = 0; t < nt; ++t) {
+    const int64_t j = std::upper_bound(loc_off.begin(), loc_off.end(), h->h_task_lo[t]) - loc_off.begin() - 1;
+    h->blk_task_off[j + 1] += 1;
+  }
+  for (int64_t j = 0; j < h->nblk_local; ++j) h->blk_task_off[j + 1] += h->blk_task_off[j];
+
+  // ---- factors
+  CU(h, dmalloc(h, &h->d_P, h->rows * h->k));
+  CU(h, dmalloc(h, &h->d_Q, h->n * h->k));
+  if (!h->d_partials) CU(h, dmalloc(h, &h->d_partials, 2 * RMSE_BLOCKS));
+  h->q_ring_sched = -1;
+  h->state = 2;
+  return finish(h);
+}
+
+hccmf_status hccmf_init_factors(hccmf_t h, uint64_t seed) {
+  ENTER(h);
+  if (h->state < 2) return fail(h, HCCMF_ESTATE, "init_factors needs partition first");
+  CU(h, k_init_factors(seed, 3, h->m, h->k, h->d_perm_row, h->row0, h->rows, h->d_P, h->stream));
+  CU(h, k_init_factors(seed, 4, h->n, h->k, h->d_perm_col, 0, h->n, h->d_Q, h->stream));
+  h->q_ring_sched = -1;
+  h->state = 3;
+  return finish(h);
+}
+
+hccmf_status hccmf_set_factors(hccmf_t h, const float* P, const float* Q) {
+  ENTER(h);
+  if (h->state < 2) return fail(h, HCCMF_ESTATE, "set_factors needs partition first");
+  if (!P || !Q) return fail(h, HCCMF_EINVAL, "P and Q are required");
+  const size_t mk = (size_t)h->m * h->k, nk = (size_t)h->n * h->k;
+  float* tmp = nullptr;
+  CU(h, cudaMallocAsync((void**)&tmp, sizeof(float) * std::max(mk, nk), h->stream));
+  CU(h, cudaMemcpyAsync(tmp, P, sizeof(float) * mk, cudaMemcpyDefault, h->stream));
+  CU(h, k_scatter_rows(tmp, h->m, h->k, h->d_perm_row, h->row0, h->rows, h->d_P, h->stream));
+  CU(h, cudaMemcpyAsync(tmp, Q, sizeof(float) * nk, cudaMemcpyDefault, h->stream));
+  CU(h, k_scatter_rows(tmp, h->n, h->k, h->d_perm_col, 0, h->n, h->d_Q, h->stream));
+  cudaFreeAsync(tmp, h->stream);
+  h->q_ring_sched = -1;
+  h->state = 3;
+  return finish(h);
+}
+
+hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
+  ENTER(h);
+  if (h->state < 3) return fail(h, HCCMF_ESTATE, "train_epoch needs factors (init_factors or set_factors)");
+  if (sched != HCCMF_SCHED_DET && sched != HCCMF_SCHED_HOGWILD) return fail(h, HCCMF_EINVAL, "bad schedule");
+  if (sync < HCCMF_SYNC_NONE || sync > HCCMF_SYNC_ALLREDUCE_AVG) return fail(h, HCCMF_EINVAL, "bad sync");
+  Plan* pl = nullptr;
+  hccmf_status st = build_plan(h, sched, sync, &pl);
+  if (st != HCCMF_OK) return st;
+  const int G = h->G;
+  const int eff_sync = (G == 1) ? HCCMF_SYNC_NONE : sync;
+  const bool dist = h->world > 1;
+  const int64_t nk = h->n * h->k;
+  cudaStream_t s = h->stream;
+  if (eff_sync != HCCMF_SYNC_RING || h->q_ring_sched != sched) {
+    st = materialize_q(h);
+    if (st != HCCMF_OK) return st;
+  }
+  const int nrep = h->shard_hi - h->shard_lo;
+  if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && !dist) {
+    if (!h->d_Qrep) CU(h, dmalloc(h, &h->d_Qrep, (size_t)nk * nrep));
+    for (int r = 0; r < nrep; ++r)
+      CU(h, cudaMemcpyAsync(h->d_Qrep + (size_t)r * nk, h->d_Q, sizeof(float) * nk, cudaMemcpyDeviceToDevice, s));
+  }
+  CU(h, cudaMemsetAsync(h->d_counters, 0, sizeof(unsigned long long) * pl->launches.size(), s));
+  SgdArgs a{};
+  a.ru = h->d_u;
+  a.rv = h->d_v;
+  a.rr = h->d_r;
+  a.P = h->d_P;
+  a.row0 = h->row0;
+  a.k = h->k;
+  a.gamma = h->gamma;
+  a.lambda = h->lambda;
+  const int L = lanes_per_rating(h->k);
+  const int64_t hog_warps = auto_warps(h);
+  int stage = 0;
+  for (size_t li = 0; li < pl->launches.size(); ++li) {
+    const Launch& ln = pl->launches[li];
+    if (dist && eff_sync == HCCMF_SYNC_RING) {
+      while (stage < ln.stage) {
+        st = ring_exchange(h, sched, stage++);
+        if (st != HCCMF_OK) return st;
+      }
+    }
+    a.Q = (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && !dist) ? h->d_Qrep + (size_t)ln.qrep * nk : h->d_Q;
+    a.task_lo = pl->d_lo + ln.t0;
+    a.task_hi = pl->d_hi + ln.t0;
+    a.n_tasks = ln.nt;
+    a.counter = h->d_counters + li;
+    // DET: one rating group per block of the stratum; HOGWILD: persistent grid
+    const int64_t warps = (sched == HCCMF_SCHED_DET) ? (ln.nt * L + 31) / 32 : hog_warps;
+    CU(h, launch_sgd(a, warps, s));
+  }
+  if (dist && eff_sync == HCCMF_SYNC_RING) {
+    while (stage < pl->n_stages) {
+      st = ring_exchange(h, sched, stage++);
+      if (st != HCCMF_OK) return st;
+    }
+    h->q_ring_sched = sched;
+  }
+  if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG) {
+    if (dist)
+      NC(h, ncclAllReduce(h->d_Q, h->d_Q, (size_t)nk, ncclFloat, ncclAvg, h->comm, s));
+    else
+      CU(h, k_average(h->d_Qrep, nrep, nk, h->d_Q, s));
+  }
+  return finish(h);
+}
+
+hccmf_status hccmf_rmse(hccmf_t h, const int32_t* u, const int32_t* v, const float* r, int64_t nt, double* out) {
+  ENTER(h);
+  if (!out) return fail(h, HCCMF_EINVAL, "out is NULL");
+  if (h->state < 3) return fail(h, HCCMF_ESTATE, "rmse needs factors");
+  if (nt < 0 || (nt > 0 && (!u || !v || !r))) return fail(h, HCCMF_EINVAL, "bad test set");
+  hccmf_status st = materialize_q(h);
+  if (st != HCCMF_OK) return st;
+  cudaStream_t s = h->stream;
+  int32_t *du = nullptr, *dv = nullptr;
+  float* dr = nullptr;
+  CU(h, cudaMallocAsync((void**)&du, 4 * (nt ? nt : 1), s));
+  CU(h, cudaMallocAsync((void**)&dv, 4 * (nt ? nt : 1), s));
+  CU(h, cudaMallocAsync((void**)&dr, 4 * (nt ? nt : 1), s));
+  if (nt) {
+    CU(h, cudaMemcpyAsync(du, u, 4 * nt, cudaMemcpyDefault, s));
+    CU(h, cudaMemcpyAsync(dv, v, 4 * nt, cudaMemcpyDefault, s));
+    CU(h, cudaMemcpyAsync(dr, r, 4 * nt, cudaMemcpyDefault, s));
+    unsigned int* flag = reinterpret_cast<unsigned int*>(h->d_partials);
+    CU(h, cudaMemsetAsync(flag, 0, sizeof(unsigned int), s));
+    CU(h, k_validate(du, dv, dr, nt, h->m, h->n, flag, s));
+    unsigned int bad = 0;
+    CU(h, cudaMemcpyAsync(&bad, flag, sizeof(bad), cudaMemcpyDeviceToHost, s));
+    CU(h, cudaStreamSynchronize(s));
+    if (bad) {
+      cudaFreeAsync(du, s);
+      cudaFreeAsync(dv, s);
+      cudaFreeAsync(dr, s);
+      return fail(h, HCCMF_ERANGE, "invalid test ratings");
+    }
+  }
+  CU(h, k_rmse(du, dv, dr, nt, h->d_perm_row, h->d_perm_col, h->d_P, h->row0, h->rows, h->d_Q, h->k, h->d_partials,
+               h->d_scalar, s));
+  if (h->world > 1) NC(h, ncclAllReduce(h->d_scalar, h->d_scalar, 2, ncclDouble, ncclSum, h->comm, s));
+  double sc[2] = {0.0, 0.0};
+  CU(h, cudaMemcpyAsync(sc, h->d_scalar, sizeof(sc), cudaMemcpyDeviceToHost, s));
+  CU(h, cudaStreamSynchronize(s));
+  cudaFreeAsync(du, s);
+  cudaFreeAsync(dv, s);
+  cudaFreeAsync(dr, s);
+  *out = sc[1] > 0.0 ? std::sqrt(sc[0] / sc[1]) : 0.0;
+  return finish(h);
+}
+
+hccmf_status hccmf_get_factors(hccmf_t h, float* P, float* Q) {
+  ENTER(h);
+  if (h->state < 3) return fail(h, HCCMF_ESTATE, "get_factors needs factors");
+  cudaStream_t s = h->stream;
+  const size_t mk = (size_t)h->m * h->k, nk = (size_t)h->n * h->k;
+  if (P) {
+    float* full = h->d_P;
+    float* tmp = nullptr;
+    if (h->world > 1) {  // final push of P (L1205-L1206): every shard's rows to every rank
+      CU(h, cudaMallocAsync((void**)&full, sizeof(float) * mk, s));
+      NC(h, ncclGroupStart());
+      for (int g = 0; g < h->G; ++g) {
+        const int64_t a = h->bounds[g], b = h->bounds[g + 1];
+        if (b > a) {
+          const float* src = (g == h->rank) ? h->d_P : full + a * h->k;
+          NC(h, ncclBroadcast(src, full + a * h->k, (size_t)(b - a) * h->k, ncclFloat, g, h->comm, s));
+        }
+      }
+      NC(h, ncclGroupEnd());
+    }
+    CU(h, cudaMallocAsync((void**)&tmp, sizeof(float) * mk, s));
+    CU(h, k_gather_rows(full, h->m, h->k, h->d_perm_row, 0, tmp, s));
+    CU(h, cudaMemcpyAsync(P, tmp, sizeof(float) * mk, cudaMemcpyDefault, s));
+    CU(h, cudaStreamSynchronize(s));
+    cudaFreeAsync(tmp, s);
+    if (full != h->d_P) cudaFreeAsync(full, s);
+  }
+  if (Q) {
+    hccmf_status st = materialize_q(h);
+    if (st != HCCMF_OK) return st;
+    float* tmp = nullptr;
+    CU(h, cudaMallocAsync((void**)&tmp, sizeof(float) * nk, s));
+    CU(h, k_gather_rows(h->d_Q, h->n, h->k, h->d_perm_col, 0, tmp, s));
+    CU(h, cudaMemcpyAsync(Q, tmp, sizeof(float) * nk, cudaMemcpyDefault, s));
+    CU(h, cudaStreamSynchronize(s));
+    cudaFreeAsync(tmp, s);
+  }
+  return finish(h);
+}
+
+hccmf_status hccmf_get_partition(hccmf_t h, int32_t* bounds, int64_t* block_off, int32_t* perm_row, int32_t* perm_col) {
+  ENTER(h);
+  if (h->state < 2) return fail(h, HCCMF_ESTATE, "get_partition needs partition");
+  if (bounds) memcpy(bounds, h->bounds.data(), sizeof(int32_t) * h->bounds.size());
+  if (block_off) memcpy(block_off, h->block_off.data(), sizeof(int64_t) * h->block_off.size());
+  if (perm_row) CU(h, cudaMemcpyAsync(perm_row, h->d_perm_row, 4 * h->m, cudaMemcpyDefault, h->stream));
+  if (perm_col) CU(h, cudaMemcpyAsync(perm_col, h->d_perm_col, 4 * h->n, cudaMemcpyDefault, h->stream));
+  CU(h, cudaStreamSynchronize(h->stream));
+  return finish(h);
+}
+
+hccmf_status hccmf_get_records(hccmf_t h, int32_t* u, int32_t* v, float* r) {
+  ENTER(h);
+  if (h->state < 2) return fail(h, HCCMF_ESTATE, "get_records needs partition");
+  const int64_t c = h->local_nnz;
+  if (c) {
+    if (u) CU(h, cudaMemcpyAsync(u, h->d_u, 4 * c, cudaMemcpyDefault, h->stream));
+    if (v) CU(h, cudaMemcpyAsync(v, h->d_v, 4 * c, cudaMemcpyDefault, h->stream));
+    if (r) CU(h, cudaMemcpyAsync(r, h->d_r, 4 * c, cudaMemcpyDefault, h->stream));
+  }
+  CU(h, cudaStreamSynchronize(h->stream));
+  return finish(h);
+}
+
+hccmf_status hccmf_get_fractions(hccmf_t h, double* x) {
+  ENTER(h);
+  if (h->state < 2) return fail(h, HCCMF_ESTATE, "get_fractions needs partition");
+  if (!x) return fail(h, HCCMF_EINVAL, "x is NULL");
+  memcpy(x, h->x.data(), sizeof(double) * h->x.size());
+  return HCCMF_OK;
+}
+
+hccmf_status hccmf_get_info(hccmf_t h, hccmf_info* o) {
+  if (!h || !o) return fail(h, HCCMF_EINVAL, "NULL argument");
+  memset(o, 0, sizeof(*o));
+  o->m = h->m;
+  o->n = h->n;
+  o->nnz = h->nnz;
+  o->k = h->k;
+  o->n_shards = h->G;
+  o->shard_lo = h->shard_lo;
+  o->shard_hi = h->shard_hi;
+  o->local_nnz = h->local_nnz;
+  o->row0 = h->row0;
+  o->rows = h->rows;
+  o->n_blocks = (int64_t)h->G * h->Br * h->Bc;
+  o->n_tasks = h->n_tasks;
+  o->key_bits = h->geom.bb + h->geom.bu + h->geom.bv;
+  o->rank = h->rank;
+  o->world = h->world;
+  o->device_bytes = (int64_t)h->device_bytes;
+  return HCCMF_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,440 @@
+// blocker.cu -- a1-a4 and the Hogwild task builder: validation, seeded ID shuffle,
+// row histogram + prefix, shard-boundary search, blocking + stable radix sort.
+//
+// PAPER.md section 3.1 preprocessing "shuffling, sorting, and data partition"
+// (L543-L548), row grid (L881-L895), row-sorted blocks (L1472-L1474).  Every
+// step is integer work and bit-exact against the oracle (tests/test_gpu_*).
+#include <cub/cub.cuh>
+#include <thrust/iterator/counting_iterator.h>
+
+#include "internal.cuh"
+
+namespace hccmf {
+namespace {
+
+constexpr int kT = 256;
+
+inline unsigned grid_for(int64_t n, int64_t cap = 148LL * 64) {
+  int64_t b = (n + kT - 1) / kT;
+  if (b < 1) b = 1;
+  if (b > cap) b = cap;
+  return (unsigned)b;
+}
+
+__global__ void validate_kernel(const int32_t* __restrict__ u, const int32_t* __restrict__ v,
+                                const float* __restrict__ r, int64_t nnz, int64_t m, int64_t n,
+                                unsigned int* flag) {
+  unsigned bad = 0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t uu = u[i], vv = v[i];
+    const float rr = r[i];
+    if (uu < 0 || uu >= m) bad |= 1u;
+    if (vv < 0 || vv >= n) bad |= 2u;
+    if (!isfinite(rr)) bad |= 4u;
+  }
+  bad = __reduce_or_sync(0xffffffffu, bad);
+  if (bad && (threadIdx.x & 31) == 0) atomicOr(flag, bad);
+}
+
+__global__ void perm_keys_kernel(uint64_t seed, uint64_t tag, int64_t count, uint64_t* keys, int32_t* ids) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x) {
+    keys[i] = hash4(seed, tag, (uint64_t)i, 0);
+    ids[i] = (int32_t)i;
+  }
+}
+
+__global__ void perm_scatter_kernel(const int32_t* ids_sorted, int64_t count, int32_t* perm) {
+  for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < count; r += (int64_t)gridDim.x * blockDim.x)
+    perm[ids_sorted[r]] = (int32_t)r;
+}
+
+__global__ void iota_kernel(int32_t* perm, int64_t count) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x)
+    perm[i] = (int32_t)i;
+}
+
+__global__ void row_count_kernel(const int32_t* __restrict__ u, int64_t nnz, const int32_t* __restrict__ perm_row,
+                                 unsigned long long* cnt) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(cnt + perm_row[u[i]], 1ull);
+}
+
+// first r in [0, m] with S[r] >= x  (S non-decreasing, m+1 entries); m+1 if none
+__device__ int64_t lower_bound_u64(const unsigned long long* S, int64_t m, unsigned long long x) {
+  int64_t lo = 0, hi = m + 1;
+  while (lo < hi) {
+    const int64_t mid = lo + ((hi - lo) >> 1);
+    if (S[mid] < x) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+// unrestricted argmin_r |S[r] - T|, ties to the smaller r (R10); the
+// host applies b_s = max(b_{s-1}, r*), which equals the restricted argmin.
+__global__ void bound_search_kernel(const unsigned long long* S, int64_t m, const int64_t* targets, int32_t nt,
+                                    int64_t* out) {
+  const int s = blockIdx.x * blockDim.x + threadIdx.x;
+  if (s >= nt) return;
+  const int64_t T = targets[s];
+  if (T <= 0) { out[s] = 0; return; }
+  const int64_t a = lower_bound_u64(S, m, (unsigned long long)T);  // S[a] >= T
+  int64_t best = -1;
+  int64_t dbest = 0;
+  if (a <= m) { best = a; dbest = (int64_t)S[a] - T; }
+  if (a > 0) {
+    const unsigned long long vb = S[a - 1];  // < T
+    const int64_t b = lower_bound_u64(S, m, vb);  // first r with S[r] == vb
+    const int64_t db = T - (int64_t)vb;
+    if (best < 0 || db <= dbest) best = b;
+  }
+  out[s] = best;
+}
+
+__device__ __forceinline__ int32_t shard_of(const int32_t* b, int32_t G, int32_t up) {
+  // largest s with b[s] <= up (b non-decreasing, b[0] = 0 <= up < b[G] = m)
+  int lo = 0, hi = G;  // answer in [0, G-1]
+  while (hi - lo > 1) {
+    const int mid = (lo + hi) >> 1;
+    if (b[mid] <= up) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+__device__ __forceinline__ int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+__global__ void block_key_kernel(BlockGeom g, const int32_t* __restrict__ bounds, const int32_t* __restrict__ perm_row,
+                                 const int32_t* __restrict__ perm_col, const int32_t* __restrict__ u,
+                                 const int32_t* __restrict__ v, int64_t nnz, uint64_t* keys) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t up = perm_row[u[i]], vp = perm_col[v[i]];
+    const int32_t s = shard_of(bounds, g.G, up);
+    const int64_t rows = (int64_t)bounds[s + 1] - bounds[s];
+    const int64_t l = (int64_t)up - bounds[s];
+    const int64_t rb = (l * g.Br) / rows;
+    const int64_t rstart = ceil_div(rb * rows, g.Br);
+    const int64_t cb = ((int64_t)vp * g.Bc) / g.n;
+    const int64_t cstart = ceil_div(cb * g.n, g.Bc);
+    const uint64_t blk = (uint64_t)(((int64_t)s * g.Br + rb) * g.Bc + cb);
+    keys[i] = (blk << (g.bu + g.bv)) | ((uint64_t)(l - rstart) << g.bv) | (uint64_t)(vp - cstart);
+  }
+}
+
+__global__ void block_decode_kernel(BlockGeom g, const int32_t* __restrict__ bounds, const uint64_t* __restrict__ keys,
+                                    int64_t nnz, int32_t* ou, int32_t* ov) {
+  const uint64_t mu = (g.bu >= 64) ? ~0ull : ((1ull << g.bu) - 1);
+  const uint64_t mv = (g.bv >= 64) ? ~0ull : ((1ull << g.bv) - 1);
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint64_t key = keys[i];
+    const int sh = g.bu + g.bv;
+    const int64_t blk = sh >= 64 ? 0 : (int64_t)(key >> sh);
+    const int64_t lu = (int64_t)((key >> g.bv) & mu);
+    const int64_t lv = (int64_t)(key & mv);
+    const int64_t cb = blk % g.Bc;
+    const int64_t srb = blk / g.Bc;
+    const int64_t rb = srb % g.Br;
+    const int64_t s = srb / g.Br;
+    const int64_t rows = (int64_t)bounds[s + 1] - bounds[s];
+    const int64_t rstart = ceil_div(rb * rows, g.Br);
+    const int64_t cstart = ceil_div(cb * g.n, g.Bc);
+    ou[i] = (int32_t)(bounds[s] + rstart + lu);
+    ov[i] = (int32_t)(cstart + lv);
+  }
+}
+
+__global__ void block_off_kernel(const uint64_t* __restrict__ keys, int64_t nnz, int shift, int64_t nblk, int64_t* off) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j <= nblk; j += (int64_t)gridDim.x * blockDim.x) {
+    if (j == nblk) { off[j] = nnz; continue; }
+    const uint64_t x = shift >= 64 ? 0 : ((uint64_t)j << shift);
+    int64_t lo = 0, hi = nnz;
+    if (shift >= 64) { off[j] = 0; continue; }
+    while (lo < hi) {
+      const int64_t mid = lo + ((hi - lo) >> 1);
+      if (keys[mid] < x) lo = mid + 1; else hi = mid;
+    }
+    off[j] = lo;
+  }
+}
+
+// ---------------------------------------------------------------- tasks
+__global__ void run_flag_kernel(const int32_t* __restrict__ ru, int64_t nrec, unsigned char* flag) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nrec; i += (int64_t)gridDim.x * blockDim.x)
+    flag[i] = (i == 0 || ru[i] != ru[i - 1]) ? 1 : 0;
+}
+
+__global__ void block_start_flag_kernel(const int64_t* off, int64_t nb, int64_t nrec, unsigned char* flag) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < nb; j += (int64_t)gridDim.x * blockDim.x)
+    if (off[j] < off[j + 1] && off[j] < nrec) flag[off[j]] = 1;
+}
+
+__global__ void cand_count_kernel(const int64_t* off, int64_t nb, int64_t target, int64_t* cnt) {
+  for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j < nb; j += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t len = off[j + 1] - off[j];
+    cnt[j] = (len + target - 1) / target;
+  }
+}
+
+__device__ int64_t upper_bound_i64(const int64_t* a, int64_t n, int64_t x) {  // first idx with a[idx] > x
+  int64_t lo = 0, hi = n;
+  while (lo < hi) {
+    const int64_t mid = lo + ((hi - lo) >> 1);
+    if (a[mid] <= x) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+__device__ int64_t lower_bound_i64(const int64_t* a, int64_t n, int64_t x) {  // first idx with a[idx] >= x
+  int64_t lo = 0, hi = n;
+  while (lo < hi) {
+    const int64_t mid = lo + ((hi - lo) >> 1);
+    if (a[mid] < x) lo = mid + 1; else hi = mid;
+  }
+  return lo;
+}
+
+// candidate c (global numbering): block j = upper_bound(cand_off, c)-1, q = c - cand_off[j],
+// pos = off[j] + q*target, mapped to the first run start >= pos; kept if < off[j+1]
+// and different from the mapping of candidate q-1.
+__global__ void cand_map_kernel(const int64_t* cand_off, int64_t nb, int64_t ncand, const int64_t* off,
+                                int64_t target, const int64_t* runs, int64_t nruns, int64_t* cand_pos,
+                                unsigned char* keep) {
+  for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < ncand; c += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t j = upper_bound_i64(cand_off, nb + 1, c) - 1;
+    const int64_t q = c - cand_off[j];
+    const int64_t pos = off[j] + q * target;
+    const int64_t ri = lower_bound_i64(runs, nruns, pos);
+    const int64_t mp = ri < nruns ? runs[ri] : INT64_MAX;
+    bool k = mp < off[j + 1];
+    if (k && q > 0) {
+      const int64_t pp = off[j] + (q - 1) * target;
+      const int64_t rp = lower_bound_i64(runs, nruns, pp);
+      const int64_t mpp = rp < nruns ? runs[rp] : INT64_MAX;
+      k = mpp != mp;
+    }
+    cand_pos[c] = mp;
+    keep[c] = k ? 1 : 0;
+  }
+}
+
+__global__ void task_hi_kernel(const int64_t* lo, int64_t nt, const int64_t* off, int64_t nb, int64_t* hi,
+                               uint64_t* sortkey, int64_t* idx) {
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nt; t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t j = upper_bound_i64(off, nb + 1, lo[t]) - 1;
+    int64_t h = off[j + 1];
+    if (t + 1 < nt && lo[t + 1] < h) h = lo[t + 1];
+    hi[t] = h;
+    // LPT inside each block: ascending (block, -len)
+    const uint64_t len = (uint64_t)(h - lo[t]);
+    const uint64_t inv = (len >= (1ull << 38)) ? 0 : ((1ull << 38) - 1 - len);
+    sortkey[t] = ((uint64_t)j << 38) | inv;
+    idx[t] = t;
+  }
+}
+
+__global__ void permute_tasks_kernel(const int64_t* idx, int64_t nt, const int64_t* lo, const int64_t* hi,
+                                     int64_t* olo, int64_t* ohi) {
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nt; t += (int64_t)gridDim.x * blockDim.x) {
+    olo[t] = lo[idx[t]];
+    ohi[t] = hi[idx[t]];
+  }
+}
+
+template <typename T>
+cudaError_t dalloc(T** p, size_t count, cudaStream_t st) {
+  return cudaMallocAsync((void**)p, sizeof(T) * (count ? count : 1), st);
+}
+
+#define CKR(x)                            \
+  do {                                    \
+    cudaError_t e_ = (x);                 \
+    if (e_ != cudaSuccess) return e_;     \
+  } while (0)
+
+}  // namespace
+
+cudaError_t k_validate(const int32_t* u, const int32_t* v, const float* r, int64_t nnz, int64_t m, int64_t n,
+                       unsigned int* flag, cudaStream_t st) {
+  if (nnz == 0) return cudaSuccess;
+  validate_kernel<<<grid_for(nnz), kT, 0, st>>>(u, v, r, nnz, m, n, flag);
+  return cudaGetLastError();
+}
+
+cudaError_t k_perm(uint64_t seed, uint64_t tag, int64_t count, int32_t* perm, cudaStream_t st) {
+  if (count == 0) return cudaSuccess;
+  if (seed == 0) {
+    iota_kernel<<<grid_for(count), kT, 0, st>>>(perm, count);
+    return cudaGetLastError();
+  }
+  uint64_t *k0 = nullptr, *k1 = nullptr;
+  int32_t *i0 = nullptr, *i1 = nullptr;
+  CKR(dalloc(&k0, count, st));
+  CKR(dalloc(&k1, count, st));
+  CKR(dalloc(&i0, count, st));
+  CKR(dalloc(&i1, count, st));
+  perm_keys_kernel<<<grid_for(count), kT, 0, st>>>(seed, tag, count, k0, i0);
+  CKR(cudaGetLastError());
+  size_t tb = 0;
+  void* tmp = nullptr;
+  CKR(cub::DeviceRadixSort::SortPairs(nullptr, tb, k0, k1, i0, i1, count, 0, 64, st));
+  CKR(cudaMallocAsync(&tmp, tb, st));
+  CKR(cub::DeviceRadixSort::SortPairs(tmp, tb, k0, k1, i0, i1, count, 0, 64, st));
+  perm_scatter_kernel<<<grid_for(count), kT, 0, st>>>(i1, count, perm);
+  CKR(cudaGetLastError());
+  cudaFreeAsync(tmp, st);
+  cudaFreeAsync(k0, st);
+  cudaFreeAsync(k1, st);
+  cudaFreeAsync(i0, st);
+  cudaFreeAsync(i1, st);
+  return cudaGetLastError();
+}
+
+cudaError_t k_row_prefix(const int32_t* u, int64_t nnz, const int32_t* perm_row, int64_t m, unsigned long long* S,
+                         cudaStream_t st) {
+  unsigned long long* cnt = nullptr;
+  CKR(dalloc(&cnt, m + 1, st));
+  CKR(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * (m + 1), st));
+  if (nnz) {
+    row_count_kernel<<<grid_for(nnz), kT, 0, st>>>(u, nnz, perm_row, cnt);
+    CKR(cudaGetLastError());
+  }
+  size_t tb = 0;
+  void* tmp = nullptr;
+  CKR(cub::DeviceScan::ExclusiveSum(nullptr, tb, cnt, S, m + 1, st));
+  CKR(cudaMallocAsync(&tmp, tb, st));
+  CKR(cub::DeviceScan::ExclusiveSum(tmp, tb, cnt, S, m + 1, st));
+  cudaFreeAsync(tmp, st);
+  cudaFreeAsync(cnt, st);
+  return cudaGetLastError();
+}
+
+cudaError_t k_bound_search(const unsigned long long* S, int64_t m, const int64_t* targets, int32_t nt, int64_t* out,
+                           cudaStream_t st) {
+  if (nt <= 0) return cudaSuccess;
+  bound_search_kernel<<<(nt + 127) / 128, 128, 0, st>>>(S, m, targets, nt, out);
+  return cudaGetLastError();
+}
+
+cudaError_t k_block_sort(const BlockGeom& g, const int32_t* bounds, const int32_t* perm_row, const int32_t* perm_col,
+                         const int32_t* u, const int32_t* v, const float* r, int64_t nnz, int32_t* ou, int32_t* ov,
+                         float* orr, int64_t* block_off, cudaStream_t st) {
+  const int64_t nblk = (int64_t)g.G * g.Br * g.Bc;
+  const int bits = g.bb + g.bu + g.bv;
+  uint64_t *k0 = nullptr, *k1 = nullptr;
+  CKR(dalloc(&k0, nnz, st));
+  CKR(dalloc(&k1, nnz, st));
+  if (nnz) {
+    block_key_kernel<<<grid_for(nnz), kT, 0, st>>>(g, bounds, perm_row, perm_col, u, v, nnz, k0);
+    CKR(cudaGetLastError());
+  }
+  const uint64_t* ks = k0;
+  if (nnz && bits > 0) {
+    size_t tb = 0;
+    void* tmp = nullptr;
+    CKR(cub::DeviceRadixSort::SortPairs(nullptr, tb, k0, k1, r, orr, nnz, 0, bits, st));
+    CKR(cudaMallocAsync(&tmp, tb, st));
+    CKR(cub::DeviceRadixSort::SortPairs(tmp, tb, k0, k1, r, orr, nnz, 0, bits, st));
+    cudaFreeAsync(tmp, st);
+    ks = k1;
+  } else if (nnz) {
+    CKR(cudaMemcpyAsync(orr, r, sizeof(float) * nnz, cudaMemcpyDeviceToDevice, st));
+  }
+  if (nnz) {
+    block_decode_kernel<<<grid_for(nnz), kT, 0, st>>>(g, bounds, ks, nnz, ou, ov);
+    CKR(cudaGetLastError());
+  }
+  block_off_kernel<<<grid_for(nblk + 1), kT, 0, st>>>(ks, nnz, g.bu + g.bv, nblk, block_off);
+  CKR(cudaGetLastError());
+  cudaFreeAsync(k0, st);
+  cudaFreeAsync(k1, st);
+  return cudaGetLastError();
+}
+
+cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, int64_t nb, int64_t target,
+                          int64_t** task_lo, int64_t** task_hi, int64_t* n_tasks, cudaStream_t st) {
+  *n_tasks = 0;
+  *task_lo = nullptr;
+  *task_hi = nullptr;
+  if (nrec == 0) {
+    CKR(cudaMalloc(task_lo, sizeof(int64_t)));
+    CKR(cudaMalloc(task_hi, sizeof(int64_t)));
+    return cudaSuccess;
+  }
+  unsigned char* flag = nullptr;
+  int64_t* runs = nullptr;
+  int64_t* nsel = nullptr;
+  CKR(dalloc(&flag, nrec, st));
+  CKR(dalloc(&runs, nrec, st));
+  CKR(dalloc(&nsel, 1, st));
+  run_flag_kernel<<<grid_for(nrec), kT, 0, st>>>(ru, nrec, flag);
+  block_start_flag_kernel<<<grid_for(nb), kT, 0, st>>>(off, nb, nrec, flag);
+  CKR(cudaGetLastError());
+  size_t tb = 0;
+  void* tmp = nullptr;
+  thrust::counting_iterator<int64_t> it(0);
+  CKR(cub::DeviceSelect::Flagged(nullptr, tb, it, flag, runs, nsel, nrec, st));
+  CKR(cudaMallocAsync(&tmp, tb, st));
+  CKR(cub::DeviceSelect::Flagged(tmp, tb, it, flag, runs, nsel, nrec, st));
+  cudaFreeAsync(tmp, st);
+  int64_t nruns = 0;
+  CKR(cudaMemcpyAsync(&nruns, nsel, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+  CKR(cudaStreamSynchronize(st));
+
+  // candidates per block
+  int64_t *ccnt = nullptr, *coff = nullptr;
+  CKR(dalloc(&ccnt, nb + 1, st));
+  CKR(dalloc(&coff, nb + 1, st));
+  CKR(cudaMemsetAsync(ccnt, 0, sizeof(int64_t) * (nb + 1), st));
+  cand_count_kernel<<<grid_for(nb), kT, 0, st>>>(off, nb, target, ccnt);
+  CKR(cudaGetLastError());
+  tb = 0;
+  CKR(cub::DeviceScan::ExclusiveSum(nullptr, tb, ccnt, coff, nb + 1, st));
+  CKR(cudaMallocAsync(&tmp, tb, st));
+  CKR(cub::DeviceScan::ExclusiveSum(tmp, tb, ccnt, coff, nb + 1, st));
+  cudaFreeAsync(tmp, st);
+  int64_t ncand = 0;
+  CKR(cudaMemcpyAsync(&ncand, coff + nb, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+  CKR(cudaStreamSynchronize(st));
+
+  int64_t* cpos = nullptr;
+  unsigned char* keep = nullptr;
+  int64_t* lo = nullptr;
+  CKR(dalloc(&cpos, ncand, st));
+  CKR(dalloc(&keep, ncand, st));
+  CKR(dalloc(&lo, ncand, st));
+  cand_map_kernel<<<grid_for(ncand), kT, 0, st>>>(coff, nb, ncand, off, target, runs, nruns, cpos, keep);
+  CKR(cudaGetLastError());
+  tb = 0;
+  CKR(cub::DeviceSelect::Flagged(nullptr, tb, cpos, keep, lo, nsel, ncand, st));
+  CKR(cudaMallocAsync(&tmp, tb, st));
+  CKR(cub::DeviceSelect::Flagged(tmp, tb, cpos, keep, lo, nsel, ncand, st));
+  cudaFreeAsync(tmp, st);
+  int64_t nt = 0;
+  CKR(cudaMemcpyAsync(&nt, nsel, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+  CKR(cudaStreamSynchronize(st));
+
+  int64_t* hi = nullptr;
+  uint64_t *sk0 = nullptr, *sk1 = nullptr;
+  int64_t *ix0 = nullptr, *ix1 = nullptr;
+  CKR(dalloc(&hi, nt, st));
+  CKR(dalloc(&sk0, nt, st));
+  CKR(dalloc(&sk1, nt, st));
+  CKR(dalloc(&ix0, nt, st));
+  CKR(dalloc(&ix1, nt, st));
+  task_hi_kernel<<<grid_for(nt), kT, 0, st>>>(lo, nt, off, nb, hi, sk0, ix0);
+  CKR(cudaGetLastError());
+  tb = 0;
+  CKR(cub::DeviceRadixSort::SortPairs(nullptr, tb, sk0, sk1, ix0, ix1, nt, 0, 64, st));
+  CKR(cudaMallocAsync(&tmp, tb, st));
+  CKR(cub::DeviceRadixSort::SortPairs(tmp, tb, sk0, sk1, ix0, ix1, nt, 0, 64, st));
+  cudaFreeAsync(tmp, st);
+  CKR(cudaMalloc(task_lo, sizeof(int64_t) * (nt ? nt : 1)));
+  CKR(cudaMalloc(task_hi, sizeof(int64_t) * (nt ? nt : 1)));
+  permute_tasks_kernel<<<grid_for(nt), kT, 0, st>>>(ix1, nt, lo, hi, *task_lo, *task_hi);
+  CKR(cudaGetLastError());
+  for (void* p : {(void*)flag, (void*)runs, (void*)nsel, (void*)ccnt, (void*)coff, (void*)cpos, (void*)keep,
+                  (void*)lo, (void*)hi, (void*)sk0, (void*)sk1, (void*)ix0, (void*)ix1})
+    cudaFreeAsync(p, st);
+  CKR(cudaStreamSynchronize(st));
+  *n_tasks = nt;
+  return cudaSuccess;
+}
+
+}  // namespace hccmf

@@ -1,0 +1,183 @@
+// eval.cu -- a0 factor init, a8 RMSE, a9 export (un-permute), Q replica average.
+#include "internal.cuh"
+
+namespace hccmf {
+namespace {
+
+constexpr int kT = 256;
+
+inline unsigned grid_for(int64_t n, int64_t cap = 148LL * 64) {
+  int64_t b = (n + kT - 1) / kT;
+  if (b < 1) b = 1;
+  if (b > cap) b = cap;
+  return (unsigned)b;
+}
+
+// a0 (R5): X[perm[i]][j] = U(H(seed, tag, i, j)) * sqrtf(1/k), original id i
+__global__ void init_kernel(uint64_t seed, uint64_t tag, int64_t rows_total, int32_t k, const int32_t* perm,
+                            int64_t row0, int64_t rows, float* X) {
+  const float sc = sqrtf(1.0f / (float)k);
+  const int64_t total = rows_total * k;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = e / k;
+    const int32_t j = (int32_t)(e - i * k);
+    const int64_t pr = (int64_t)perm[i] - row0;
+    if (pr < 0 || pr >= rows) continue;
+    X[pr * k + j] = uniform24(hash4(seed, tag, (uint64_t)i, (uint64_t)j)) * sc;
+  }
+}
+
+__global__ void scatter_kernel(const float4* src, int64_t rows_total, int32_t k4, const int32_t* perm, int64_t row0,
+                               int64_t rows, float4* dst) {
+  const int64_t total = rows_total * k4;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = e / k4;
+    const int32_t j = (int32_t)(e - i * k4);
+    const int64_t pr = (int64_t)perm[i] - row0;
+    if (pr < 0 || pr >= rows) continue;
+    dst[pr * k4 + j] = src[e];
+  }
+}
+
+__global__ void gather_kernel(const float4* src, int64_t rows_total, int32_t k4, const int32_t* perm, int64_t row0,
+                              float4* dst) {
+  const int64_t total = rows_total * k4;
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < total; e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = e / k4;
+    const int32_t j = (int32_t)(e - i * k4);
+    dst[e] = src[((int64_t)perm[i] - row0) * k4 + j];
+  }
+}
+
+// a8: one rating group of L lanes per test rating (same lane mapping as the SGD
+// kernel), fp32 dot product, squared error accumulated in fp64 per group in a
+// fixed order, then a fixed-order tree per CTA -> partials[blockIdx].
+template <int L>
+__global__ void __launch_bounds__(kT) rmse_kernel(const int32_t* __restrict__ tu, const int32_t* __restrict__ tv,
+                                                  const float* __restrict__ tr, int64_t nt,
+                                                  const int32_t* __restrict__ perm_row,
+                                                  const int32_t* __restrict__ perm_col, const float* __restrict__ P,
+                                                  int64_t row0, int64_t rows, const float* __restrict__ Q, int32_t k,
+                                                  double* partials) {
+  constexpr unsigned FM = 0xffffffffu;
+  const int lane = threadIdx.x & 31;
+  const int sl = lane & (L - 1);
+  const int64_t group = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / L;
+  const int64_t ngroups = (int64_t)gridDim.x * blockDim.x / L;
+  double acc = 0.0, cnt = 0.0;
+  const int64_t iters = (nt + ngroups - 1) / ngroups;
+  for (int64_t it = 0; it < iters; ++it) {
+    const int64_t i = it * ngroups + group;
+    const bool in = i < nt;
+    int64_t up = -1, vp = 0;
+    float rv = 0.f;
+    if (in) {
+      up = (int64_t)perm_row[tu[i]] - row0;
+      vp = perm_col[tv[i]];
+      rv = tr[i];
+    }
+    const bool act = in && up >= 0 && up < rows;
+    float d = 0.f;
+    if (act) {
+      for (int c = sl * 4; c < k; c += 4 * L) {
+        const float4 p = *reinterpret_cast<const float4*>(P + up * k + c);
+        const float4 q = *reinterpret_cast<const float4*>(Q + vp * k + c);
+        d = fmaf(p.x, q.x, d);
+        d = fmaf(p.y, q.y, d);
+        d = fmaf(p.z, q.z, d);
+        d = fmaf(p.w, q.w, d);
+      }
+    }
+#pragma unroll
+    for (int o = L / 2; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
+    if (act && sl == 0) {
+      const double e = (double)rv - (double)d;
+      acc += e * e;
+      cnt += 1.0;
+    }
+  }
+  __shared__ double sa[kT], sc[kT];
+  sa[threadIdx.x] = acc;
+  sc[threadIdx.x] = cnt;
+  __syncthreads();
+  for (int s = kT / 2; s > 0; s >>= 1) {
+    if (threadIdx.x < s) {
+      sa[threadIdx.x] += sa[threadIdx.x + s];
+      sc[threadIdx.x] += sc[threadIdx.x + s];
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    partials[2 * blockIdx.x] = sa[0];
+    partials[2 * blockIdx.x + 1] = sc[0];
+  }
+}
+
+__global__ void rmse_final_kernel(const double* partials, int nb, double* out2) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    double s = 0.0, c = 0.0;
+    for (int b = 0; b < nb; ++b) {
+      s += partials[2 * b];
+      c += partials[2 * b + 1];
+    }
+    out2[0] = s;
+    out2[1] = c;
+  }
+}
+
+__global__ void average_kernel(const float* reps, int32_t G, int64_t count, float* out) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < count; e += (int64_t)gridDim.x * blockDim.x) {
+    double s = 0.0;
+    for (int g = 0; g < G; ++g) s += (double)reps[(int64_t)g * count + e];
+    out[e] = (float)(s / (double)G);
+  }
+}
+
+}  // namespace
+
+cudaError_t k_init_factors(uint64_t seed, uint64_t tag, int64_t rows_total, int32_t k, const int32_t* perm,
+                           int64_t row0, int64_t rows, float* X, cudaStream_t st) {
+  if (rows_total == 0) return cudaSuccess;
+  init_kernel<<<grid_for(rows_total * k), kT, 0, st>>>(seed, tag, rows_total, k, perm, row0, rows, X);
+  return cudaGetLastError();
+}
+
+cudaError_t k_scatter_rows(const float* src, int64_t rows_total, int32_t k, const int32_t* perm, int64_t row0,
+                           int64_t rows, float* dst, cudaStream_t st) {
+  const int32_t k4 = k / 4;
+  scatter_kernel<<<grid_for(rows_total * k4), kT, 0, st>>>(reinterpret_cast<const float4*>(src), rows_total, k4,
+                                                           perm, row0, rows, reinterpret_cast<float4*>(dst));
+  return cudaGetLastError();
+}
+
+cudaError_t k_gather_rows(const float* src, int64_t rows_total, int32_t k, const int32_t* perm, int64_t row0,
+                          float* dst, cudaStream_t st) {
+  const int32_t k4 = k / 4;
+  gather_kernel<<<grid_for(rows_total * k4), kT, 0, st>>>(reinterpret_cast<const float4*>(src), rows_total, k4, perm,
+                                                          row0, reinterpret_cast<float4*>(dst));
+  return cudaGetLastError();
+}
+
+cudaError_t k_rmse(const int32_t* tu, const int32_t* tv, const float* tr, int64_t nt, const int32_t* perm_row,
+                   const int32_t* perm_col, const float* P, int64_t row0, int64_t rows, const float* Q, int32_t k,
+                   double* partials, double* out2, cudaStream_t st) {
+  const int L = lanes_per_rating(k);
+  switch (L) {
+#define RM(LL)                                                                                                    \
+  case LL:                                                                                                        \
+    rmse_kernel<LL><<<RMSE_BLOCKS, kT, 0, st>>>(tu, tv, tr, nt, perm_row, perm_col, P, row0, rows, Q, k, partials); \
+    break;
+    RM(1) RM(2) RM(4) RM(8) RM(16) RM(32)
+#undef RM
+    default: return cudaErrorInvalidValue;
+  }
+  rmse_final_kernel<<<1, 32, 0, st>>>(partials, RMSE_BLOCKS, out2);
+  return cudaGetLastError();
+}
+
+cudaError_t k_average(const float* reps, int32_t G, int64_t count, float* out, cudaStream_t st) {
+  average_kernel<<<grid_for(count), kT, 0, st>>>(reps, G, count, out);
+  return cudaGetLastError();
+}
+
+}  // namespace hccmf

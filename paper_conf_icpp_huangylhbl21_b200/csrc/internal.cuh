@@ -1,0 +1,163 @@
+// internal.cuh -- shared declarations of libhccmf (product path; no oracle code).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "hccmf.h"
+
+namespace hccmf {
+
+// ------------------------------------------------------------------ hashing
+// DESIGN.md R8: SplitMix64 finaliser (Steele, Lea, Flood 2014) and the
+// counter-based hash H(seed, tag, a, b) = sm(sm(sm(seed ^ tag<<56) ^ a) ^ b).
+__host__ __device__ __forceinline__ uint64_t splitmix(uint64_t x) {
+  uint64_t z = x + 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+__host__ __device__ __forceinline__ uint64_t hash4(uint64_t seed, uint64_t tag, uint64_t a, uint64_t b) {
+  return splitmix(splitmix(splitmix(seed ^ (tag << 56)) ^ a) ^ b);
+}
+// 24-bit uniform in [0,1): exact in fp32.
+__host__ __device__ __forceinline__ float uniform24(uint64_t h) {
+  return (float)(uint32_t)(h >> 40) * (1.0f / 16777216.0f);
+}
+
+// --------------------------------------------------------------- SGD plans
+// One kernel launch of the SGD kernel: tasks [t0, t0+nt) of the plan's task
+// arrays, against Q replica `qrep` (logical all-reduce) ; `stage` = ring stage.
+struct Launch {
+  int64_t t0, nt;
+  int32_t qrep;
+  int32_t stage;
+};
+
+struct Plan {
+  int sched = -1, sync = -1;
+  int64_t* d_lo = nullptr;  // record ranges [lo, hi) in local record indices
+  int64_t* d_hi = nullptr;
+  int64_t n_tasks = 0;
+  std::vector<Launch> launches;
+  int32_t n_stages = 1;
+};
+
+struct SgdArgs {
+  const int32_t* __restrict__ ru;
+  const int32_t* __restrict__ rv;
+  const float* __restrict__ rr;
+  float* P;         // local P rows [row0, row0 + rows)
+  float* Q;         // n x k (or one replica)
+  int64_t row0;
+  int32_t k;
+  float gamma, lambda;
+  const int64_t* __restrict__ task_lo;
+  const int64_t* __restrict__ task_hi;
+  int64_t n_tasks;
+  unsigned long long* counter;
+};
+
+// launch the SGD kernel for a list of tasks; warps = concurrent warps wanted
+cudaError_t launch_sgd(const SgdArgs& a, int64_t warps, cudaStream_t st);
+// sub-warp width used for k (lanes per rating)
+int lanes_per_rating(int k);
+
+// ---------------------------------------------------------------- blocker
+struct BlockGeom {  // a4 block geometry for the bit-exact sort key
+  int32_t G, Br, Bc;
+  int64_t m, n;
+  int32_t bu, bv, bb;  // key bits: local row, local col, block id
+};
+
+cudaError_t k_validate(const int32_t* u, const int32_t* v, const float* r, int64_t nnz, int64_t m,
+                       int64_t n, unsigned int* flag, cudaStream_t st);
+cudaError_t k_perm(uint64_t seed, uint64_t tag, int64_t count, int32_t* perm, cudaStream_t st);
+cudaError_t k_row_prefix(const int32_t* u, int64_t nnz, const int32_t* perm_row, int64_t m,
+                         unsigned long long* S /* m+1 */, cudaStream_t st);
+cudaError_t k_bound_search(const unsigned long long* S, int64_t m, const int64_t* targets, int32_t nt,
+                           int64_t* out, cudaStream_t st);
+cudaError_t k_block_sort(const BlockGeom& g, const int32_t* bounds, const int32_t* perm_row,
+                         const int32_t* perm_col, const int32_t* u, const int32_t* v, const float* r,
+                         int64_t nnz, int32_t* ou, int32_t* ov, float* orr, int64_t* block_off,
+                         cudaStream_t st);
+cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* blk_off_local /*nb+1, local idx*/,
+                          int64_t nb, int64_t target, int64_t** task_lo, int64_t** task_hi, int64_t* n_tasks,
+                          cudaStream_t st);
+
+// ------------------------------------------------------------ eval/export
+cudaError_t k_init_factors(uint64_t seed, uint64_t tag, int64_t rows_total, int32_t k, const int32_t* perm,
+                           int64_t row0, int64_t rows, float* X, cudaStream_t st);
+cudaError_t k_scatter_rows(const float* src /*orig order*/, int64_t rows_total, int32_t k, const int32_t* perm,
+                           int64_t row0, int64_t rows, float* dst, cudaStream_t st);
+cudaError_t k_gather_rows(const float* src /*permuted, local*/, int64_t rows_total, int32_t k,
+                          const int32_t* perm, int64_t row0, float* dst /*orig order*/, cudaStream_t st);
+cudaError_t k_rmse(const int32_t* tu, const int32_t* tv, const float* tr, int64_t nt, const int32_t* perm_row,
+                   const int32_t* perm_col, const float* P, int64_t row0, int64_t rows, const float* Q, int32_t k,
+                   double* partials /*2*RMSE_BLOCKS*/, double* out2 /*sum, count*/, cudaStream_t st);
+cudaError_t k_average(const float* reps, int32_t G, int64_t count, float* out, cudaStream_t st);
+constexpr int RMSE_BLOCKS = 592;
+
+}  // namespace hccmf
+
+// ------------------------------------------------------------- the handle
+struct hccmf_ctx {
+  int64_t m = 0, n = 0;
+  int32_t k = 0;
+  float gamma = 0.f, lambda = 0.f;
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int32_t rank = 0, world = 1;
+  ncclComm_t comm = nullptr;
+  int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
+  hccmf_status sticky = HCCMF_OK;
+  std::string err;
+  int64_t opt_warps = 0, opt_task = 256;
+  bool sync_stream = true;
+  size_t device_bytes = 0;
+
+  // a1 input (global COO, device)
+  int64_t nnz = 0;
+  int32_t* d_in_u = nullptr;
+  int32_t* d_in_v = nullptr;
+  float* d_in_r = nullptr;
+
+  // a2-a4
+  int32_t G = 1, Br = 1, Bc = 1;
+  uint64_t seed = 0;
+  std::vector<double> x;
+  std::vector<int32_t> bounds;     // G+1
+  std::vector<int64_t> block_off;  // global, G*Br*Bc+1
+  hccmf::BlockGeom geom{};
+  int32_t* d_perm_row = nullptr;
+  int32_t* d_perm_col = nullptr;
+  int32_t shard_lo = 0, shard_hi = 1;
+  int64_t rec0 = 0, local_nnz = 0;
+  int32_t* d_u = nullptr;  // sorted local records (permuted ids)
+  int32_t* d_v = nullptr;
+  float* d_r = nullptr;
+  int64_t blk0 = 0, nblk_local = 0;   // first local block, count
+  std::vector<int64_t> blk_task_off;  // nblk_local+1 into base tasks
+  int64_t n_tasks = 0;
+  int64_t* d_task_lo = nullptr;
+  int64_t* d_task_hi = nullptr;
+  std::vector<int64_t> h_task_lo, h_task_hi;  // host copies for plan building
+
+  // factors
+  int64_t row0 = 0, rows = 0;
+  float* d_P = nullptr;
+  float* d_Q = nullptr;
+  float* d_Qrep = nullptr;  // logical all-reduce replicas
+  unsigned long long* d_counters = nullptr;
+  int64_t n_counters = 0;
+  double* d_partials = nullptr;
+  double* d_scalar = nullptr;
+
+  int q_ring_sched = -1;  // >= 0: distributed ring left only this rank's Q group valid
+  std::vector<hccmf::Plan> plans;
+};
