@@ -21,8 +21,8 @@
  *  - Factor layout: P is m x k row-major fp32 (p_u contiguous); Q is n x k
  *    row-major fp32 (q_v contiguous) -- this is the paper's k x n item matrix Q
  *    (Table 1) TRANSPOSED.
- *  - Input pointers may be host or device memory (classified with
- *    cudaPointerGetAttributes).  The library COPIES inputs; the caller keeps
+ *  - Input pointers may be host or device memory (resolved through unified
+ *    virtual addressing, cudaMemcpyDefault).  The library COPIES inputs; the caller keeps
  *    ownership and may free them when the call returns.  Output pointers are
  *    caller-allocated, host or device.  The handle owns all device memory it
  *    allocates; hccmf_destroy frees it.
@@ -124,7 +124,19 @@ typedef enum {
                                     256); tasks never split a user's run          */
     HCCMF_OPT_SYNC_STREAM = 3,   /* 1 (default): calls return after the stream is
                                     synchronised; 0: return after enqueueing      */
-    HCCMF_OPT_RING_SUBBLOCKS = 4 /* reserved                                       */
+    HCCMF_OPT_RING_SUBBLOCKS = 4,/* reserved                                       */
+    HCCMF_OPT_HOGWILD_ATOMIC = 5,/* 1 (default): Hogwild applies q_v increments with
+                                    vector atomic adds (Hogwild!'s component-wise
+                                    atomic model, no lost updates); 0: plain stores
+                                    (racing writers may overwrite: the paper's
+                                    "coverage", L1680-L1686)                      */
+    HCCMF_OPT_CONFLICT_RATIO = 6,/* auto Hogwild concurrency: at most n / value
+                                    rating groups in flight (default 4; 0 = no cap) */
+    HCCMF_OPT_HEAVY_FIRST = 7    /* Hogwild task order inside a block: tasks with more
+                                    than `value` ratings run first, longest first;
+                                    the rest keep the shuffled user order.  -1
+                                    (default): shuffled order only; 0: pure LPT.
+                                    Takes effect at the next hccmf_partition.     */
 } hccmf_option;
 
 /* ------------------------------------------------------------------ lifecycle */

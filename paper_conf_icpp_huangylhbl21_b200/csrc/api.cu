@@ -290,11 +290,20 @@ hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
   return HCCMF_OK;
 }
 
+// Hogwild concurrency (R14): the number of rating groups in flight sets
+// the staleness of q_v reads, so it is capped at n / opt_conflict groups, and at 32
+// resident warps per SM.
 int64_t auto_warps(hccmf_t h) {
   if (h->opt_warps > 0) return h->opt_warps;
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
-  return (int64_t)sms * 32;
+  int64_t w = (int64_t)sms * 32;
+  if (h->opt_conflict > 0) {
+    const int64_t groups_per_warp = 32 / lanes_per_rating(h->k);
+    const int64_t cap = std::max<int64_t>(1, (h->n / h->opt_conflict) / groups_per_warp);
+    w = std::min(w, cap);
+  }
+  return w;
 }
 
 // column-group row range [a, b) of Q for ring group g
@@ -417,6 +426,16 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
       h->sync_stream = value != 0;
       return HCCMF_OK;
     case HCCMF_OPT_RING_SUBBLOCKS:
+      return HCCMF_OK;
+    case HCCMF_OPT_HOGWILD_ATOMIC:
+      h->opt_atomic = value != 0;
+      return HCCMF_OK;
+    case HCCMF_OPT_HEAVY_FIRST:
+      h->opt_heavy = value;
+      return HCCMF_OK;
+    case HCCMF_OPT_CONFLICT_RATIO:
+      if (value < 0) return fail(h, HCCMF_EINVAL, "conflict ratio must be >= 0");
+      h->opt_conflict = value;
       return HCCMF_OK;
     default:
       return fail(h, HCCMF_EINVAL, "unknown option %d", option);
@@ -611,7 +630,7 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   CU(h, cudaMallocAsync((void**)&dLoc, sizeof(int64_t) * (h->nblk_local + 1), st));
   CU(h, cudaMemcpyAsync(dLoc, loc_off.data(), sizeof(int64_t) * (h->nblk_local + 1), cudaMemcpyHostToDevice, st));
   int64_t nt = 0;
-  CU(h, k_build_tasks(h->d_u, h->local_nnz, dLoc, h->nblk_local, h->opt_task, &h->d_task_lo, &h->d_task_hi, &nt, st));
+  CU(h, k_build_tasks(h->d_u, h->local_nnz, dLoc, h->nblk_local, h->opt_task, h->opt_heavy, &h->d_task_lo, &h->d_task_hi, &nt, st));
   h->device_bytes += 2 * sizeof(int64_t) * (nt ? nt : 1);
   h->n_tasks = nt;
   cudaFreeAsync(dLoc, st);
@@ -699,6 +718,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   a.k = h->k;
   a.gamma = h->gamma;
   a.lambda = h->lambda;
+  a.atomic_q = (sched == HCCMF_SCHED_HOGWILD && h->opt_atomic) ? 1 : 0;
   const int L = lanes_per_rating(h->k);
   const int64_t hog_warps = auto_warps(h);
   int stage = 0;

@@ -214,17 +214,19 @@ __global__ void cand_map_kernel(const int64_t* cand_off, int64_t nb, int64_t nca
   }
 }
 
-__global__ void task_hi_kernel(const int64_t* lo, int64_t nt, const int64_t* off, int64_t nb, int64_t* hi,
-                               uint64_t* sortkey, int64_t* idx) {
+__global__ void task_hi_kernel(const int64_t* lo, int64_t nt, const int64_t* off, int64_t nb, int64_t heavy,
+                               int64_t* hi, uint64_t* sortkey, int64_t* idx) {
   for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nt; t += (int64_t)gridDim.x * blockDim.x) {
     const int64_t j = upper_bound_i64(off, nb + 1, lo[t]) - 1;
     int64_t h = off[j + 1];
     if (t + 1 < nt && lo[t + 1] < h) h = lo[t + 1];
     hi[t] = h;
-    // LPT inside each block: ascending (block, -len)
+    // inside each block: tasks longer than `heavy` first, longest first (LPT),
+    // then the rest in record order (the shuffled user order); heavy < 0: none
     const uint64_t len = (uint64_t)(h - lo[t]);
+    const bool is_heavy = heavy >= 0 && (int64_t)len > heavy;
     const uint64_t inv = (len >= (1ull << 38)) ? 0 : ((1ull << 38) - 1 - len);
-    sortkey[t] = ((uint64_t)j << 38) | inv;
+    sortkey[t] = ((uint64_t)j << 39) | (is_heavy ? inv : ((1ull << 38) | (uint64_t)t));
     idx[t] = t;
   }
 }
@@ -348,7 +350,7 @@ cudaError_t k_block_sort(const BlockGeom& g, const int32_t* bounds, const int32_
 }
 
 cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, int64_t nb, int64_t target,
-                          int64_t** task_lo, int64_t** task_hi, int64_t* n_tasks, cudaStream_t st) {
+                          int64_t heavy, int64_t** task_lo, int64_t** task_hi, int64_t* n_tasks, cudaStream_t st) {
   *n_tasks = 0;
   *task_lo = nullptr;
   *task_hi = nullptr;
@@ -418,7 +420,7 @@ cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, i
   CKR(dalloc(&sk1, nt, st));
   CKR(dalloc(&ix0, nt, st));
   CKR(dalloc(&ix1, nt, st));
-  task_hi_kernel<<<grid_for(nt), kT, 0, st>>>(lo, nt, off, nb, hi, sk0, ix0);
+  task_hi_kernel<<<grid_for(nt), kT, 0, st>>>(lo, nt, off, nb, heavy, hi, sk0, ix0);
   CKR(cudaGetLastError());
   tb = 0;
   CKR(cub::DeviceRadixSort::SortPairs(nullptr, tb, sk0, sk1, ix0, ix1, nt, 0, 64, st));

@@ -60,6 +60,7 @@ struct SgdArgs {
   const int64_t* __restrict__ task_hi;
   int64_t n_tasks;
   unsigned long long* counter;
+  int32_t atomic_q;  // Hogwild: apply q_v increments with vector atomics
 };
 
 // launch the SGD kernel for a list of tasks; warps = concurrent warps wanted
@@ -86,7 +87,7 @@ cudaError_t k_block_sort(const BlockGeom& g, const int32_t* bounds, const int32_
                          int64_t nnz, int32_t* ou, int32_t* ov, float* orr, int64_t* block_off,
                          cudaStream_t st);
 cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* blk_off_local /*nb+1, local idx*/,
-                          int64_t nb, int64_t target, int64_t** task_lo, int64_t** task_hi, int64_t* n_tasks,
+                          int64_t nb, int64_t target, int64_t heavy, int64_t** task_lo, int64_t** task_hi, int64_t* n_tasks,
                           cudaStream_t st);
 
 // ------------------------------------------------------------ eval/export
@@ -117,7 +118,7 @@ struct hccmf_ctx {
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_warps = 0, opt_task = 256;
+  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 4, opt_heavy = -1;
   bool sync_stream = true;
   size_t device_bytes = 0;
 

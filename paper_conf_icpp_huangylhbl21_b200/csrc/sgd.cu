@@ -48,12 +48,28 @@ __device__ __forceinline__ void store_row(float* row, const float4 (&x)[VEC], in
   }
 }
 
+// Hogwild! (Recht et al., the paper's ref [21], L216-L219) applies each update as
+// atomic component-wise additions: q_v += delta with one 128-bit vector reduction
+// per lane (red.global.add.v4.f32, sm_90+), so racing groups never lose an update
+// -- only read a slightly stale q_v.
+template <int L, int VEC, bool FULL>
+__device__ __forceinline__ void red_row(float* row, const float4 (&d)[VEC], int sl, int k) {
+#pragma unroll
+  for (int i = 0; i < VEC; ++i) {
+    const int c = (i * L + sl) * 4;
+    if (FULL || c < k)
+      asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(row + c), "f"(d[i].x),
+                   "f"(d[i].y), "f"(d[i].z), "f"(d[i].w)
+                   : "memory");
+  }
+}
+
 __device__ __forceinline__ float upd(float a, float b, float e, float g, float lam) {
   // a + gamma * (e * b - lambda * a)
   return a + g * (e * b - lam * a);
 }
 
-template <int L, int VEC, bool FULL>
+template <int L, int VEC, bool FULL, bool ATOMIC>
 __global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
   constexpr unsigned FM = 0xffffffffu;
   const int lane = threadIdx.x & 31;
@@ -66,9 +82,10 @@ __global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
   int wu = 0, wv = 0;
   float wr = 0.f;
   int cu = -1;
-  float4 p[VEC];
+  int lastv = -1;  // q_v forwarding: the item this group updated last and its new value
+  float4 p[VEC], lastq[VEC];
 #pragma unroll
-  for (int i = 0; i < VEC; ++i) p[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int i = 0; i < VEC; ++i) p[i] = lastq[i] = make_float4(0.f, 0.f, 0.f, 0.f);
 
   while (true) {
     // ---- task queue: one atomic per rating group, broadcast inside the group
@@ -83,6 +100,7 @@ __global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
         cur = a.task_lo[t];
         end = a.task_hi[t];
         have_win = false;
+        lastv = -1;
       } else {
         done = true;
       }
@@ -115,7 +133,12 @@ __global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
         load_row<L, VEC, FULL>(a.P + (int64_t)(uu - a.row0) * k, p, sl, k);
         cu = uu;
       }
-      load_row<L, VEC, FULL>(a.Q + (int64_t)vv * k, q, sl, k);
+      if (vv == lastv) {  // consecutive ratings of one item (duplicates): serial read-after-write
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) q[i] = lastq[i];
+      } else {
+        load_row<L, VEC, FULL>(a.Q + (int64_t)vv * k, q, sl, k);
+      }
 #pragma unroll
       for (int i = 0; i < VEC; ++i) {
         d = fmaf(p[i].x, q[i].x, d);
@@ -135,10 +158,17 @@ __global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
         const float4 pp = p[i], qq = q[i];
         p[i] = make_float4(upd(pp.x, qq.x, e, g, lam), upd(pp.y, qq.y, e, g, lam),
                            upd(pp.z, qq.z, e, g, lam), upd(pp.w, qq.w, e, g, lam));
-        q[i] = make_float4(upd(qq.x, pp.x, e, g, lam), upd(qq.y, pp.y, e, g, lam),
-                           upd(qq.z, pp.z, e, g, lam), upd(qq.w, pp.w, e, g, lam));
+        // increment gamma (e p_old - lambda q); ATOMIC adds it with a vector red
+        const float4 dq = make_float4(g * (e * pp.x - lam * qq.x), g * (e * pp.y - lam * qq.y),
+                                      g * (e * pp.z - lam * qq.z), g * (e * pp.w - lam * qq.w));
+        lastq[i] = make_float4(qq.x + dq.x, qq.y + dq.y, qq.z + dq.z, qq.w + dq.w);
+        q[i] = ATOMIC ? dq : lastq[i];
       }
-      store_row<L, VEC, FULL>(a.Q + (int64_t)vv * k, q, sl, k);
+      lastv = vv;
+      if (ATOMIC)
+        red_row<L, VEC, FULL>(a.Q + (int64_t)vv * k, q, sl, k);
+      else
+        store_row<L, VEC, FULL>(a.Q + (int64_t)vv * k, q, sl, k);
       ++cur;
     }
   }
@@ -151,7 +181,10 @@ cudaError_t launch_t(const SgdArgs& a, int64_t warps, cudaStream_t st) {
   int64_t w = warps < need_warps ? warps : need_warps;
   if (w < 1) return cudaSuccess;
   const int64_t blocks = (w * 32 + kThreads - 1) / kThreads;
-  sgd_kernel<L, VEC, FULL><<<(unsigned)blocks, kThreads, 0, st>>>(a);
+  if (a.atomic_q)
+    sgd_kernel<L, VEC, FULL, true><<<(unsigned)blocks, kThreads, 0, st>>>(a);
+  else
+    sgd_kernel<L, VEC, FULL, false><<<(unsigned)blocks, kThreads, 0, st>>>(a);
   return cudaGetLastError();
 }
 
