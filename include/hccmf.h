@@ -132,11 +132,14 @@ typedef enum {
                                     "coverage", L1680-L1686)                      */
     HCCMF_OPT_CONFLICT_RATIO = 6,/* auto Hogwild concurrency: at most n / value
                                     rating groups in flight (default 4; 0 = no cap) */
-    HCCMF_OPT_HEAVY_FIRST = 7    /* Hogwild task order inside a block: tasks with more
+    HCCMF_OPT_HEAVY_FIRST = 7,   /* Hogwild task order inside a block: tasks with more
                                     than `value` ratings run first, longest first;
                                     the rest keep the shuffled user order.  -1
                                     (default): shuffled order only; 0: pure LPT.
                                     Takes effect at the next hccmf_partition.     */
+    HCCMF_OPT_VEC = 8            /* float4 slots of p_u / q_v per lane (1, 2, 4; 0 =
+                                    auto: k/32 clamped to [1, 4]); sets the lanes
+                                    per rating L = k / (4 VEC)                    */
 } hccmf_option;
 
 /* ------------------------------------------------------------------ lifecycle */
@@ -223,6 +226,20 @@ HCCMF_API hccmf_status hccmf_get_records(hccmf_t h, int32_t* u, int32_t* v, floa
 HCCMF_API hccmf_status hccmf_get_fractions(hccmf_t h, double* x);
 
 HCCMF_API hccmf_status hccmf_get_info(hccmf_t h, hccmf_info* out);
+
+/* Host-only (no device needed): the a5-a7 schedule that shard `shard` of a
+ * distributed handle executes (shard = -1: all G logical shards of one handle).
+ * Launch i runs blocks[launch_off[i] .. launch_off[i+1]) (block index
+ * (s*Br + rb)*Bc + cb) concurrently at ring stage launch_stage[i]; blocks of one
+ * launch share no P rows and no Q columns (DET) or no users (HOGWILD).  For RING,
+ * ring[4t .. 4t+3] = Q rows [send_lo, send_hi) the shard sends to shard-1 after
+ * stage t and [recv_lo, recv_hi) it receives from shard+1 (R19).
+ * Size query: pass blocks or launch_off NULL (or too small *n_blocks /
+ * *n_launches): the required counts are written and HCCMF_OK returned.
+ * launch_off needs *n_launches + 1 entries; ring needs 4*G. */
+HCCMF_API hccmf_status hccmf_schedule(int32_t G, int32_t Br, int32_t Bc, int64_t n, int32_t sched, int32_t sync,
+                                      int32_t shard, int64_t* blocks, int64_t* n_blocks, int64_t* launch_off,
+                                      int32_t* launch_stage, int64_t* n_launches, int64_t* ring);
 
 /* Library version string, e.g. "hccmf 0.1 sm_100a". */
 HCCMF_API const char* hccmf_version(void);

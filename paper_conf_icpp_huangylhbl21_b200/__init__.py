@@ -23,7 +23,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libhccmf.so")
+LIB_PATH = os.environ.get("HCCMF_LIB") or os.path.join(_HERE, "libhccmf.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is not built; run `python -c 'import __graft_entry__ as g; g.build()'` "
@@ -34,7 +34,7 @@ STATUS = {0: "OK", -1: "EINVAL", -2: "ERANGE", -3: "ENOMEM", -4: "ESTATE", -5: "
 SCHED = {"det": 0, "hogwild": 1}
 SYNC = {"none": 0, "ring": 1, "allreduce": 2}
 DP = {"DP0": 0, "DP1": 1, "DP2": 2}
-OPT = {"hogwild_warps": 1, "task_ratings": 2, "sync_stream": 3, "hogwild_atomic": 5, "conflict_ratio": 6, "heavy_first": 7}
+OPT = {"hogwild_warps": 1, "task_ratings": 2, "sync_stream": 3, "hogwild_atomic": 5, "conflict_ratio": 6, "heavy_first": 7, "vec": 8}
 
 
 class HccmfError(RuntimeError):
@@ -90,6 +90,7 @@ def lib():
             "hccmf_get_fractions": (st, [P, P]),
             "hccmf_get_info": (st, [P, ctypes.POINTER(Info)]),
             "hccmf_version": (ctypes.c_char_p, []),
+            "hccmf_schedule": (st, [i32, i32, i32, i64, i32, i32, i32, P, P, P, P, P, P]),
         }
         for name, (res, args) in sig.items():
             fn = getattr(L, name)
@@ -118,6 +119,26 @@ def _buf(x, dtype):
         pass
     a = np.ascontiguousarray(x, dtype=dtype)
     return a.ctypes.data, a
+
+
+def schedule(G, Br, Bc, n, sched="det", sync="none", shard=-1):
+    """The launch/block schedule (and ring exchange ranges) one shard executes; host-only."""
+    L = lib()
+    nb, nl = ctypes.c_int64(0), ctypes.c_int64(0)
+    code = L.hccmf_schedule(G, Br, Bc, n, SCHED[sched], SYNC[sync], shard, None, ctypes.byref(nb), None, None,
+                            ctypes.byref(nl), None)
+    if code != OK:
+        raise HccmfError(code, L.hccmf_last_error(None).decode())
+    blocks = np.empty(nb.value, np.int64)
+    off = np.empty(nl.value + 1, np.int64)
+    stage = np.empty(nl.value, np.int32)
+    ring = np.zeros((G, 4), np.int64)
+    code = L.hccmf_schedule(G, Br, Bc, n, SCHED[sched], SYNC[sync], shard, blocks.ctypes.data, ctypes.byref(nb),
+                            off.ctypes.data, stage.ctypes.data, ctypes.byref(nl), ring.ctypes.data)
+    if code != OK:
+        raise HccmfError(code, L.hccmf_last_error(None).decode())
+    launches = [blocks[off[i]:off[i + 1]] for i in range(nl.value)]
+    return launches, stage, ring
 
 
 class Model:

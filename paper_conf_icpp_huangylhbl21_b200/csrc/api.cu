@@ -193,84 +193,112 @@ void free_partition(hccmf_t h) {
 }
 
 // ------------------------------------------------------------ SGD plans
+// The a5/a6/a7 schedule as block lists (pure host logic, also exported through
+// hccmf_schedule so multi-process tests can run it without a device):
+// launches in order; blocks inside one launch share no P rows and no Q columns
+// (DET) or no users (HOGWILD), so running them concurrently is the serial
+// order of DESIGN.md R19.
+struct BlockLaunch {
+  std::vector<int64_t> blocks;
+  int32_t qrep, stage;
+};
+
+const char* schedule_blocks(int G, int Br, int Bc, int sched, int sync, int shard_lo, int shard_hi,
+                            std::vector<BlockLaunch>& out, int* n_stages) {
+  out.clear();
+  *n_stages = 1;
+  auto blk = [&](int64_t s, int64_t rb, int64_t cb) { return (s * Br + rb) * Bc + cb; };
+  const int eff_sync = (G == 1) ? HCCMF_SYNC_NONE : sync;
+  if (eff_sync == HCCMF_SYNC_NONE && G != 1) return "sync NONE needs n_shards == 1";
+  if (sched == HCCMF_SCHED_DET) {
+    if (eff_sync == HCCMF_SYNC_RING) {
+      if (Bc != G * Br) return "DET+RING needs grid_cols == n_shards * grid_rows";
+      const int c = Br;
+      *n_stages = G;
+      for (int t = 0; t < G; ++t)
+        for (int t2 = 0; t2 < c; ++t2) {
+          BlockLaunch L{{}, 0, t};
+          for (int s = shard_lo; s < shard_hi; ++s) {
+            const int g = (s + t) % G;
+            for (int i = 0; i < c; ++i) L.blocks.push_back(blk(s, i, (int64_t)g * c + (i + t2) % c));
+          }
+          out.push_back(L);
+        }
+    } else {
+      if (Br != Bc) return "DET needs grid_rows == grid_cols (sync NONE/ALLREDUCE)";
+      const int c = Br;
+      for (int s = shard_lo; s < shard_hi; ++s)
+        for (int t2 = 0; t2 < c; ++t2) {
+          BlockLaunch L{{}, s - shard_lo, 0};
+          for (int i = 0; i < c; ++i) L.blocks.push_back(blk(s, i, (i + t2) % c));
+          out.push_back(L);
+        }
+    }
+  } else {
+    if (eff_sync == HCCMF_SYNC_RING) {
+      if (Bc % G != 0) return "HOGWILD+RING needs grid_cols % n_shards == 0";
+      const int c = Bc / G;
+      *n_stages = G;
+      for (int t = 0; t < G; ++t)
+        for (int j = 0; j < c; ++j) {
+          BlockLaunch L{{}, 0, t};
+          for (int s = shard_lo; s < shard_hi; ++s) {
+            const int g = (s + t) % G;
+            for (int rb = 0; rb < Br; ++rb) L.blocks.push_back(blk(s, rb, (int64_t)g * c + j));
+          }
+          out.push_back(L);
+        }
+    } else {
+      // column-block-major phases: a user's p_u is touched by one task per launch
+      for (int s = shard_lo; s < shard_hi; ++s)
+        for (int cb = 0; cb < Bc; ++cb) {
+          BlockLaunch L{{}, s - shard_lo, 0};
+          for (int rb = 0; rb < Br; ++rb) L.blocks.push_back(blk(s, rb, cb));
+          out.push_back(L);
+        }
+    }
+  }
+  return nullptr;
+}
+
+// Q rows [a, b) of ring column group g (columns of column blocks [g c, (g+1) c))
+void ring_cols(int64_t n, int G, int Br, int Bc, int sched, int g, int64_t* a, int64_t* b) {
+  const int c = (sched == HCCMF_SCHED_DET) ? Br : Bc / G;
+  *a = ceil_div((int64_t)g * c * n, Bc);
+  *b = ceil_div((int64_t)(g + 1) * c * n, Bc);
+}
+
 hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
   for (auto& p : h->plans)
     if (p.sched == sched && p.sync == sync) {
       *out = &p;
       return HCCMF_OK;
     }
-  const int G = h->G, Br = h->Br, Bc = h->Bc;
+  std::vector<BlockLaunch> bl;
   Plan pl;
   pl.sched = sched;
   pl.sync = sync;
+  const char* msg = schedule_blocks(h->G, h->Br, h->Bc, sched, sync, h->shard_lo, h->shard_hi, bl, &pl.n_stages);
+  if (msg) return fail(h, HCCMF_EINVAL, "%s", msg);
   std::vector<int64_t> lo, hi;
-  auto local_off = [&](int64_t blk) { return h->block_off[blk] - h->rec0; };
-  auto add_block_det = [&](int64_t blk) {
-    const int64_t a = local_off(blk), b = local_off(blk + 1);
-    if (b > a) {
-      lo.push_back(a);
-      hi.push_back(b);
-    }
-  };
-  auto add_block_hog = [&](int64_t blk) {
-    const int64_t j = blk - h->blk0;
-    for (int64_t t = h->blk_task_off[j]; t < h->blk_task_off[j + 1]; ++t) {
-      lo.push_back(h->h_task_lo[t]);
-      hi.push_back(h->h_task_hi[t]);
-    }
-  };
-  auto close_launch = [&](int64_t& t0, int32_t qrep, int32_t stage) {
-    const int64_t nt = (int64_t)lo.size() - t0;
-    pl.launches.push_back(Launch{t0, nt, qrep, stage});
-    t0 = (int64_t)lo.size();
-  };
-  int64_t t0 = 0;
-  const bool G1 = (G == 1);
-  const int eff_sync = G1 ? HCCMF_SYNC_NONE : sync;
-  if (eff_sync == HCCMF_SYNC_NONE && !G1) return fail(h, HCCMF_EINVAL, "sync NONE needs n_shards == 1");
-  if (sched == HCCMF_SCHED_DET) {
-    if (eff_sync == HCCMF_SYNC_RING) {
-      if (Bc != G * Br) return fail(h, HCCMF_EINVAL, "DET+RING needs grid_cols == n_shards * grid_rows");
-      const int c = Br;
-      pl.n_stages = G;
-      for (int t = 0; t < G; ++t)
-        for (int t2 = 0; t2 < c; ++t2) {
-          for (int s = h->shard_lo; s < h->shard_hi; ++s) {
-            const int g = (s + t) % G;
-            for (int i = 0; i < c; ++i) add_block_det(blk_index(h, s, i, (int64_t)g * c + (i + t2) % c));
-          }
-          close_launch(t0, 0, t);
+  for (const BlockLaunch& L : bl) {
+    const int64_t t0 = (int64_t)lo.size();
+    for (int64_t b : L.blocks) {
+      if (sched == HCCMF_SCHED_DET) {  // one task per non-empty block
+        const int64_t a = h->block_off[b] - h->rec0, e = h->block_off[b + 1] - h->rec0;
+        if (e > a) {
+          lo.push_back(a);
+          hi.push_back(e);
         }
-    } else {
-      if (Br != Bc) return fail(h, HCCMF_EINVAL, "DET needs grid_rows == grid_cols (sync NONE/ALLREDUCE)");
-      const int c = Br;
-      for (int s = h->shard_lo; s < h->shard_hi; ++s)
-        for (int t2 = 0; t2 < c; ++t2) {
-          for (int i = 0; i < c; ++i) add_block_det(blk_index(h, s, i, (i + t2) % c));
-          close_launch(t0, s - h->shard_lo, 0);
+      } else {  // the block's user-aligned tasks
+        const int64_t j = b - h->blk0;
+        for (int64_t t = h->blk_task_off[j]; t < h->blk_task_off[j + 1]; ++t) {
+          lo.push_back(h->h_task_lo[t]);
+          hi.push_back(h->h_task_hi[t]);
         }
+      }
     }
-  } else {
-    if (eff_sync == HCCMF_SYNC_RING) {
-      if (Bc % G != 0) return fail(h, HCCMF_EINVAL, "HOGWILD+RING needs grid_cols %% n_shards == 0");
-      const int c = Bc / G;
-      pl.n_stages = G;
-      for (int t = 0; t < G; ++t)
-        for (int j = 0; j < c; ++j) {
-          for (int s = h->shard_lo; s < h->shard_hi; ++s) {
-            const int g = (s + t) % G;
-            for (int rb = 0; rb < Br; ++rb) add_block_hog(blk_index(h, s, rb, (int64_t)g * c + j));
-          }
-          close_launch(t0, 0, t);
-        }
-    } else {
-      // column-block-major phases: a user's p_u is touched by one task per launch
-      for (int s = h->shard_lo; s < h->shard_hi; ++s)
-        for (int cb = 0; cb < Bc; ++cb) {
-          for (int rb = 0; rb < Br; ++rb) add_block_hog(blk_index(h, s, rb, cb));
-          close_launch(t0, s - h->shard_lo, 0);
-        }
-    }
+    pl.launches.push_back(Launch{t0, (int64_t)lo.size() - t0, L.qrep, L.stage});
   }
   pl.n_tasks = (int64_t)lo.size();
   CU(h, dmalloc(h, &pl.d_lo, pl.n_tasks));
@@ -299,7 +327,7 @@ int64_t auto_warps(hccmf_t h) {
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
   int64_t w = (int64_t)sms * 32;
   if (h->opt_conflict > 0) {
-    const int64_t groups_per_warp = 32 / lanes_per_rating(h->k);
+    const int64_t groups_per_warp = 32 / sgd_lanes(h->k, (int)h->opt_vec);
     const int64_t cap = std::max<int64_t>(1, (h->n / h->opt_conflict) / groups_per_warp);
     w = std::min(w, cap);
   }
@@ -308,9 +336,7 @@ int64_t auto_warps(hccmf_t h) {
 
 // column-group row range [a, b) of Q for ring group g
 void ring_group_cols(hccmf_t h, int sched, int g, int64_t* a, int64_t* b) {
-  const int c = (sched == HCCMF_SCHED_DET) ? h->Br : h->Bc / h->G;
-  *a = col_start(h, (int64_t)g * c);
-  *b = col_start(h, (int64_t)(g + 1) * c);
+  ring_cols(h->n, h->G, h->Br, h->Bc, sched, g, a, b);
 }
 
 hccmf_status ring_exchange(hccmf_t h, int sched, int t) {
@@ -429,6 +455,10 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
       return HCCMF_OK;
     case HCCMF_OPT_HOGWILD_ATOMIC:
       h->opt_atomic = value != 0;
+      return HCCMF_OK;
+    case HCCMF_OPT_VEC:
+      if (value != 0 && value != 1 && value != 2 && value != 4) return fail(h, HCCMF_EINVAL, "vec must be 0, 1, 2 or 4");
+      h->opt_vec = value;
       return HCCMF_OK;
     case HCCMF_OPT_HEAVY_FIRST:
       h->opt_heavy = value;
@@ -719,7 +749,8 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   a.gamma = h->gamma;
   a.lambda = h->lambda;
   a.atomic_q = (sched == HCCMF_SCHED_HOGWILD && h->opt_atomic) ? 1 : 0;
-  const int L = lanes_per_rating(h->k);
+  a.vec_pref = (int32_t)h->opt_vec;
+  const int L = sgd_lanes(h->k, (int)h->opt_vec);
   const int64_t hog_warps = auto_warps(h);
   int stage = 0;
   for (size_t li = 0; li < pl->launches.size(); ++li) {
@@ -867,6 +898,38 @@ hccmf_status hccmf_get_fractions(hccmf_t h, double* x) {
   if (h->state < 2) return fail(h, HCCMF_ESTATE, "get_fractions needs partition");
   if (!x) return fail(h, HCCMF_EINVAL, "x is NULL");
   memcpy(x, h->x.data(), sizeof(double) * h->x.size());
+  return HCCMF_OK;
+}
+
+hccmf_status hccmf_schedule(int32_t G, int32_t Br, int32_t Bc, int64_t n, int32_t sched, int32_t sync, int32_t shard,
+                            int64_t* blocks, int64_t* n_blocks, int64_t* launch_off, int32_t* launch_stage,
+                            int64_t* n_launches, int64_t* ring) {
+  if (G < 1 || Br < 1 || Bc < 1 || n < 1 || !n_blocks || !n_launches || shard < -1 || shard >= G)
+    return fail(nullptr, HCCMF_EINVAL, "bad schedule arguments");
+  const int lo = shard < 0 ? 0 : shard, hi = shard < 0 ? G : shard + 1;
+  std::vector<BlockLaunch> bl;
+  int n_stages = 1;
+  const char* msg = schedule_blocks(G, Br, Bc, sched, sync, lo, hi, bl, &n_stages);
+  if (msg) return fail(nullptr, HCCMF_EINVAL, "%s", msg);
+  int64_t nb = 0;
+  for (const auto& L : bl) nb += (int64_t)L.blocks.size();
+  const int64_t cap_b = *n_blocks, cap_l = *n_launches;
+  *n_blocks = nb;
+  *n_launches = (int64_t)bl.size();
+  if (!blocks || !launch_off || cap_b < nb || cap_l < (int64_t)bl.size()) return HCCMF_OK;  // size query
+  int64_t k = 0;
+  for (size_t i = 0; i < bl.size(); ++i) {
+    launch_off[i] = k;
+    if (launch_stage) launch_stage[i] = bl[i].stage;
+    for (int64_t b : bl[i].blocks) blocks[k++] = b;
+  }
+  launch_off[bl.size()] = k;
+  if (ring && sync == HCCMF_SYNC_RING && G > 1)
+    for (int t = 0; t < G; ++t) {
+      const int s = lo;
+      ring_cols(n, G, Br, Bc, sched, (s + t) % G, &ring[4 * t + 0], &ring[4 * t + 1]);
+      ring_cols(n, G, Br, Bc, sched, (s + t + 1) % G, &ring[4 * t + 2], &ring[4 * t + 3]);
+    }
   return HCCMF_OK;
 }
 

@@ -61,11 +61,15 @@ struct SgdArgs {
   int64_t n_tasks;
   unsigned long long* counter;
   int32_t atomic_q;  // Hogwild: apply q_v increments with vector atomics
+  int32_t vec_pref;  // float4 slots per lane (0 = auto)
 };
 
 // launch the SGD kernel for a list of tasks; warps = concurrent warps wanted
 cudaError_t launch_sgd(const SgdArgs& a, int64_t warps, cudaStream_t st);
-// sub-warp width used for k (lanes per rating)
+// lane geometry of the SGD kernel: L lanes per rating group, VEC float4 per lane
+void sgd_geometry(int k, int vec_pref, int* L, int* VEC);
+int sgd_lanes(int k, int vec_pref);
+// lanes per rating of the RMSE kernel (one float4 per lane)
 int lanes_per_rating(int k);
 
 // ---------------------------------------------------------------- blocker
@@ -118,7 +122,7 @@ struct hccmf_ctx {
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 4, opt_heavy = -1;
+  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 4, opt_heavy = -1, opt_vec = 0;
   bool sync_stream = true;
   size_t device_bytes = 0;
 

@@ -245,6 +245,7 @@ def test_hogwild_single_group_is_the_serial_oracle(pkg, orc, atomic, k):
     mdl.load(u, v, r)
     mdl.partition(1, (1, 1), seed=3)
     mdl.set_option("hogwild_warps", 1)
+    mdl.set_option("vec", k // 128)  # 32 lanes per rating: one group in the one warp
     mdl.set_option("hogwild_atomic", atomic)
     mdl.set_factors(P0, Q0)
     for _ in range(2):

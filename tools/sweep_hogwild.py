@@ -26,6 +26,8 @@ ap.add_argument("--warps", default="148,592,1184,2368,4736")
 ap.add_argument("--atomic", default="0,1")
 ap.add_argument("--task", type=int, default=256)
 ap.add_argument("--grid", default="1,1")
+ap.add_argument("--vec", default="0")
+ap.add_argument("--repeat", type=int, default=1)
 ap.add_argument("--every", action="store_true", help="test RMSE after every epoch")
 args = ap.parse_args()
 cfg = synth.CONFIGS[args.config]
@@ -40,8 +42,10 @@ mdl.set_option("task_ratings", args.task)
 mdl.load(u, v, r)
 mdl.partition(1, (Br, Bc), seed=cfg.seed)
 dtu, dtv, dtr = (torch.from_numpy(x).cuda() for x in (tu, tv, tr))
-for at in (int(x) for x in args.atomic.split(",")):
-    for w in (int(x) for x in args.warps.split(",")):
+for at, vec, w in [(a_, v_, w_) for a_ in (int(x) for x in args.atomic.split(","))
+                   for v_ in (int(x) for x in args.vec.split(",")) for w_ in (int(x) for x in args.warps.split(",")) for _ in range(args.repeat)]:
+    if True:
+        mdl.set_option("vec", vec)
         mdl.set_option("hogwild_atomic", at)
         mdl.set_option("hogwild_warps", w)
         mdl.init(1)
@@ -57,5 +61,5 @@ for at in (int(x) for x in args.atomic.split(",")):
                 rms.append(round(mdl.rmse(dtu, dtv, dtr), 5))
         rm = rms[-1]
         tmin = min(ts[1:] if len(ts) > 1 else ts)
-        print(json.dumps({"config": cfg.name, "atomic": at, "warps": w, "epoch_ms": tmin,
+        print(json.dumps({"config": cfg.name, "atomic": at, "vec": vec, "warps": w, "epoch_ms": tmin,
                           "gupd_s": cfg.nnz / tmin / 1e6, "test_rmse": rm, "per_epoch": rms}), flush=True)
