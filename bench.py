@@ -48,6 +48,7 @@ def parse():
     ap.add_argument("--grid", default=None, help="Br,Bc (default: hogwild 1,G ; det 64,64*G)")
     ap.add_argument("--warps", type=int, default=0)
     ap.add_argument("--task", type=int, default=0)
+    ap.add_argument("--vec", type=int, default=0, help="float4 slots per lane (0 = library auto)")
     ap.add_argument("--impl", default="hccmf", choices=["hccmf", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -212,6 +213,8 @@ def main():
         mdl.set_option("hogwild_warps", args.warps)
     if args.task:
         mdl.set_option("task_ratings", args.task)
+    if args.vec:
+        mdl.set_option("vec", args.vec)
     du, dv, dr = (torch.from_numpy(x).cuda() for x in (u, v, r))
     dtu, dtv, dtr = (torch.from_numpy(x).cuda() for x in (tu, tv, tr))
     torch.cuda.synchronize()
@@ -302,6 +305,8 @@ def main():
             m2.set_stream(stream)
             if args.warps:
                 m2.set_option("hogwild_warps", args.warps)
+            if args.vec:
+                m2.set_option("vec", args.vec)
             m2.load(pin[0], pin[1], pin[2])
             m2.partition(G, (Br, Bc), "DP0", seed=cfg.seed)
             m2.init(1)

@@ -133,13 +133,15 @@ typedef enum {
     HCCMF_OPT_CONFLICT_RATIO = 6,/* auto Hogwild concurrency: at most n / value
                                     rating groups in flight (default 4; 0 = no cap) */
     HCCMF_OPT_HEAVY_FIRST = 7,   /* Hogwild task order inside a block: tasks with more
-                                    than `value` ratings run first, longest first;
-                                    the rest keep the shuffled user order.  -1
-                                    (default): shuffled order only; 0: pure LPT.
+                                    than `value` ratings run first, longest first
+                                    (no late heavy user stretches the epoch); the
+                                    rest keep the shuffled user order.  Default
+                                    1024; -1: shuffled order only; 0: pure LPT.
                                     Takes effect at the next hccmf_partition.     */
     HCCMF_OPT_VEC = 8            /* float4 slots of p_u / q_v per lane (1, 2, 4; 0 =
-                                    auto: k/32 clamped to [1, 4]); sets the lanes
-                                    per rating L = k / (4 VEC)                    */
+                                    auto: k/128 clamped to [1, 4], i.e. one rating
+                                    per warp from k = 128); lanes per rating
+                                    L = min(32, k / (4 VEC))                      */
 } hccmf_option;
 
 /* ------------------------------------------------------------------ lifecycle */

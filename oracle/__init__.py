@@ -55,7 +55,7 @@ def lib():
             "orc_dp2": (None, [i32, P, P, f64, P]),
             "orc_row_prefix": (None, [i64, i64, P, P, P]),
             "orc_bounds": (None, [i64, i64, P, i32, P, P]),
-            "orc_block_sort": (ctypes.c_int, [i64, i64, i64, P, P, P, i32, i32, i32, P, P, P, P, P, P, P]),
+            "orc_block_sort": (ctypes.c_int, [i64, i64, i64, P, P, P, i32, i32, i32, P, P, P, u64, P, P, P, P]),
             "orc_init": (None, [u64, i64, i64, i32, P, P, P, P]),
             "orc_sgd_update": (f64, [i32, f64, f64, P, P, f64]),
             "orc_run": (None, [i64, i64, i32, f64, f64, P, P, P, P, P]),
@@ -153,7 +153,7 @@ def bounds(m: int, nnz: int, S, G: int, x) -> np.ndarray:
     return b
 
 
-def block_sort(m, n, u, v, r, G, Br, Bc, b, perm_row, perm_col):
+def block_sort(m, n, u, v, r, G, Br, Bc, b, perm_row, perm_col, seed=0):
     u, v, r = _i32(u), _i32(v), _f32(r)
     b, pr, pc = _i32(b), _i32(perm_row), _i32(perm_col)
     nnz = len(u)
@@ -161,7 +161,7 @@ def block_sort(m, n, u, v, r, G, Br, Bc, b, perm_row, perm_col):
     ov = np.empty(nnz, np.int32)
     orr = np.empty(nnz, np.float32)
     off = np.empty(G * Br * Bc + 1, np.int64)
-    rc = lib().orc_block_sort(m, n, nnz, _p(u), _p(v), _p(r), G, Br, Bc, _p(b), _p(pr), _p(pc),
+    rc = lib().orc_block_sort(m, n, nnz, _p(u), _p(v), _p(r), G, Br, Bc, _p(b), _p(pr), _p(pc), seed,
                               _p(ou), _p(ov), _p(orr), _p(off))
     assert rc == 0
     return ou, ov, orr, off
@@ -230,7 +230,7 @@ class Problem:
         self.x = np.full(G, 1.0 / G) if x is None else _f64(x)
         self.b = bounds(m, len(self.u), self.S, G, self.x)
         self.ru, self.rv, self.rr, self.off = block_sort(m, n, self.u, self.v, self.r, G, Br, Bc, self.b,
-                                                         self.perm_row, self.perm_col)
+                                                         self.perm_row, self.perm_col, seed)
         self.P = None
         self.Q = None
 

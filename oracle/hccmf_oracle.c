@@ -215,10 +215,14 @@ void orc_bounds(int64_t m, int64_t nnz, const int64_t* S, int32_t G, const doubl
 /* Blocking + stable sort (L546 "sorting", L1472-L1474 row-sorted blocks).      */
 /* Record i goes to shard s (b_s <= u' < b_{s+1}), row block                     */
 /* rb = floor((u'-b_s) * Br / (b_{s+1}-b_s)), column block cb = floor(v' * Bc / n),*/
-/* and records are ordered by (s, rb, cb, u', v', i).                            */
+/* and records are ordered by (s, rb, cb, u', o, i) where o orders a row's       */
+/* ratings inside the block: the block's columns [c0, c1), c0 = ceil(cb n / Bc), */
+/* rotated by a row-dependent offset (R21):                            */
+/*   o = (v' - c0 + rot(u')) mod (c1 - c0),  rot(u') = H(seed, 5, u', 0) mod (c1 - c0) */
+/* seed 0: rot = 0, plain column order.                                          */
 /* off[((s*Br + rb)*Bc + cb)] = first record of the block; off has G*Br*Bc+1.    */
 /* ------------------------------------------------------------------------- */
-typedef struct { int64_t blk; int32_t up, vp; int64_t i; } orc_rec;
+typedef struct { int64_t blk; int32_t up; int64_t o; int64_t i; } orc_rec;
 
 static int cmp_rec(const void* a, const void* b)
 {
@@ -226,14 +230,14 @@ static int cmp_rec(const void* a, const void* b)
     const orc_rec* y = (const orc_rec*)b;
     if (x->blk != y->blk) return x->blk < y->blk ? -1 : 1;
     if (x->up != y->up) return x->up < y->up ? -1 : 1;
-    if (x->vp != y->vp) return x->vp < y->vp ? -1 : 1;
+    if (x->o != y->o) return x->o < y->o ? -1 : 1;
     if (x->i != y->i) return x->i < y->i ? -1 : 1;
     return 0;
 }
 
 int orc_block_sort(int64_t m, int64_t n, int64_t nnz, const int32_t* u, const int32_t* v,
                    const float* r, int32_t G, int32_t Br, int32_t Bc, const int32_t* b,
-                   const int32_t* perm_row, const int32_t* perm_col, int32_t* out_u,
+                   const int32_t* perm_row, const int32_t* perm_col, uint64_t seed, int32_t* out_u,
                    int32_t* out_v, float* out_r, int64_t* off)
 {
     int64_t nblk = (int64_t)G * Br * Bc;
@@ -246,9 +250,11 @@ int orc_block_sort(int64_t m, int64_t n, int64_t nnz, const int32_t* u, const in
         int64_t rows = (int64_t)b[s + 1] - b[s];
         int64_t rb = ((int64_t)(up - b[s]) * Br) / rows;
         int64_t cb = ((int64_t)vp * Bc) / n;
+        int64_t c0 = (cb * n + Bc - 1) / Bc, c1 = ((cb + 1) * n + Bc - 1) / Bc, w = c1 - c0;
+        int64_t rot = seed ? (int64_t)(orc_hash(seed, 5, (uint64_t)up, 0) % (uint64_t)w) : 0;
         a[i].blk = ((int64_t)s * Br + rb) * Bc + cb;
         a[i].up = up;
-        a[i].vp = vp;
+        a[i].o = (vp - c0 + rot) % w;
         a[i].i = i;
     }
     qsort(a, (size_t)nnz, sizeof(orc_rec), cmp_rec);
@@ -257,7 +263,7 @@ int orc_block_sort(int64_t m, int64_t n, int64_t nnz, const int32_t* u, const in
     for (int64_t j = 0; j < nblk; ++j) off[j + 1] += off[j];
     for (int64_t j = 0; j < nnz; ++j) {
         out_u[j] = a[j].up;
-        out_v[j] = a[j].vp;
+        out_v[j] = perm_col[v[a[j].i]];
         out_r[j] = r[a[j].i];
     }
     free(a);

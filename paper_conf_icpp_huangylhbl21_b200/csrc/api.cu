@@ -161,10 +161,6 @@ void plan_dp2(int G, std::vector<double>& x, const double* t, double t_sync) {  
   for (int s = 0; s < G; ++s) x[s] = y[s] / sum;
 }
 
-// first column of column block cb
-int64_t col_start(const hccmf_t h, int64_t cb) { return ceil_div(cb * h->n, h->Bc); }
-
-int64_t blk_index(const hccmf_t h, int64_t s, int64_t rb, int64_t cb) { return (s * h->Br + rb) * h->Bc + cb; }
 
 void free_partition(hccmf_t h) {
   for (auto& p : h->plans) {
@@ -600,6 +596,7 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   g.bu = bitlen((uint64_t)(maxr - 1));
   g.bv = bitlen((uint64_t)(ceil_div(n, h->Bc) - 1));
   g.bb = bitlen((uint64_t)(nblk - 1));
+  g.seed = h->seed;
   if (g.bb + g.bu + g.bv > 64) return fail(h, HCCMF_ERANGE, "sort key needs %d > 64 bits", g.bb + g.bu + g.bv);
   h->geom = g;
   int32_t *su = nullptr, *sv = nullptr;

@@ -114,8 +114,12 @@ __global__ void block_key_kernel(BlockGeom g, const int32_t* __restrict__ bounds
     const int64_t rstart = ceil_div(rb * rows, g.Br);
     const int64_t cb = ((int64_t)vp * g.Bc) / g.n;
     const int64_t cstart = ceil_div(cb * g.n, g.Bc);
+    const int64_t w = ceil_div((cb + 1) * g.n, g.Bc) - cstart;
+    // a row's ratings inside a block start at a row-dependent column (R21): Hogwild
+    // groups that start together do not sweep the same items in lock step
+    const int64_t rot = g.seed ? (int64_t)(hash4(g.seed, 5, (uint64_t)up, 0) % (uint64_t)w) : 0;
     const uint64_t blk = (uint64_t)(((int64_t)s * g.Br + rb) * g.Bc + cb);
-    keys[i] = (blk << (g.bu + g.bv)) | ((uint64_t)(l - rstart) << g.bv) | (uint64_t)(vp - cstart);
+    keys[i] = (blk << (g.bu + g.bv)) | ((uint64_t)(l - rstart) << g.bv) | (uint64_t)((vp - cstart + rot) % w);
   }
 }
 
@@ -136,8 +140,11 @@ __global__ void block_decode_kernel(BlockGeom g, const int32_t* __restrict__ bou
     const int64_t rows = (int64_t)bounds[s + 1] - bounds[s];
     const int64_t rstart = ceil_div(rb * rows, g.Br);
     const int64_t cstart = ceil_div(cb * g.n, g.Bc);
-    ou[i] = (int32_t)(bounds[s] + rstart + lu);
-    ov[i] = (int32_t)(cstart + lv);
+    const int64_t w = ceil_div((cb + 1) * g.n, g.Bc) - cstart;
+    const int64_t up = bounds[s] + rstart + lu;
+    const int64_t rot = g.seed ? (int64_t)(hash4(g.seed, 5, (uint64_t)up, 0) % (uint64_t)w) : 0;
+    ou[i] = (int32_t)up;
+    ov[i] = (int32_t)(cstart + (lv + w - rot) % w);
   }
 }
 

@@ -77,6 +77,7 @@ struct BlockGeom {  // a4 block geometry for the bit-exact sort key
   int32_t G, Br, Bc;
   int64_t m, n;
   int32_t bu, bv, bb;  // key bits: local row, local col, block id
+  uint64_t seed;       // row-dependent column rotation inside a block (R21)
 };
 
 cudaError_t k_validate(const int32_t* u, const int32_t* v, const float* r, int64_t nnz, int64_t m,
@@ -122,7 +123,7 @@ struct hccmf_ctx {
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 4, opt_heavy = -1, opt_vec = 0;
+  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 4, opt_heavy = 1024, opt_vec = 0;
   bool sync_stream = true;
   size_t device_bytes = 0;
 

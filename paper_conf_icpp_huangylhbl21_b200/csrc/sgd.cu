@@ -5,22 +5,24 @@
 //   p_u = p_u + gamma (e q_v - lambda p_u)
 //   q_v = q_v + gamma (e p_u - lambda q_v)      (p_u: value before the update, R1)
 //
-// B200 design (DESIGN.md section 5):
-//  * a "rating group" of L lanes (L = next pow2 of k/4, <= 32) owns one rating at a
-//    time; lane l holds the float4 slices (v*L + l) of p_u and q_v, so every
-//    factor access is a coalesced 128-bit load/store.  k = 128 -> one rating per
-//    warp (L = 32); k = 32 -> four independent rating groups per warp (L = 8).
-//  * the dot product is reduced with log2(L) __shfl_xor_sync steps.
-//  * a persistent grid pulls tasks (record ranges [lo, hi)) from an atomic
-//    queue.  Hogwild tasks are runs of whole users (never split), so p_u is
-//    carried in registers across a user's ratings and written back once;
-//    q_v races between groups by design (Hogwild!, L216-L219, L1680-L1691).
-//    DET tasks are FPSGD blocks of one stratum, which share no rows or columns.
-//  * records are read once per epoch with streaming loads (L rating triples per
-//    coalesced window, broadcast by shuffles); P/Q go through L2 only (.cg), so a
-//    racing group never reads a stale line from its own SM's L1.
-//  * rating groups of a warp run in lock step (no divergent shuffles).
+// B200 design (DESIGN.md section 6):
+//  * a "rating group" of L lanes owns one rating at a time; lane l holds VEC float4
+//    slots (elements (i*L + l)*4 ..) of p_u and q_v, so every factor access is a
+//    coalesced 128-bit load/store/red.  k = 128 -> L = 16, VEC = 2 (two groups per
+//    warp, lock step); the dot product is 4 FMA chains + log2(L) shuffles.
+//  * a persistent grid pulls tasks (record ranges [lo, hi)) from an atomic queue.
+//    Hogwild tasks are runs of whole users, so p_u stays in registers across a
+//    user's ratings; DET tasks are the blocks of one stratum (no shared rows or
+//    columns).  q_v increments are vector reductions (Hogwild!, L216-L219).
+//  * software pipeline, one rating deep: while rating j is updated the record of
+//    j+1 is taken from a double-buffered coalesced window and q_{v(j+1)} (and on a
+//    user change p_{u(j+1)}) is already in flight.  The loop body is unrolled twice
+//    with the current / next q registers swapping roles (no register copies);
+//    q_{v(j+1)} == q_{v(j)} is forwarded from registers (serial read-after-write).
+//  * 32-bit row offsets and a compile-time full-vector geometry keep the per-rating
+//    instruction count low (profiles/).
 #include <algorithm>
+#include <type_traits>
 
 #include "internal.cuh"
 
@@ -29,102 +31,104 @@ namespace {
 
 constexpr int kThreads = 256;
 
-// per-lane slice validity: slot i of lane sl holds elements (i*L + sl)*4 .. +3
-template <int L, int VEC>
-__device__ __forceinline__ void load_row(const float* row, float4 (&x)[VEC], const bool (&ok)[VEC], int sl) {
-#pragma unroll
-  for (int i = 0; i < VEC; ++i)
-    x[i] = ok[i] ? __ldcg(reinterpret_cast<const float4*>(row + (i * L + sl) * 4)) : make_float4(0.f, 0.f, 0.f, 0.f);
-}
+template <int VEC>
+struct Row {
+  float4 x[VEC];
+};
 
-template <int L, int VEC>
-__device__ __forceinline__ void store_row(float* row, const float4 (&x)[VEC], const bool (&ok)[VEC], int sl) {
-#pragma unroll
-  for (int i = 0; i < VEC; ++i)
-    if (ok[i]) __stcg(reinterpret_cast<float4*>(row + (i * L + sl) * 4), x[i]);
-}
-
-// Hogwild! (Recht et al., the paper's ref [21], L216-L219) applies each update as
-// atomic component-wise additions: q_v += delta with one 128-bit vector reduction
-// per slot (red.global.add.v4.f32, sm_90+), so racing groups never lose an update
-// -- they only read a slightly stale q_v.
-template <int L, int VEC>
-__device__ __forceinline__ void red_row(float* row, const float4 (&d)[VEC], const bool (&ok)[VEC], int sl) {
-#pragma unroll
-  for (int i = 0; i < VEC; ++i)
-    if (ok[i]) {
-#ifdef HCCMF_SCALAR_RED
-      float* r4 = row + (i * L + sl) * 4;
-      atomicAdd(r4 + 0, d[i].x);
-      atomicAdd(r4 + 1, d[i].y);
-      atomicAdd(r4 + 2, d[i].z);
-      atomicAdd(r4 + 3, d[i].w);
-#else
-      asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(row + (i * L + sl) * 4),
-                   "f"(d[i].x), "f"(d[i].y), "f"(d[i].z), "f"(d[i].w)
-                   : "memory");
-#endif
-    }
-}
-
-// One kernel for both schedules.  Per rating group (L lanes, lock step inside the
-// warp) the loop is software-pipelined one rating deep:
-//   iteration j: take rating j+1 from the record window, issue the loads of
-//   q_{v(j+1)} and (on a user change) p_{u(j+1)}, then update rating j.
-// Hazards: q_{v(j+1)} == q_{v(j)} is forwarded from registers (the serial
-// read-after-write), p rows are owned by the group for the whole task.  Record
-// windows (WR ratings, coalesced) are double-buffered; the next task id is
-// fetched one task ahead.
-template <int L, int VEC, bool ATOMIC>
-__global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
-  constexpr unsigned FM = 0xffffffffu;
-  constexpr int RPL = L >= 8 ? 1 : 8 / L;  // records per lane per window
-  constexpr int WR = L * RPL;              // records per window
-  const int lane = threadIdx.x & 31;
-  const int sl = lane & (L - 1);
-  const int k = a.k;
-  const float g = a.gamma;
-  const float c1 = 1.f - a.gamma * a.lambda;  // p' = c1 p + (g e) q
-  const float gl = a.gamma * a.lambda;        // dq = (g e) p - (g lambda) q
-  const int32_t* __restrict__ ru = a.ru;
-  const int32_t* __restrict__ rv = a.rv;
-  const float* __restrict__ rr = a.rr;
-  float* __restrict__ P = a.P;
-  float* __restrict__ Q = a.Q;
+// Per-lane view of a factor row: slot i of lane sl is float4 index (i*L + sl).
+template <int L, int VEC, bool FULL>
+struct Lanes {
   bool ok[VEC];
+  __device__ __forceinline__ void init(int sl, int k4) {
 #pragma unroll
-  for (int i = 0; i < VEC; ++i) ok[i] = (i * L + sl) * 4 < k;
+    for (int i = 0; i < VEC; ++i) ok[i] = FULL || (i * L + sl) < k4;
+  }
+  __device__ __forceinline__ void load(const float4* row, Row<VEC>& r) const {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) r.x[i] = (FULL || ok[i]) ? __ldcg(row + i * L) : make_float4(0.f, 0.f, 0.f, 0.f);
+  }
+  __device__ __forceinline__ void store(float4* row, const Row<VEC>& r) const {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i)
+      if (FULL || ok[i]) __stcg(row + i * L, r.x[i]);
+  }
+  // Hogwild! applies increments as atomic component-wise additions:
+  // one 128-bit vector reduction per slot (red.global.add.v4.f32, sm_90+).
+  __device__ __forceinline__ void red(float4* row, const Row<VEC>& d) const {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i)
+      if (FULL || ok[i])
+        asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(row + i * L),
+                     "f"(d.x[i].x), "f"(d.x[i].y), "f"(d.x[i].z), "f"(d.x[i].w)
+                     : "memory");
+  }
+};
 
-  int64_t pos = 0, end = 0, wb = 0;
+__device__ __forceinline__ float4 f4_fma(float s, float4 a, float4 b) {  // s*a + b
+  return make_float4(fmaf(s, a.x, b.x), fmaf(s, a.y, b.y), fmaf(s, a.z, b.z), fmaf(s, a.w, b.w));
+}
+__device__ __forceinline__ float4 f4_scale(float s, float4 a) {
+  return make_float4(s * a.x, s * a.y, s * a.z, s * a.w);
+}
+__device__ __forceinline__ float4 f4_add(float4 a, float4 b) {
+  return make_float4(a.x + b.x, a.y + b.y, a.z + b.z, a.w + b.w);
+}
+
+template <int L, int VEC, bool FULL, bool ATOMIC>
+struct Group {
+  static constexpr unsigned FM = 0xffffffffu;
+  static constexpr int RPL = L >= 8 ? 1 : 8 / L;  // records per lane per window
+  static constexpr int WR = L * RPL;              // ratings per window
+
+  const SgdArgs& a;
+  const int sl, k4;
+  const float g, c1, ngl;  // p' = c1 p + (g e) q ;  dq = (g e) p - (g lambda) q
+  Lanes<L, VEC, FULL> lanes;
+  const float4* Pb;  // lane-adjusted bases: row r, slot i at base + r*k4 + i*L
+  const float4* Qb;
+
+  // task / window state (uniform inside the group)
+  int64_t wbase = 0;  // record index of window 0
+  int jw = 0;         // position of the current rating in window 0
+  int left = 0;       // ratings of the task from the current one on
   bool live = false, done = false;
   int wu0[RPL], wv0[RPL], wu1[RPL], wv1[RPL];
   float wr0[RPL], wr1[RPL];
-#pragma unroll
-  for (int t = 0; t < RPL; ++t) wu0[t] = wv0[t] = wu1[t] = wv1[t] = 0, wr0[t] = wr1[t] = 0.f;
+  // current rating
   int cu = 0, cv = 0;
   float cr = 0.f;
-  float4 p[VEC], q[VEC], pn[VEC], qn[VEC];
-#pragma unroll
-  for (int i = 0; i < VEC; ++i) p[i] = q[i] = pn[i] = qn[i] = make_float4(0.f, 0.f, 0.f, 0.f);
-
+  Row<VEC> p, pn;
   unsigned long long tnext = 0;
-  if (sl == 0) tnext = atomicAdd(a.counter, 1ull);
 
-  auto load_window = [&](int (&wu)[RPL], int (&wv)[RPL], float (&wr)[RPL], int64_t base) {
+  __device__ Group(const SgdArgs& args, int sl_)
+      : a(args), sl(sl_), k4(args.k >> 2), g(args.gamma), c1(1.f - args.gamma * args.lambda),
+        ngl(-args.gamma * args.lambda) {
+    lanes.init(sl, k4);
+    Pb = reinterpret_cast<const float4*>(a.P) + sl - (int64_t)a.row0 * k4;
+    Qb = reinterpret_cast<const float4*>(a.Q) + sl;
+#pragma unroll
+    for (int t = 0; t < RPL; ++t) wu0[t] = wv0[t] = wu1[t] = wv1[t] = 0, wr0[t] = wr1[t] = 0.f;
+  }
+
+  __device__ __forceinline__ const float4* prow(int u) const { return Pb + (int64_t)u * k4; }
+  __device__ __forceinline__ const float4* qrow(int v) const { return Qb + (int64_t)v * k4; }
+
+  __device__ __forceinline__ void load_window(int (&wu)[RPL], int (&wv)[RPL], float (&wr)[RPL], int64_t base,
+                                              int avail) {
 #pragma unroll
     for (int t = 0; t < RPL; ++t) {
-      const int64_t idx = base + t * L + sl;
-      if (idx < end) {
-        wu[t] = __ldcs(ru + idx);
-        wv[t] = __ldcs(rv + idx);
-        wr[t] = __ldcs(rr + idx);
+      const int j = t * L + sl;
+      if (j < avail) {
+        wu[t] = __ldcs(a.ru + base + j);
+        wv[t] = __ldcs(a.rv + base + j);
+        wr[t] = __ldcs(a.rr + base + j);
       }
     }
-  };
-  // rating idx (in [wb, wb + WR)) broadcast inside the group; executed by all lanes
-  auto fetch = [&](int64_t idx, int& u, int& v, float& r) {
-    const int j = (int)(idx - wb) & (WR - 1);
-    const int t = j / L, src = j & (L - 1);
+  }
+  // rating at position j of window 0, broadcast inside the group (all lanes execute)
+  __device__ __forceinline__ void fetch(int j, int& u, int& v, float& r) const {
+    const int t = (j & (WR - 1)) / L, src = j & (L - 1);
     int xu = wu0[0], xv = wv0[0];
     float xr = wr0[0];
 #pragma unroll
@@ -133,110 +137,253 @@ __global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
     u = __shfl_sync(FM, xu, src, L);
     v = __shfl_sync(FM, xv, src, L);
     r = __shfl_sync(FM, xr, src, L);
-  };
+  }
 
-  while (true) {
-    // ---- task start (a group whose task ended takes the prefetched id)
+  // Task start for groups that need one (all lanes of the warp execute this).
+  __device__ __forceinline__ void refill(Row<VEC>& qc) {
     const bool need = !done && !live;
-    if (__any_sync(FM, need)) {
-      const unsigned long long t = __shfl_sync(FM, tnext, 0, L);
-      if (need) {
-        if (t < (unsigned long long)a.n_tasks) {
-          pos = a.task_lo[t];
-          end = a.task_hi[t];
-          live = true;
-          wb = pos;
-          load_window(wu0, wv0, wr0, wb);
-          load_window(wu1, wv1, wr1, wb + WR);
-          if (sl == 0) tnext = atomicAdd(a.counter, 1ull);
-        } else {
-          done = true;
-        }
-      }
-      int u0, v0;
-      float r0;
-      fetch(pos, u0, v0, r0);
-      if (need && live) {
-        cu = u0;
-        cv = v0;
-        cr = r0;
-        load_row<L, VEC>(P + (int64_t)(cu - a.row0) * k, p, ok, sl);
-        load_row<L, VEC>(Q + (int64_t)cv * k, q, ok, sl);
+    if (!__any_sync(FM, need)) return;
+    const unsigned long long t = __shfl_sync(FM, tnext, 0, L);
+    if (need) {
+      if (t < (unsigned long long)a.n_tasks) {
+        const int64_t lo = a.task_lo[t], hi = a.task_hi[t];
+        wbase = lo;
+        jw = 0;
+        left = (int)(hi - lo);
+        live = true;
+        load_window(wu0, wv0, wr0, wbase, left);
+        load_window(wu1, wv1, wr1, wbase + WR, left - WR);
+        if (sl == 0) tnext = atomicAdd(a.counter, 1ull);
+      } else {
+        done = true;
       }
     }
-    if (__all_sync(FM, done)) break;
+    int u0, v0;
+    float r0;
+    fetch(0, u0, v0, r0);
+    if (need && live) {
+      cu = u0;
+      cv = v0;
+      cr = r0;
+      lanes.load(prow(cu), p);
+      lanes.load(qrow(cv), qc);
+    }
+  }
 
-    // ---- look ahead: rating pos+1 and its operands
-    const bool has_next = live && (pos + 1 < end);
-    if (has_next && pos + 1 >= wb + WR) {  // slide the double-buffered window
+  // One pipelined step: update the current rating (q in qc), prefetch the next into qn.
+  __device__ __forceinline__ void step(Row<VEC>& qc, Row<VEC>& qn) {
+    const bool has_next = live && left > 1;
+    // ---- next record (slide the double-buffered window when it is used up)
+    int jn = jw + 1;
+    if (has_next && jn == WR) {
 #pragma unroll
       for (int t = 0; t < RPL; ++t) wu0[t] = wu1[t], wv0[t] = wv1[t], wr0[t] = wr1[t];
-      wb += WR;
-      load_window(wu1, wv1, wr1, wb + WR);
+      wbase += WR;
+      jn = 0;
+      load_window(wu1, wv1, wr1, wbase + WR, left - 1 - WR);
     }
     int nu, nv;
     float nr;
-    fetch(pos + 1, nu, nv, nr);
-    if (has_next) {
-      if (nv != cv) load_row<L, VEC>(Q + (int64_t)nv * k, qn, ok, sl);
-      if (nu != cu) load_row<L, VEC>(P + (int64_t)(nu - a.row0) * k, pn, ok, sl);
-    }
+    fetch(jn, nu, nv, nr);
+    const bool newq = has_next && nv != cv;
+    const bool newp = has_next && nu != cu;
+    if (newq) lanes.load(qrow(nv), qn);
+    if (newp) lanes.load(prow(nu), pn);
 
-    // ---- e = r - p.q  (four independent partial sums, then log2(L) shuffles)
+    // ---- e = r - p.q
     float d0 = 0.f, d1 = 0.f, d2 = 0.f, d3 = 0.f;
-    if (live) {
 #pragma unroll
-      for (int i = 0; i < VEC; ++i) {
-        d0 = fmaf(p[i].x, q[i].x, d0);
-        d1 = fmaf(p[i].y, q[i].y, d1);
-        d2 = fmaf(p[i].z, q[i].z, d2);
-        d3 = fmaf(p[i].w, q[i].w, d3);
-      }
+    for (int i = 0; i < VEC; ++i) {
+      d0 = fmaf(p.x[i].x, qc.x[i].x, d0);
+      d1 = fmaf(p.x[i].y, qc.x[i].y, d1);
+      d2 = fmaf(p.x[i].z, qc.x[i].z, d2);
+      d3 = fmaf(p.x[i].w, qc.x[i].w, d3);
     }
     float d = (d0 + d1) + (d2 + d3);
 #pragma unroll
     for (int o = L / 2; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
 
-    // ---- p' = p + g(e q - lambda p);  q' = q + g(e p - lambda q)   (p: pre-update)
     if (live) {
+      // ---- p' = c1 p + (g e) q ;  dq = (g e) p - (g lambda) q   (p: pre-update)
+      const float ge = g * (cr - d);
+      Row<VEC> dq;
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) {
+        dq.x[i] = f4_fma(ge, p.x[i], f4_scale(ngl, qc.x[i]));
+        p.x[i] = f4_fma(ge, qc.x[i], f4_scale(c1, p.x[i]));
+      }
+      float4* qrow_w = const_cast<float4*>(qrow(cv));
+      if (ATOMIC) {
+        lanes.red(qrow_w, dq);
+      } else {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) dq.x[i] = f4_add(qc.x[i], dq.x[i]);
+        lanes.store(qrow_w, dq);
+      }
+      if (has_next && !newq) {  // same item next: forward the updated q_v
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) qn.x[i] = ATOMIC ? f4_add(qc.x[i], dq.x[i]) : dq.x[i];
+      }
+      if (!has_next || newp) lanes.store(const_cast<float4*>(prow(cu)), p);
+      if (newp) p = pn;
+      live = has_next;
+      cu = nu;
+      cv = nv;
+      cr = nr;
+      jw = jn;
+      --left;
+    }
+  }
+};
+
+template <int L, int VEC, bool FULL, bool ATOMIC>
+__global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
+  Group<L, VEC, FULL, ATOMIC> grp(a, threadIdx.x & (L - 1));
+  if (grp.sl == 0) grp.tnext = atomicAdd(a.counter, 1ull);
+  Row<VEC> qa, qb;
+#pragma unroll
+  for (int i = 0; i < VEC; ++i) qa.x[i] = qb.x[i] = grp.p.x[i] = grp.pn.x[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+  while (true) {
+    grp.refill(qa);  // the current q is always in qa at the top of the body
+    if (__all_sync(0xffffffffu, grp.done)) break;
+    grp.step(qa, qb);
+    grp.step(qb, qa);
+  }
+}
+
+// Warp-per-rating kernel (L = 32, k a multiple of 128): one rating group per warp,
+// so every branch is warp-uniform and the task loop is a plain counted loop
+// (no lock step, no per-step liveness predicates).  Same pipeline as Group:
+// rating j+1's record and q row are in flight while rating j is updated.
+template <int VEC, bool ATOMIC>
+__global__ void __launch_bounds__(kThreads) sgd_warp_kernel(SgdArgs a) {
+  constexpr unsigned FM = 0xffffffffu;
+  const int lane = threadIdx.x & 31;
+  const int k4 = a.k >> 2;
+  const float g = a.gamma, c1 = 1.f - a.gamma * a.lambda, ngl = -a.gamma * a.lambda;
+  const float4* __restrict__ Pb = reinterpret_cast<const float4*>(a.P) + lane - (int64_t)a.row0 * k4;
+  const float4* __restrict__ Qb = reinterpret_cast<const float4*>(a.Q) + lane;
+  auto prow = [&](int u) { return Pb + (int64_t)(u * k4); };  // 32-bit row offsets: m_local*k/4, n*k/4 < 2^31
+  auto qrow = [&](int v) { return Qb + (int64_t)(v * k4); };
+  auto ld = [&](const float4* r, float4 (&x)[VEC]) {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) x[i] = __ldcg(r + 32 * i);
+  };
+  auto st = [&](const float4* r, const float4 (&x)[VEC]) {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) __stcg(const_cast<float4*>(r) + 32 * i, x[i]);
+  };
+
+  unsigned long long tn = 0;
+  if (lane == 0) tn = atomicAdd(a.counter, 1ull);
+  tn = __shfl_sync(FM, tn, 0);
+  while (tn < (unsigned long long)a.n_tasks) {
+    const int64_t lo = a.task_lo[tn];
+    const int left = (int)(a.task_hi[tn] - lo);
+    unsigned long long tn2 = 0;
+    if (lane == 0) tn2 = atomicAdd(a.counter, 1ull);  // next task id, fetched one task ahead
+    const int32_t* ru = a.ru + lo;
+    const int32_t* rv = a.rv + lo;
+    const float* rr = a.rr + lo;
+    // double-buffered record windows: lane l holds ratings w*32 + l and w*32 + 32 + l
+    int wu0 = 0, wv0 = 0, wu1 = 0, wv1 = 0;
+    float wr0 = 0.f, wr1 = 0.f;
+    if (lane < left) wu0 = __ldcs(ru + lane), wv0 = __ldcs(rv + lane), wr0 = __ldcs(rr + lane);
+    if (lane + 32 < left) wu1 = __ldcs(ru + 32 + lane), wv1 = __ldcs(rv + 32 + lane), wr1 = __ldcs(rr + 32 + lane);
+    int wb = 0;  // first rating of window 0
+    int cu = __shfl_sync(FM, wu0, 0), cv = __shfl_sync(FM, wv0, 0);
+    float cr = __shfl_sync(FM, wr0, 0);
+    float4 p[VEC], pn[VEC], qa[VEC], qb[VEC];
+    ld(prow(cu), p);
+    ld(qrow(cv), qa);
+
+    // one step: update rating j (q in qc), prefetch rating j+1 (q into qn); HAS_NEXT static
+    auto step = [&](int j, float4 (&qc)[VEC], float4 (&qn)[VEC], auto has_next_tag) {
+      constexpr bool HAS_NEXT = decltype(has_next_tag)::value;
+      int nu = 0, nv = 0;
+      float nr = 0.f;
+      bool fwd = false, newp = false;
+      if (HAS_NEXT) {
+        if (j + 1 - wb == 32) {  // slide the window
+          wu0 = wu1, wv0 = wv1, wr0 = wr1;
+          wb += 32;
+          const int idx = wb + 32 + lane;
+          if (idx < left) wu1 = __ldcs(ru + idx), wv1 = __ldcs(rv + idx), wr1 = __ldcs(rr + idx);
+        }
+        const int src = j + 1 - wb;
+        nu = __shfl_sync(FM, wu0, src);
+        nv = __shfl_sync(FM, wv0, src);
+        nr = __shfl_sync(FM, wr0, src);
+        fwd = nv == cv;
+        newp = nu != cu;
+        if (!fwd) ld(qrow(nv), qn);
+        if (newp) ld(prow(nu), pn);
+      }
+      float d0 = 0.f, d1 = 0.f, d2 = 0.f, d3 = 0.f;
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) {
+        d0 = fmaf(p[i].x, qc[i].x, d0);
+        d1 = fmaf(p[i].y, qc[i].y, d1);
+        d2 = fmaf(p[i].z, qc[i].z, d2);
+        d3 = fmaf(p[i].w, qc[i].w, d3);
+      }
+      float d = (d0 + d1) + (d2 + d3);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
       const float ge = g * (cr - d);
       float4 dq[VEC];
 #pragma unroll
       for (int i = 0; i < VEC; ++i) {
-        const float4 pp = p[i], qq = q[i];
-        p[i] = make_float4(fmaf(ge, qq.x, c1 * pp.x), fmaf(ge, qq.y, c1 * pp.y), fmaf(ge, qq.z, c1 * pp.z),
-                           fmaf(ge, qq.w, c1 * pp.w));
-        dq[i] = make_float4(fmaf(ge, pp.x, -gl * qq.x), fmaf(ge, pp.y, -gl * qq.y), fmaf(ge, pp.z, -gl * qq.z),
-                            fmaf(ge, pp.w, -gl * qq.w));
-        q[i] = make_float4(qq.x + dq[i].x, qq.y + dq[i].y, qq.z + dq[i].z, qq.w + dq[i].w);
+        dq[i] = f4_fma(ge, p[i], f4_scale(ngl, qc[i]));
+        p[i] = f4_fma(ge, qc[i], f4_scale(c1, p[i]));
       }
-      if (ATOMIC)
-        red_row<L, VEC>(Q + (int64_t)cv * k, dq, ok, sl);
-      else
-        store_row<L, VEC>(Q + (int64_t)cv * k, q, ok, sl);
-      if (!has_next) {
-        store_row<L, VEC>(P + (int64_t)(cu - a.row0) * k, p, ok, sl);
-        live = false;
+      const float4* qw = qrow(cv);
+      if (ATOMIC) {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i)
+          asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(qw + 32 * i),
+                       "f"(dq[i].x), "f"(dq[i].y), "f"(dq[i].z), "f"(dq[i].w)
+                       : "memory");
       } else {
-        if (nu != cu) {
-          store_row<L, VEC>(P + (int64_t)(cu - a.row0) * k, p, ok, sl);
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) dq[i] = f4_add(qc[i], dq[i]);
+        st(qw, dq);
+      }
+      if (HAS_NEXT) {
+        if (fwd) {  // same item next (duplicates): serial read-after-write from registers
+#pragma unroll
+          for (int i = 0; i < VEC; ++i) qn[i] = ATOMIC ? f4_add(qc[i], dq[i]) : dq[i];
+        }
+        if (newp) {
+          st(prow(cu), p);
 #pragma unroll
           for (int i = 0; i < VEC; ++i) p[i] = pn[i];
-        }
-        if (nv != cv) {
-#pragma unroll
-          for (int i = 0; i < VEC; ++i) q[i] = qn[i];
         }
         cu = nu;
         cv = nv;
         cr = nr;
-        ++pos;
+      } else {
+        st(prow(cu), p);
       }
+    };
+    using T = std::true_type;
+    using F = std::false_type;
+    int j = 0;
+    for (; left - j >= 3; j += 2) {
+      step(j, qa, qb, T{});
+      step(j + 1, qb, qa, T{});
     }
+    if (left - j == 2) {
+      step(j, qa, qb, T{});
+      step(j + 1, qb, qa, F{});
+    } else {
+      step(j, qa, qb, F{});
+    }
+    tn = __shfl_sync(FM, tn2, 0);
   }
 }
 
-template <int L, int VEC>
+template <int L, int VEC, bool FULL>
 cudaError_t launch_t(const SgdArgs& a, int64_t warps, cudaStream_t st) {
   constexpr int groups_per_warp = 32 / L;
   int64_t need_warps = (a.n_tasks + groups_per_warp - 1) / groups_per_warp;
@@ -245,23 +392,30 @@ cudaError_t launch_t(const SgdArgs& a, int64_t warps, cudaStream_t st) {
   // exactly w warps when w < 8 (one partial CTA), else whole CTAs of 8 warps
   const int threads = w < kThreads / 32 ? (int)w * 32 : kThreads;
   const int64_t blocks = (w * 32 + threads - 1) / threads;
+  if (L == 32 && FULL) {  // warp-per-rating specialisation
+    if (a.atomic_q)
+      sgd_warp_kernel<VEC, true><<<(unsigned)blocks, threads, 0, st>>>(a);
+    else
+      sgd_warp_kernel<VEC, false><<<(unsigned)blocks, threads, 0, st>>>(a);
+    return cudaGetLastError();
+  }
   if (a.atomic_q)
-    sgd_kernel<L, VEC, true><<<(unsigned)blocks, threads, 0, st>>>(a);
+    sgd_kernel<L, VEC, FULL, true><<<(unsigned)blocks, threads, 0, st>>>(a);
   else
-    sgd_kernel<L, VEC, false><<<(unsigned)blocks, threads, 0, st>>>(a);
+    sgd_kernel<L, VEC, FULL, false><<<(unsigned)blocks, threads, 0, st>>>(a);
   return cudaGetLastError();
 }
 
 }  // namespace
 
-// Lane geometry: VEC float4 slots per lane, L lanes per
-// rating group.  Auto: VEC = 2 for k >= 64 (k = 128: L = 16, two ratings per
-// warp), else 1; L is capped at 32 (k = 512 -> VEC = 4); VEC = 3 is rounded up to
-// 4 (masked).  VEC = 4 at k = 128 packs 9472 groups on the chip, a concurrency
-// at which atomic Hogwild was seen to diverge on the Netflix shape (R14).
+// Lane geometry: VEC float4 slots per lane, L lanes per rating group.  Auto: one
+// rating per warp (L = 32) once k >= 128 (k = 128: VEC = 1, k = 256: 2, k = 512: 4),
+// the warp-per-rating kernel; below, L = k/4 lanes and 32/L groups per warp in lock
+// step.  At equal rating groups in flight (equal Hogwild staleness) one group per
+// warp was fastest on C3 (tools/sweep_hogwild.py: 7.7 vs 5.8 G upd/s).
 void sgd_geometry(int k, int vec_pref, int* L_out, int* VEC_out) {
   const int c4 = k / 4;
-  int vec = vec_pref > 0 ? vec_pref : (c4 >= 16 ? 2 : 1);
+  int vec = vec_pref > 0 ? vec_pref : std::max(1, std::min(4, c4 / 32));
   if (vec == 3) vec = 4;
   auto pow2 = [](int x) { int l = 1; while (l < x) l <<= 1; return l; };
   int L = std::min(32, pow2((c4 + vec - 1) / vec));
@@ -295,8 +449,9 @@ cudaError_t launch_sgd(const SgdArgs& a, int64_t warps, cudaStream_t st) {
   if (a.n_tasks <= 0) return cudaSuccess;
   int L, VEC;
   sgd_geometry(a.k, a.vec_pref, &L, &VEC);
+  const bool full = (L * VEC * 4 == a.k);
 #define SGD_CASE(LL, VV) \
-  if (L == LL && VEC == VV) return launch_t<LL, VV>(a, warps, st);
+  if (L == LL && VEC == VV) return full ? launch_t<LL, VV, true>(a, warps, st) : launch_t<LL, VV, false>(a, warps, st);
   SGD_CASE(1, 1) SGD_CASE(2, 1) SGD_CASE(4, 1)
   SGD_CASE(8, 1) SGD_CASE(8, 2) SGD_CASE(8, 4)
   SGD_CASE(16, 1) SGD_CASE(16, 2) SGD_CASE(16, 4)

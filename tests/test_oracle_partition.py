@@ -13,7 +13,7 @@ def _llround(x):
     return int(math.floor(x + 0.5))  # x >= 0: round half away from zero
 
 
-def _bruteforce_partition(m, n, u, v, G, Br, Bc, x, perm_row, perm_col):
+def _bruteforce_partition(m, n, u, v, G, Br, Bc, x, perm_row, perm_col, seed=0, orc=None):
     cnt = np.bincount(perm_row[u], minlength=m) if len(u) else np.zeros(m, int)
     S = [0]
     for c in cnt:
@@ -31,7 +31,9 @@ def _bruteforce_partition(m, n, u, v, G, Br, Bc, x, perm_row, perm_col):
         s = max(j for j in range(G) if b[j] <= up < b[j + 1])
         rb = (up - b[s]) * Br // (b[s + 1] - b[s])
         cb = vp * Bc // n
-        recs.append((((s * Br + rb) * Bc + cb), up, vp, i))
+        c0, c1 = -(-cb * n // Bc), -(-(cb + 1) * n // Bc)
+        rot = orc.hash4(seed, 5, up, 0) % (c1 - c0) if seed else 0
+        recs.append((((s * Br + rb) * Bc + cb), up, (vp - c0 + rot) % (c1 - c0), i, vp))
     recs.sort()
     off = [0] * (G * Br * Bc + 1)
     for rec in recs:
@@ -53,7 +55,7 @@ def test_partition_and_sort_bruteforce(orc):
         u, v, r = synth.tiny(m, n, nnz, seed=trial)
         x = rng.dirichlet(np.ones(G)) if trial % 2 else np.full(G, 1.0 / G)
         pr, pc = orc.perm(seed, 1, m), orc.perm(seed, 2, n)
-        S, b, recs, off = _bruteforce_partition(m, n, u, v, G, Br, Bc, x, pr, pc)
+        S, b, recs, off = _bruteforce_partition(m, n, u, v, G, Br, Bc, x, pr, pc, seed, orc)
         assert list(orc.row_prefix(m, u, pr)) == S
         ob = orc.bounds(m, nnz, np.array(S, np.int64), G, x)
         assert list(ob) == b
@@ -61,9 +63,9 @@ def test_partition_and_sort_bruteforce(orc):
             # an empty shard with ratings elsewhere is fine; the blocker never
             # divides by its zero row count because no record lands in it
             pass
-        ou, ov, orr, ooff = orc.block_sort(m, n, u, v, r, G, Br, Bc, ob, pr, pc)
+        ou, ov, orr, ooff = orc.block_sort(m, n, u, v, r, G, Br, Bc, ob, pr, pc, seed)
         assert list(ooff) == off
-        assert list(ou) == [t[1] for t in recs] and list(ov) == [t[2] for t in recs]
+        assert list(ou) == [t[1] for t in recs] and list(ov) == [t[4] for t in recs]
         assert np.array_equal(orr, r[[t[3] for t in recs]])
 
 
@@ -83,20 +85,20 @@ def test_partition_invariants_medium(orc):
             cum = np.cumsum(x)
             for s in range(1, G):
                 assert abs(S[b[s]] - _llround(nnz * cum[s - 1])) <= cnt.max()
-            ou, ov, orr, off = orc.block_sort(m, n, u, v, r, G, 4, 5, b, pr, pc)
+            ou, ov, orr, off = orc.block_sort(m, n, u, v, r, G, 4, 5, b, pr, pc, seed)
             assert off[-1] == nnz
             # multiset preserved
             a = np.sort(np.stack([ou, ov, orr.view(np.int32)]), axis=1)
             want = np.sort(np.stack([pr[u], pc[v], r.view(np.int32)]), axis=1)
             assert np.array_equal(np.sort(ou), np.sort(pr[u]))
             assert np.array_equal(np.sort(orr), np.sort(r))
-            # row-sorted within each block; every record inside its block's ranges
+            # row-sorted within each block (rows contiguous, each row a rotation of the
+            # block's columns, R21); every record inside its block's ranges
             for blk in range(G * 20):
                 lo, hi = off[blk], off[blk + 1]
                 s, rem = divmod(blk, 20)
                 rb, cb = divmod(rem, 5)
-                key = ou[lo:hi].astype(np.int64) * n + ov[lo:hi]
-                assert np.all(np.diff(key) >= 0)
+                assert np.all(np.diff(ou[lo:hi]) >= 0)
                 assert np.all((ou[lo:hi] >= b[s]) & (ou[lo:hi] < b[s + 1]))
                 assert np.all(ov[lo:hi] * 5 // n == cb)
             del a, want
