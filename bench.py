@@ -35,6 +35,7 @@ import synth  # noqa: E402
 METRIC = "rating updates/sec (whole box)"
 UNIT = "updates/s"
 FALLBACK_HBM_GBS = 6650.0
+DEVICE_GEN_NNZ = 1_000_000_000
 
 
 def parse():
@@ -111,6 +112,17 @@ def ncu_traffic(cfg_name, sched):
             return json.load(f).get(f"{cfg_name}/{sched}")
     except Exception:
         return None
+
+
+def host_mem_available():
+    try:
+        with open("/proc/meminfo") as f:
+            for line in f:
+                if line.startswith("MemAvailable:"):
+                    return int(line.split()[1]) * 1024
+    except OSError:
+        pass
+    return 0
 
 
 def host_cpu():
@@ -202,9 +214,17 @@ def main():
         Br, Bc = 64, 64 * (G if sync == "ring" else 1)
 
     t_gen = time.perf_counter()
-    (u, v, r), (tu, tv, tr) = synth.make(cfg)
+    on_device = cfg.nnz > DEVICE_GEN_NNZ  # C5: 37 GB of COO, drawn on the GPU (synth.make_device)
+    if on_device:
+        (du, dv, dr), (dtu, dtv, dtr) = synth.make_device(cfg, device=f"cuda:{local}")
+        u = v = r = tu = tv = tr = None
+        S = 2_000_000
+        sample = (du[:S].cpu().numpy(), dv[:S].cpu().numpy(), dr[:S].cpu().numpy())
+    else:
+        (u, v, r), (tu, tv, tr) = synth.make(cfg)
+        sample = (u, v, r)
+    torch.cuda.synchronize()
     t_gen = time.perf_counter() - t_gen
-    nnz, nt = len(u), len(tu)
 
     stream = torch.cuda.Stream()
     mdl = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, dist=world > 1, device=local)
@@ -215,16 +235,22 @@ def main():
         mdl.set_option("task_ratings", args.task)
     if args.vec:
         mdl.set_option("vec", args.vec)
-    du, dv, dr = (torch.from_numpy(x).cuda() for x in (u, v, r))
-    dtu, dtv, dtr = (torch.from_numpy(x).cuda() for x in (tu, tv, tr))
+    if not on_device:
+        du, dv, dr = (torch.from_numpy(x).cuda() for x in (u, v, r))
+        dtu, dtv, dtr = (torch.from_numpy(x).cuda() for x in (tu, tv, tr))
+    nnz, nt = int(du.numel()), int(dtu.numel())
     torch.cuda.synchronize()
     t_prep = time.perf_counter()
     mdl.load(du, dv, dr)
+    if on_device:  # keep a host-free copy only where it fits; free the generator's 37 GB first
+        del du, dv, dr
+        torch.cuda.empty_cache()
     mdl.partition(G, (Br, Bc), "DP0", seed=cfg.seed)
     mdl.init(1)
     t_prep = time.perf_counter() - t_prep
     info = mdl.info()
-    del du, dv, dr
+    if not on_device:
+        del du, dv, dr
     rm0 = mdl.rmse(dtu, dtv, dtr)
     mdl.set_option("sync_stream", 0)
 
@@ -293,8 +319,20 @@ def main():
            "paper_context": {"netflix_hcc_updates_per_s": 2228476993,
                              "hardware": "2x Xeon Gold 6242 + RTX 2080 + RTX 2080S (Table 4, L2001)"}}
 
+    mdl.close()  # free HBM before the e2e jobs build their own handles
     # ---- e2e: the whole job through the public API from pinned host buffers
-    if not args.no_e2e:
+    e2e_skip = None
+    if on_device and not args.no_e2e:
+        need = 12 * (nnz + nt) * 2 + 4 * (cfg.m + cfg.n) * cfg.k
+        if host_mem_available() < need:
+            e2e_skip = f"host memory {host_mem_available() / 1e9:.0f} GB < {need / 1e9:.0f} GB for pinned COO + P, Q"
+        else:
+            (u, v, r), (tu, tv, tr) = synth.make_device(cfg, device=f"cuda:{local}")
+            u, v, r, tu, tv, tr = (x.cpu().numpy() for x in (u, v, r, tu, tv, tr))
+            torch.cuda.empty_cache()
+    if e2e_skip:
+        out["e2e"] = {"value": None, "unit": UNIT, "skipped": e2e_skip}
+    elif not args.no_e2e:
         pin = [torch.from_numpy(x).pin_memory() for x in (u, v, r, tu, tv, tr)]
         Ph = torch.empty((cfg.m, cfg.k), dtype=torch.float32).pin_memory()
         Qh = torch.empty((cfg.n, cfg.k), dtype=torch.float32).pin_memory()
@@ -336,14 +374,13 @@ def main():
                               "host pinned buffers", "s_per_step": e2e_s}
 
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        val, S, ep, dt = oracle_sample(cfg, u, v, r, args.cpu_seconds)
+        val, S, ep, dt = oracle_sample(cfg, *sample, args.cpu_seconds)
         model, ncpu = host_cpu()
         out["cpu_baseline"] = {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
                                "sample": f"{ep} serial fp64 oracle epoch(s) over the first {S} ratings of the "
                                          f"same stream, {dt:.1f} s on 1 of {ncpu} cores ({model})"}
     if rank == 0:
         print(json.dumps(out), flush=True)
-    mdl.close()
     if world > 1:
         dist.destroy_process_group()
 

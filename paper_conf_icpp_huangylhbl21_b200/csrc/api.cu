@@ -317,14 +317,14 @@ hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
 // Hogwild concurrency (R14): the number of rating groups in flight sets
 // the staleness of q_v reads, so it is capped at n / opt_conflict groups, and at 32
 // resident warps per SM.
-int64_t auto_warps(hccmf_t h) {
+int64_t auto_warps(hccmf_t h, int64_t items_in_play) {
   if (h->opt_warps > 0) return h->opt_warps;
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
   int64_t w = (int64_t)sms * 32;
   if (h->opt_conflict > 0) {
     const int64_t groups_per_warp = 32 / sgd_lanes(h->k, (int)h->opt_vec);
-    const int64_t cap = std::max<int64_t>(1, (h->n / h->opt_conflict) / groups_per_warp);
+    const int64_t cap = std::max<int64_t>(1, (items_in_play / h->opt_conflict) / groups_per_warp);
     w = std::min(w, cap);
   }
   return w;
@@ -748,7 +748,8 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   a.atomic_q = (sched == HCCMF_SCHED_HOGWILD && h->opt_atomic) ? 1 : 0;
   a.vec_pref = (int32_t)h->opt_vec;
   const int L = sgd_lanes(h->k, (int)h->opt_vec);
-  const int64_t hog_warps = auto_warps(h);
+  // a ring stage races only on its column group's items
+  const int64_t hog_warps = auto_warps(h, eff_sync == HCCMF_SYNC_RING ? h->n / G : h->n);
   int stage = 0;
   for (size_t li = 0; li < pl->launches.size(); ++li) {
     const Launch& ln = pl->launches[li];
