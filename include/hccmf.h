@@ -138,10 +138,15 @@ typedef enum {
                                     rest keep the shuffled user order.  Default
                                     1024; -1: shuffled order only; 0: pure LPT.
                                     Takes effect at the next hccmf_partition.     */
-    HCCMF_OPT_VEC = 8            /* float4 slots of p_u / q_v per lane (1, 2, 4; 0 =
+    HCCMF_OPT_VEC = 8,           /* float4 slots of p_u / q_v per lane (1, 2, 4; 0 =
                                     auto: k/128 clamped to [1, 4], i.e. one rating
                                     per warp from k = 128); lanes per rating
                                     L = min(32, k / (4 VEC))                      */
+    HCCMF_OPT_DET_WAVE = 9       /* 1 (default): a single-shard DET epoch on a square
+                                    grid runs as one wavefront kernel (warp i waits
+                                    only for warp i+1's previous stratum) when the
+                                    B warps fit on the device; 0: one launch per
+                                    stratum.  Same update order either way.       */
 } hccmf_option;
 
 /* ------------------------------------------------------------------ lifecycle */

@@ -181,6 +181,8 @@ void free_partition(hccmf_t h) {
   dfree(h, h->d_Qrep, (size_t)h->n * h->k * (h->shard_hi - h->shard_lo));
   dfree(h, h->d_counters, h->n_counters);
   h->n_counters = 0;
+  dfree(h, h->d_blk_off, h->nblk_local + 1);
+  dfree(h, h->d_progress, h->Br);
   h->local_nnz = 0;
   h->rows = 0;
   h->blk_task_off.clear();
@@ -452,6 +454,9 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
     case HCCMF_OPT_HOGWILD_ATOMIC:
       h->opt_atomic = value != 0;
       return HCCMF_OK;
+    case HCCMF_OPT_DET_WAVE:
+      h->opt_wave = value != 0;
+      return HCCMF_OK;
     case HCCMF_OPT_VEC:
       if (value != 0 && value != 1 && value != 2 && value != 4) return fail(h, HCCMF_EINVAL, "vec must be 0, 1, 2 or 4");
       h->opt_vec = value;
@@ -661,6 +666,10 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   h->device_bytes += 2 * sizeof(int64_t) * (nt ? nt : 1);
   h->n_tasks = nt;
   cudaFreeAsync(dLoc, st);
+  // local block offsets stay on the device for the DET wavefront
+  CU(h, dmalloc(h, &h->d_blk_off, h->nblk_local + 1));
+  CU(h, cudaMemcpyAsync(h->d_blk_off, loc_off.data(), sizeof(int64_t) * (h->nblk_local + 1), cudaMemcpyHostToDevice, st));
+  CU(h, dmalloc(h, &h->d_progress, h->Br));
   h->h_task_lo.resize(nt);
   h->h_task_hi.resize(nt);
   if (nt) {
@@ -717,10 +726,27 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   if (h->state < 3) return fail(h, HCCMF_ESTATE, "train_epoch needs factors (init_factors or set_factors)");
   if (sched != HCCMF_SCHED_DET && sched != HCCMF_SCHED_HOGWILD) return fail(h, HCCMF_EINVAL, "bad schedule");
   if (sync < HCCMF_SYNC_NONE || sync > HCCMF_SYNC_ALLREDUCE_AVG) return fail(h, HCCMF_EINVAL, "bad sync");
+  const int G = h->G;
+  if (sched == HCCMF_SCHED_DET && G == 1 && h->opt_wave && h->Br == h->Bc && h->Br > 1 &&
+      wave_supported(h->k, (int)h->opt_vec, h->Br)) {
+    // DET as one wavefront kernel: same order of updates as the strata (R19)
+    SgdArgs a{};
+    a.ru = h->d_u;
+    a.rv = h->d_v;
+    a.rr = h->d_r;
+    a.P = h->d_P;
+    a.Q = h->d_Q;
+    a.row0 = h->row0;
+    a.k = h->k;
+    a.gamma = h->gamma;
+    a.lambda = h->lambda;
+    a.vec_pref = (int32_t)h->opt_vec;
+    CU(h, launch_wave(a, h->d_blk_off, h->Br, h->d_progress, h->stream));
+    return finish(h);
+  }
   Plan* pl = nullptr;
   hccmf_status st = build_plan(h, sched, sync, &pl);
   if (st != HCCMF_OK) return st;
-  const int G = h->G;
   const int eff_sync = (G == 1) ? HCCMF_SYNC_NONE : sync;
   const bool dist = h->world > 1;
   const int64_t nk = h->n * h->k;

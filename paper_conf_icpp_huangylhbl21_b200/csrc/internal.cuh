@@ -66,6 +66,10 @@ struct SgdArgs {
 
 // launch the SGD kernel for a list of tasks; warps = concurrent warps wanted
 cudaError_t launch_sgd(const SgdArgs& a, int64_t warps, cudaStream_t st);
+// DET as one wavefront kernel (G == 1, square B x B grid, warp-per-rating geometry)
+bool wave_supported(int k, int vec_pref, int B);
+cudaError_t launch_wave(const SgdArgs& a, const int64_t* off /* local block offsets, B*B+1 */, int B,
+                        int* progress /* B ints */, cudaStream_t st);
 // lane geometry of the SGD kernel: L lanes per rating group, VEC float4 per lane
 void sgd_geometry(int k, int vec_pref, int* L, int* VEC);
 int sgd_lanes(int k, int vec_pref);
@@ -123,7 +127,7 @@ struct hccmf_ctx {
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 4, opt_heavy = 1024, opt_vec = 0;
+  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 4, opt_heavy = 1024, opt_vec = 0, opt_wave = 1;
   bool sync_stream = true;
   size_t device_bytes = 0;
 
@@ -163,6 +167,8 @@ struct hccmf_ctx {
   int64_t n_counters = 0;
   double* d_partials = nullptr;
   double* d_scalar = nullptr;
+  int64_t* d_blk_off = nullptr;  // local block offsets (DET wavefront), nblk_local + 1
+  int* d_progress = nullptr;     // wavefront progress counters, Br
 
   int q_ring_sched = -1;  // >= 0: distributed ring left only this rank's Q group valid
   std::vector<hccmf::Plan> plans;

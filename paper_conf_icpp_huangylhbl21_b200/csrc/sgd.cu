@@ -251,37 +251,46 @@ __global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
   }
 }
 
-// Warp-per-rating kernel (L = 32, k a multiple of 128): one rating group per warp,
-// so every branch is warp-uniform and the task loop is a plain counted loop
-// (no lock step, no per-step liveness predicates).  Same pipeline as Group:
-// rating j+1's record and q row are in flight while rating j is updated.
+// Warp-per-rating path (L = 32, k a multiple of 128): one rating group per warp, so
+// every branch is warp-uniform and a task is a plain counted loop (no lock step, no
+// per-step liveness predicates).  Same pipeline as Group: rating j+1's record and
+// q row are in flight while rating j is updated.
 template <int VEC, bool ATOMIC>
-__global__ void __launch_bounds__(kThreads) sgd_warp_kernel(SgdArgs a) {
-  constexpr unsigned FM = 0xffffffffu;
-  const int lane = threadIdx.x & 31;
-  const int k4 = a.k >> 2;
-  const float g = a.gamma, c1 = 1.f - a.gamma * a.lambda, ngl = -a.gamma * a.lambda;
-  const float4* __restrict__ Pb = reinterpret_cast<const float4*>(a.P) + lane - (int64_t)a.row0 * k4;
-  const float4* __restrict__ Qb = reinterpret_cast<const float4*>(a.Q) + lane;
-  auto prow = [&](int u) { return Pb + (int64_t)(u * k4); };  // 32-bit row offsets: m_local*k/4, n*k/4 < 2^31
-  auto qrow = [&](int v) { return Qb + (int64_t)(v * k4); };
-  auto ld = [&](const float4* r, float4 (&x)[VEC]) {
+struct WarpSgd {
+  static constexpr unsigned FM = 0xffffffffu;
+  const SgdArgs& a;
+  int lane, k4;
+  float g, c1, ngl;
+  const float4* __restrict__ Pb;
+  const float4* __restrict__ Qb;
+
+  __device__ WarpSgd(const SgdArgs& args) : a(args) {
+    lane = threadIdx.x & 31;
+    k4 = a.k >> 2;
+    g = a.gamma;
+    c1 = 1.f - a.gamma * a.lambda;
+    ngl = -a.gamma * a.lambda;
+    Pb = reinterpret_cast<const float4*>(a.P) + lane - (int64_t)a.row0 * k4;
+    Qb = reinterpret_cast<const float4*>(a.Q) + lane;
+  }
+  // 32-bit row offsets: m_local * k/4 and n * k/4 < 2^31
+  __device__ __forceinline__ const float4* prow(int u) const { return Pb + (int64_t)(u * k4); }
+  __device__ __forceinline__ const float4* qrow(int v) const { return Qb + (int64_t)(v * k4); }
+  __device__ __forceinline__ void ld(const float4* r, float4 (&x)[VEC]) const {
 #pragma unroll
     for (int i = 0; i < VEC; ++i) x[i] = __ldcg(r + 32 * i);
-  };
-  auto st = [&](const float4* r, const float4 (&x)[VEC]) {
+  }
+  __device__ __forceinline__ void st(const float4* r, const float4 (&x)[VEC]) const {
 #pragma unroll
     for (int i = 0; i < VEC; ++i) __stcg(const_cast<float4*>(r) + 32 * i, x[i]);
-  };
+  }
 
-  unsigned long long tn = 0;
-  if (lane == 0) tn = atomicAdd(a.counter, 1ull);
-  tn = __shfl_sync(FM, tn, 0);
-  while (tn < (unsigned long long)a.n_tasks) {
-    const int64_t lo = a.task_lo[tn];
-    const int left = (int)(a.task_hi[tn] - lo);
-    unsigned long long tn2 = 0;
-    if (lane == 0) tn2 = atomicAdd(a.counter, 1ull);  // next task id, fetched one task ahead
+  // all ratings of records [lo, lo + left), left >= 1, in order
+  __device__ __forceinline__ void run(int64_t lo, int left) {
+    auto ld = [&](const float4* r, float4 (&x)[VEC]) { this->ld(r, x); };
+    auto st = [&](const float4* r, const float4 (&x)[VEC]) { this->st(r, x); };
+    auto prow = [&](int u) { return this->prow(u); };
+    auto qrow = [&](int v) { return this->qrow(v); };
     const int32_t* ru = a.ru + lo;
     const int32_t* rv = a.rv + lo;
     const float* rr = a.rr + lo;
@@ -379,7 +388,59 @@ __global__ void __launch_bounds__(kThreads) sgd_warp_kernel(SgdArgs a) {
     } else {
       step(j, qa, qb, F{});
     }
+  }
+};
+
+template <int VEC, bool ATOMIC>
+__global__ void __launch_bounds__(kThreads) sgd_warp_kernel(SgdArgs a) {
+  constexpr unsigned FM = 0xffffffffu;
+  WarpSgd<VEC, ATOMIC> w(a);
+  unsigned long long tn = 0;
+  if (w.lane == 0) tn = atomicAdd(a.counter, 1ull);
+  tn = __shfl_sync(FM, tn, 0);
+  while (tn < (unsigned long long)a.n_tasks) {
+    const int64_t lo = a.task_lo[tn];
+    const int left = (int)(a.task_hi[tn] - lo);
+    unsigned long long tn2 = 0;
+    if (w.lane == 0) tn2 = atomicAdd(a.counter, 1ull);  // next task id, fetched one task ahead
+    w.run(lo, left);
     tn = __shfl_sync(FM, tn2, 0);
+  }
+}
+
+// DET as a wavefront (a5): warp i owns row block i and walks its blocks
+// (i, (i+t) mod B) for t = 0..B-1.  Column block (i+t) mod B was last updated by
+// row block i+1 at stratum t-1, so warp i waits only for warp i+1's progress
+// counter (release/acquire through L2) instead of a grid-wide barrier per stratum;
+// the order of updates on every P row and Q row is the strata order of R19.
+// All B warps must be co-resident (checked by the launcher).
+template <int VEC>
+__global__ void __launch_bounds__(kThreads) sgd_wave_kernel(SgdArgs a, const int64_t* __restrict__ off, int B,
+                                                            int* progress) {
+  constexpr unsigned FM = 0xffffffffu;
+  const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+  if (i >= B) return;
+  WarpSgd<VEC, false> w(a);
+  const int nb = (i + 1) % B;
+  for (int t = 0; t < B; ++t) {
+    if (t > 0 && B > 1) {
+      if (w.lane == 0) {
+        int seen;
+        do {
+          asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + nb) : "memory");
+          if (seen < t) __nanosleep(64);
+        } while (seen < t);
+      }
+      __syncwarp();
+    }
+    const int64_t blk = (int64_t)i * B + (i + t) % B;
+    const int64_t lo = off[blk], hi = off[blk + 1];
+    if (hi > lo) w.run(lo, (int)(hi - lo));
+    __syncwarp();
+    if (w.lane == 0) {
+      __threadfence();
+      asm volatile("st.release.gpu.global.s32 [%0], %1;" ::"l"(progress + i), "r"(t + 1) : "memory");
+    }
   }
 }
 
@@ -443,6 +504,43 @@ int lanes_per_rating(int k) {  // RMSE kernel: one float4 slot per lane
   int L = 1;
   while (L < c4) L <<= 1;
   return L;
+}
+
+bool wave_supported(int k, int vec_pref, int B) {
+  int L, VEC;
+  sgd_geometry(k, vec_pref, &L, &VEC);
+  if (L != 32 || L * VEC * 4 != k) return false;
+  int dev = 0, sms = 0, per_sm = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaError_t e = cudaSuccess;
+  switch (VEC) {
+    case 1: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sgd_wave_kernel<1>, kThreads, 0); break;
+    case 2: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sgd_wave_kernel<2>, kThreads, 0); break;
+    case 4: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sgd_wave_kernel<4>, kThreads, 0); break;
+    default: return false;
+  }
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  // co-residency with head room: at most half of the resident warps
+  return (int64_t)B * 2 <= (int64_t)sms * per_sm * (kThreads / 32);
+}
+
+cudaError_t launch_wave(const SgdArgs& a, const int64_t* off, int B, int* progress, cudaStream_t st) {
+  int L, VEC;
+  sgd_geometry(a.k, a.vec_pref, &L, &VEC);
+  cudaError_t e = cudaMemsetAsync(progress, 0, sizeof(int) * B, st);
+  if (e != cudaSuccess) return e;
+  const int64_t blocks = ((int64_t)B * 32 + kThreads - 1) / kThreads;
+  switch (VEC) {
+    case 1: sgd_wave_kernel<1><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress); break;
+    case 2: sgd_wave_kernel<2><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress); break;
+    case 4: sgd_wave_kernel<4><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
 }
 
 cudaError_t launch_sgd(const SgdArgs& a, int64_t warps, cudaStream_t st) {

@@ -295,3 +295,28 @@ def test_hogwild_logical_shards_band_c2(pkg, orc, sync, G, Bc):
     # multi-GPU schedules on G logical shards; the oracle runs the same schedule serially
     want, got = _band(pkg, orc, "c2", 1.0, 32, 20, sync=sync, G=G, Br=1, Bc=Bc, repeats=1)
     assert all(abs(g - want) <= 0.005 for g in got), (want, got)
+
+
+@pytest.mark.parametrize("k,B", [(128, 24), (256, 9)])
+def test_det_wavefront_equals_strata(pkg, orc, k, B):
+    # the wavefront kernel and the per-stratum launches apply the same updates in the
+    # same per-row / per-column order: bit-identical factors, and the oracle to 1e-4
+    cfg = synth.CONFIGS["c1"]
+    (u, v, r), _ = synth.make(cfg)
+    prob = orc.Problem(cfg.m, cfg.n, k, 0.02, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=6)
+    prob.init(2)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    outs = []
+    for wave in (1, 0):
+        mdl = _gpu_problem(pkg, cfg.m, cfg.n, k, 0.02, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=6)
+        mdl.set_option("det_wave", wave)
+        mdl.set_factors(P0, Q0)
+        for _ in range(2):
+            mdl.train_epoch("det", "none")
+        outs.append(mdl.factors())
+    for _ in range(2):
+        prob.epoch("det", "none")
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+    Po, Qo = prob.factors()
+    assert max(np.abs(outs[0][0] - Po).max(), np.abs(outs[0][1] - Qo).max()) <= 1e-4

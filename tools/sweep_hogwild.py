@@ -29,6 +29,7 @@ ap.add_argument("--grid", default="1,1")
 ap.add_argument("--vec", default="0")
 ap.add_argument("--repeat", type=int, default=1)
 ap.add_argument("--heavy", type=int, default=-1)
+ap.add_argument("--sched", default="hogwild")
 ap.add_argument("--every", action="store_true", help="test RMSE after every epoch")
 args = ap.parse_args()
 cfg = synth.CONFIGS[args.config]
@@ -55,7 +56,7 @@ for at, vec, w in [(a_, v_, w_) for a_ in (int(x) for x in args.atomic.split(","
         for e in range(args.epochs):
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record(st)
-            mdl.train_epoch("hogwild", "none")
+            mdl.train_epoch(args.sched, "none")
             b.record(st)
             b.synchronize()
             ts.append(a.elapsed_time(b))
