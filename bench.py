@@ -114,6 +114,25 @@ def ncu_traffic(cfg_name, sched):
         return None
 
 
+def epochs_to_rmse(name, curve):
+    """first epoch whose test RMSE <= oracle RMSE@E + 0.005, against the
+    oracle's stored reference curve (tests/golden/oracle_curve_<cfg>.json, written by
+    tools/oracle_curves.py from oracle/ alone)."""
+    out = {"test_per_epoch": [round(x, 6) for x in curve], "epochs": len(curve) - 1}
+    try:
+        with open(os.path.join(ROOT, "tests", "golden", f"oracle_curve_{name}.json")) as f:
+            ref = json.load(f)
+    except OSError:
+        return out
+    E = ref["epochs"]
+    target = ref["test_rmse"][E] + 0.005
+    first = lambda c: next((e for e in range(1, len(c)) if c[e] <= target), None)  # noqa: E731
+    out.update({"oracle_E": E, "oracle_at_E": ref["test_rmse"][E], "target": target,
+                "epochs_to_rmse": first(curve), "oracle_epochs_to_rmse": first(ref["test_rmse"]),
+                "band_at_E": (abs(curve[E] - ref["test_rmse"][E]) if len(curve) > E else None)})
+    return out
+
+
 def host_mem_available():
     try:
         with open("/proc/meminfo") as f:
@@ -262,8 +281,7 @@ def main():
             ev[1].record(stream)
         return mdl.rmse(dtu, dtv, dtr)
 
-    for _ in range(args.warmup):
-        step()
+    curve = [rm0] + [step() for _ in range(args.warmup)]
     kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     clocks = Clocks(local)
@@ -313,8 +331,7 @@ def main():
            "roofline": roof, "clocks": clk,
            "gpu_launches": args.steps * ((Bc if args.sched == "hogwild" else Br) * (G if sync == "ring" else 1)
                                          + 3),
-           "rmse": {"test_initial": rm0, "test_after_warmup_plus_timed": rms[-1],
-                    "epochs": args.warmup + args.steps},
+           "rmse": epochs_to_rmse(args.config, curve + rms),
            "prep_s": t_prep, "gen_s": t_gen,
            "paper_context": {"netflix_hcc_updates_per_s": 2228476993,
                              "hardware": "2x Xeon Gold 6242 + RTX 2080 + RTX 2080S (Table 4, L2001)"}}

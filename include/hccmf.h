@@ -99,6 +99,13 @@ typedef struct {
     double t_sync;        /* DP2: per-shard sync time, s                            */
     uint64_t seed;        /* a2 ID shuffle seed; 0 = identity permutation          */
     int32_t storage;      /* 0 = fp32 factors (the only value accepted this round) */
+    int32_t grid_dim;     /* 0 (default): row grid, shards of users, only Q moves;
+                             1: column grid, shards of items, only P moves (Strategy 1
+                             "transmitting P only", L1216-L1218); 2: the paper's rule
+                             (L884-L886): rows if m >= n, else columns.  Under a column
+                             grid every caller-facing call keeps its orientation (P is
+                             still m x k, rmse takes (u, v)); get_partition, get_records
+                             and hccmf_info describe the transposed problem. */
 } hccmf_partition_opts;
 
 typedef struct {
@@ -114,6 +121,7 @@ typedef struct {
     int32_t key_bits;        /* bits of the a4 sort key                           */
     int32_t rank, world;     /* 0, 1 for a single-process handle                  */
     int64_t device_bytes;    /* device memory currently owned by the handle       */
+    int32_t transposed;      /* 1: column grid (m, n, rows describe R^T)          */
 } hccmf_info;
 
 /* Tunables for hccmf_set_option (values are int64). */
@@ -142,11 +150,17 @@ typedef enum {
                                     auto: k/128 clamped to [1, 4], i.e. one rating
                                     per warp from k = 128); lanes per rating
                                     L = min(32, k / (4 VEC))                      */
-    HCCMF_OPT_DET_WAVE = 9       /* 1 (default): a single-shard DET epoch on a square
+    HCCMF_OPT_DET_WAVE = 9,      /* 1 (default): a single-shard DET epoch on a square
                                     grid runs as one wavefront kernel (warp i waits
                                     only for warp i+1's previous stratum) when the
                                     B warps fit on the device; 0: one launch per
                                     stratum.  Same update order either way.       */
+    HCCMF_OPT_SYNC_PHASES = 10   /* ALLREDUCE_AVG + HOGWILD: rounds per epoch (>= 1,
+                                    default 1; must divide grid_rows).  Round ph runs
+                                    every shard's row blocks [ph Br/S, (ph+1) Br/S)
+                                    on its Q copy, then averages Q: the paper's
+                                    several pull-compute-push pipelines per epoch
+                                    (L1251-L1269, Fig. 6; R22).         */
 } hccmf_option;
 
 /* ------------------------------------------------------------------ lifecycle */
@@ -247,6 +261,21 @@ HCCMF_API hccmf_status hccmf_get_info(hccmf_t h, hccmf_info* out);
 HCCMF_API hccmf_status hccmf_schedule(int32_t G, int32_t Br, int32_t Bc, int64_t n, int32_t sched, int32_t sync,
                                       int32_t shard, int64_t* blocks, int64_t* n_blocks, int64_t* launch_off,
                                       int32_t* launch_stage, int64_t* n_launches, int64_t* ring);
+
+/* Host-only: the time cost model of section 3.2 and the strategy choice of 3.3.
+ * Worker i (p of them) has runtime memory bandwidth B[i] and bus bandwidth Bbus[i]
+ * (bytes/s); the server B_server.  With D = n (q_only: Strategy 1, L1203-L1233) or
+ * m + n, and elem_bytes per parameter (4 fp32, 2 fp16: Strategy 2):
+ *   T_i,e = nnz (16k+4) / B_i;  x = DP0 (Eq. 6);
+ *   T_i = x_i nnz (16k+4) / B_i + 2 elem k D / Bbus_i        (Eq. 2)
+ *   T_sync = 3 t elem k D / B_server                          (Eq. 3)
+ *   T = max T_i if max T_i / T_sync >= lambda_sync (the paper's threshold "lambda" = 10,
+ *   L855-L859) and *strategy = HCCMF_DP1; else T = max T_i + T_sync, HCCMF_DP2 (Eq. 5).
+ * x, T_i: [p] caller-allocated. */
+HCCMF_API hccmf_status hccmf_cost_model(int32_t p, int64_t m, int64_t n, int64_t nnz, int32_t k, const double* B,
+                                        const double* Bbus, double B_server, int32_t t, int32_t q_only,
+                                        int32_t elem_bytes, double lambda_sync, double* x, double* T_i,
+                                        double* T_sync, double* T, int32_t* strategy);
 
 /* Library version string, e.g. "hccmf 0.1 sm_100a". */
 HCCMF_API const char* hccmf_version(void);

@@ -63,6 +63,8 @@ def lib():
             "orc_rmse": (f64, [i64, P, P, P, i32, P, P, P, P]),
             "orc_objective": (f64, [i64, P, P, P, i32, f64, P, P, P, P]),
             "orc_unpermute": (None, [i64, i32, P, P, P]),
+            "orc_epoch_phased": (ctypes.c_int, [i32, i32, i32, i32, P, i64, i32, f64, f64, P, P, P, P, P]),
+            "orc_cost_model": (i32, [i32, i64, i64, i64, i32, P, P, f64, i32, i32, i32, f64, P, P, P, P]),
         }
         for name, (res, args) in sig.items():
             fn = getattr(L, name)
@@ -138,6 +140,19 @@ def dp2(x, t, t_sync: float) -> np.ndarray:
     return out
 
 
+def cost_model(m, n, nnz, k, B, Bbus, B_server, t=1, q_only=1, elem=4, lambda_sync=10.0):
+    """Eq. 1-5 time cost model; returns (x, T_i, T_sync, T, branch) with branch 1 = DP1, 2 = DP2."""
+    B, Bbus = _f64(B), _f64(Bbus)
+    p = len(B)
+    x = np.empty(p)
+    Ti = np.empty(p)
+    Ts = ctypes.c_double()
+    T = ctypes.c_double()
+    br = lib().orc_cost_model(p, m, n, nnz, k, _p(B), _p(Bbus), B_server, t, q_only, elem, lambda_sync, _p(x),
+                              _p(Ti), ctypes.byref(Ts), ctypes.byref(T))
+    return x, Ti, Ts.value, T.value, int(br)
+
+
 def row_prefix(m: int, u, perm_row) -> np.ndarray:
     u, pr = _i32(u), _i32(perm_row)
     S = np.empty(m + 1, dtype=np.int64)
@@ -199,6 +214,15 @@ def epoch(sched, sync, G, Br, Bc, off, n, k, gamma, lam, ru, rv, rr, P, Q):
         raise ValueError("oracle epoch: invalid grid for this schedule")
 
 
+def epoch_phased(G, Br, Bc, phases, off, n, k, gamma, lam, ru, rv, rr, P, Q):
+    """All-reduce epoch with `phases` sub-epoch syncs (serial inside each replica)."""
+    off = np.ascontiguousarray(off, dtype=np.int64)
+    rc = lib().orc_epoch_phased(G, Br, Bc, phases, _p(off), n, P.shape[1], gamma, lam, _p(ru), _p(rv), _p(rr),
+                                _p(P), _p(Q))
+    if rc != 0:
+        raise ValueError("oracle phased epoch: Br must be a multiple of phases")
+
+
 def rmse(tu, tv, tr, perm_row, perm_col, P, Q) -> float:
     tu, tv, tr = _i32(tu), _i32(tv), _f32(tr)
     return float(lib().orc_rmse(len(tu), _p(tu), _p(tv), _p(tr), P.shape[1], _p(_i32(perm_row)),
@@ -247,6 +271,10 @@ class Problem:
     def epoch(self, sched="det", sync="none"):
         epoch(sched, sync, self.G, self.Br, self.Bc, self.off, self.n, self.k, self.gamma, self.lam,
               self.ru, self.rv, self.rr, self.P, self.Q)
+
+    def epoch_phased(self, phases):
+        epoch_phased(self.G, self.Br, self.Bc, phases, self.off, self.n, self.k, self.gamma, self.lam, self.ru,
+                     self.rv, self.rr, self.P, self.Q)
 
     def factors(self):
         return unpermute(self.perm_row, self.P), unpermute(self.perm_col, self.Q)

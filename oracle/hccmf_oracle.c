@@ -440,3 +440,72 @@ void orc_unpermute(int64_t rows, int32_t k, const int32_t* perm, const double* X
     for (int64_t i = 0; i < rows; ++i)
         memcpy(X + i * k, Xp + (int64_t)perm[i] * k, sizeof(double) * (size_t)k);
 }
+
+/* ------------------------------------------------------------------------- */
+/* Time cost model (section 3.2, Eq. 1-5) and the strategy choice    */
+/* (section 3.3): per worker i with runtime memory bandwidth B_i and bus        */
+/* bandwidth Bbus_i, elem bytes per parameter (R18):                           */
+/*   T_i,e   = nnz (16k + 4) / B_i                       (whole data, Eq. 2)   */
+/*   x       = DP0 (Eq. 6 on T_i,e)                                            */
+/*   T_i     = x_i nnz (16k + 4) / B_i + 2 elem k D / Bbus_i   (Eq. 2)          */
+/*   T_sync  = 3 t elem k D / B_server                        (Eq. 3)          */
+/*   D = n (Strategy 1, only Q moves, L1203-L1233) or m + n                     */
+/*   T = max T_i           if max T_i / T_sync >= lambda_sync  (Eq. 5)         */
+/*     = max T_i + T_sync  otherwise                                           */
+/* Returns 1 when the sync term is negligible (DP1 applies), 2 otherwise (DP2). */
+/* ------------------------------------------------------------------------- */
+int32_t orc_cost_model(int32_t p, int64_t m, int64_t n, int64_t nnz, int32_t k, const double* B,
+                       const double* Bbus, double B_server, int32_t t, int32_t q_only, int32_t elem,
+                       double lambda_sync, double* x, double* T_i, double* T_sync, double* T)
+{
+    double D = q_only ? (double)n : (double)(m + n);
+    double* Te = (double*)malloc(sizeof(double) * (size_t)p);
+    for (int32_t i = 0; i < p; ++i) Te[i] = (double)nnz * (16.0 * k + 4.0) / B[i];
+    orc_dp0(p, Te, x);
+    double Tmax = 0.0;
+    for (int32_t i = 0; i < p; ++i) {
+        T_i[i] = x[i] * (double)nnz * (16.0 * k + 4.0) / B[i] + 2.0 * elem * k * D / Bbus[i];
+        if (T_i[i] > Tmax) Tmax = T_i[i];
+    }
+    *T_sync = 3.0 * t * elem * k * D / B_server;
+    free(Te);
+    if (Tmax / *T_sync >= lambda_sync) {
+        *T = Tmax;
+        return 1;
+    }
+    *T = Tmax + *T_sync;
+    return 2;
+}
+
+/* Sub-epoch synchronisation (Strategy 3's several pull-compute-push
+ * pipelines per epoch, L1251-L1269, Fig. 6; R22): the all-reduce mode in
+ * `phases` rounds.  Round phi runs, on every shard's own copy of Q, the shard's row
+ * blocks [phi*Br/phases, (phi+1)*Br/phases) -- every column block of each, records
+ * in stored order -- and then Q = (sum_s Q_s) / G.  phases = 1 is
+ * orc_epoch(serial, allreduce).  Needs Br % phases == 0; returns -1 otherwise. */
+int orc_epoch_phased(int32_t G, int32_t Br, int32_t Bc, int32_t phases, const int64_t* off, int64_t n,
+                     int32_t k, double gamma, double lambda, const int32_t* ru, const int32_t* rv,
+                     const float* rr, double* P, double* Q)
+{
+    if (phases < 1 || Br % phases != 0) return -1;
+    int32_t per = Br / phases;
+    size_t qn = (size_t)n * (size_t)k;
+    double* Qs = (double*)malloc(sizeof(double) * qn);
+    double* Qsum = (double*)malloc(sizeof(double) * qn);
+    for (int32_t ph = 0; ph < phases; ++ph) {
+        memset(Qsum, 0, sizeof(double) * qn);
+        for (int32_t s = 0; s < G; ++s) {
+            memcpy(Qs, Q, sizeof(double) * qn);
+            for (int32_t rb = ph * per; rb < (ph + 1) * per; ++rb)
+                for (int32_t cb = 0; cb < Bc; ++cb) {
+                    int64_t blk = ((int64_t)s * Br + rb) * Bc + cb;
+                    orc_run(off[blk], off[blk + 1], k, gamma, lambda, ru, rv, rr, P, Qs);
+                }
+            for (size_t i = 0; i < qn; ++i) Qsum[i] += Qs[i];
+        }
+        for (size_t i = 0; i < qn; ++i) Q[i] = Qsum[i] / (double)G;
+    }
+    free(Qs);
+    free(Qsum);
+    return 0;
+}

@@ -34,7 +34,7 @@ STATUS = {0: "OK", -1: "EINVAL", -2: "ERANGE", -3: "ENOMEM", -4: "ESTATE", -5: "
 SCHED = {"det": 0, "hogwild": 1}
 SYNC = {"none": 0, "ring": 1, "allreduce": 2}
 DP = {"DP0": 0, "DP1": 1, "DP2": 2}
-OPT = {"hogwild_warps": 1, "task_ratings": 2, "sync_stream": 3, "hogwild_atomic": 5, "conflict_ratio": 6, "heavy_first": 7, "vec": 8, "det_wave": 9}
+OPT = {"hogwild_warps": 1, "task_ratings": 2, "sync_stream": 3, "hogwild_atomic": 5, "conflict_ratio": 6, "heavy_first": 7, "vec": 8, "det_wave": 9, "sync_phases": 10}
 
 
 class HccmfError(RuntimeError):
@@ -46,7 +46,8 @@ class HccmfError(RuntimeError):
 class PartitionOpts(ctypes.Structure):
     _fields_ = [("n_shards", ctypes.c_int32), ("grid_rows", ctypes.c_int32), ("grid_cols", ctypes.c_int32),
                 ("strategy", ctypes.c_int32), ("x", ctypes.c_void_p), ("t_meas", ctypes.c_void_p),
-                ("t_sync", ctypes.c_double), ("seed", ctypes.c_uint64), ("storage", ctypes.c_int32)]
+                ("t_sync", ctypes.c_double), ("seed", ctypes.c_uint64), ("storage", ctypes.c_int32),
+                ("grid_dim", ctypes.c_int32)]
 
 
 class Info(ctypes.Structure):
@@ -54,7 +55,8 @@ class Info(ctypes.Structure):
                 ("n_shards", ctypes.c_int32), ("shard_lo", ctypes.c_int32), ("shard_hi", ctypes.c_int32),
                 ("local_nnz", ctypes.c_int64), ("row0", ctypes.c_int64), ("rows", ctypes.c_int64),
                 ("n_blocks", ctypes.c_int64), ("n_tasks", ctypes.c_int64), ("key_bits", ctypes.c_int32),
-                ("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("device_bytes", ctypes.c_int64)]
+                ("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("device_bytes", ctypes.c_int64),
+                ("transposed", ctypes.c_int32)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -91,6 +93,8 @@ def lib():
             "hccmf_get_info": (st, [P, ctypes.POINTER(Info)]),
             "hccmf_version": (ctypes.c_char_p, []),
             "hccmf_schedule": (st, [i32, i32, i32, i64, i32, i32, i32, P, P, P, P, P, P]),
+            "hccmf_cost_model": (st, [i32, i64, i64, i64, i32, P, P, ctypes.c_double, i32, i32, i32,
+                                      ctypes.c_double, P, P, P, P, P]),
         }
         for name, (res, args) in sig.items():
             fn = getattr(L, name)
@@ -139,6 +143,22 @@ def schedule(G, Br, Bc, n, sched="det", sync="none", shard=-1):
         raise HccmfError(code, L.hccmf_last_error(None).decode())
     launches = [blocks[off[i]:off[i + 1]] for i in range(nl.value)]
     return launches, stage, ring
+
+
+def cost_model(m, n, nnz, k, B, Bbus, B_server, t=1, q_only=True, elem_bytes=4, lambda_sync=10.0):
+    """Section 3.2 time cost model (Eq. 1-5): returns (x, T_i, T_sync, T, strategy name)."""
+    B = np.ascontiguousarray(B, np.float64)
+    Bbus = np.ascontiguousarray(Bbus, np.float64)
+    p = len(B)
+    x, Ti = np.empty(p), np.empty(p)
+    Ts, T, strat = ctypes.c_double(), ctypes.c_double(), ctypes.c_int32()
+    L = lib()
+    code = L.hccmf_cost_model(p, m, n, nnz, k, B.ctypes.data, Bbus.ctypes.data, float(B_server), t, int(q_only),
+                              elem_bytes, float(lambda_sync), x.ctypes.data, Ti.ctypes.data, ctypes.byref(Ts),
+                              ctypes.byref(T), ctypes.byref(strat))
+    if code != OK:
+        raise HccmfError(code, L.hccmf_last_error(None).decode())
+    return x, Ti, Ts.value, T.value, {1: "DP1", 2: "DP2"}[strat.value]
 
 
 class Model:
@@ -211,11 +231,15 @@ class Model:
         assert len(kv) == nnz and len(kr) == nnz, "u, v, r must have the same length"
         self._check(lib().hccmf_load_ratings(self._h, pu, pv, pr, nnz))
 
-    def partition(self, n_shards=1, grid=(1, 1), strategy="DP0", seed=0, x=None, t_meas=None, t_sync=0.0):
+    def partition(self, n_shards=1, grid=(1, 1), strategy="DP0", seed=0, x=None, t_meas=None, t_sync=0.0,
+                  grid_dim="rows"):
+        """grid_dim: "rows" (shards of users, Q moves), "cols" (shards of items, P moves) or
+        "auto" (the paper's rule, L884-L886)."""
         px, kx = _buf(x, np.float64)
         pt, kt = _buf(t_meas, np.float64)
         o = PartitionOpts(int(n_shards), int(grid[0]), int(grid[1]), DP[strategy] if isinstance(strategy, str)
-                          else int(strategy), px, pt, float(t_sync), int(seed), 0)
+                          else int(strategy), px, pt, float(t_sync), int(seed), 0,
+                          {"rows": 0, "cols": 1, "auto": 2}[grid_dim])
         self._check(lib().hccmf_partition(self._h, ctypes.byref(o)))
         self.G, self.grid = int(n_shards), (int(grid[0]), int(grid[1]))
 
@@ -261,8 +285,8 @@ class Model:
         inf = self.info()
         b = np.empty(inf["n_shards"] + 1, np.int32)
         off = np.empty(inf["n_blocks"] + 1, np.int64)
-        pr = np.empty(self.m, np.int32)
-        pc = np.empty(self.n, np.int32)
+        pr = np.empty(inf["m"], np.int32)
+        pc = np.empty(inf["n"], np.int32)
         self._check(lib().hccmf_get_partition(self._h, b.ctypes.data, off.ctypes.data, pr.ctypes.data,
                                               pc.ctypes.data))
         return b, off, pr, pc

@@ -198,11 +198,11 @@ void free_partition(hccmf_t h) {
 // order of DESIGN.md R19.
 struct BlockLaunch {
   std::vector<int64_t> blocks;
-  int32_t qrep, stage;
+  int32_t qrep, stage, phase = 0;
 };
 
 const char* schedule_blocks(int G, int Br, int Bc, int sched, int sync, int shard_lo, int shard_hi,
-                            std::vector<BlockLaunch>& out, int* n_stages) {
+                            std::vector<BlockLaunch>& out, int* n_stages, int phases = 1) {
   out.clear();
   *n_stages = 1;
   auto blk = [&](int64_t s, int64_t rb, int64_t cb) { return (s * Br + rb) * Bc + cb; };
@@ -246,6 +246,17 @@ const char* schedule_blocks(int G, int Br, int Bc, int sched, int sync, int shar
           }
           out.push_back(L);
         }
+    } else if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && phases > 1) {
+      // sub-epoch sync (R22): round ph runs row blocks [ph Br/phases, (ph+1) Br/phases)
+      if (Br % phases != 0) return "sync phases must divide grid_rows";
+      const int per = Br / phases;
+      for (int ph = 0; ph < phases; ++ph)
+        for (int s = shard_lo; s < shard_hi; ++s)
+          for (int cb = 0; cb < Bc; ++cb) {
+            BlockLaunch L{{}, s - shard_lo, 0, ph};
+            for (int rb = ph * per; rb < (ph + 1) * per; ++rb) L.blocks.push_back(blk(s, rb, cb));
+            out.push_back(L);
+          }
     } else {
       // column-block-major phases: a user's p_u is touched by one task per launch
       for (int s = shard_lo; s < shard_hi; ++s)
@@ -268,7 +279,7 @@ void ring_cols(int64_t n, int G, int Br, int Bc, int sched, int g, int64_t* a, i
 
 hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
   for (auto& p : h->plans)
-    if (p.sched == sched && p.sync == sync) {
+    if (p.sched == sched && p.sync == sync && p.phases == (sched == HCCMF_SCHED_HOGWILD ? (int)h->opt_phases : 1)) {
       *out = &p;
       return HCCMF_OK;
     }
@@ -276,8 +287,10 @@ hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
   Plan pl;
   pl.sched = sched;
   pl.sync = sync;
-  const char* msg = schedule_blocks(h->G, h->Br, h->Bc, sched, sync, h->shard_lo, h->shard_hi, bl, &pl.n_stages);
+  const char* msg = schedule_blocks(h->G, h->Br, h->Bc, sched, sync, h->shard_lo, h->shard_hi, bl, &pl.n_stages,
+                                    sched == HCCMF_SCHED_HOGWILD ? (int)h->opt_phases : 1);
   if (msg) return fail(h, HCCMF_EINVAL, "%s", msg);
+  pl.phases = sched == HCCMF_SCHED_HOGWILD ? (int)h->opt_phases : 1;
   std::vector<int64_t> lo, hi;
   for (const BlockLaunch& L : bl) {
     const int64_t t0 = (int64_t)lo.size();
@@ -296,7 +309,7 @@ hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
         }
       }
     }
-    pl.launches.push_back(Launch{t0, (int64_t)lo.size() - t0, L.qrep, L.stage});
+    pl.launches.push_back(Launch{t0, (int64_t)lo.size() - t0, L.qrep, L.stage, L.phase});
   }
   pl.n_tasks = (int64_t)lo.size();
   CU(h, dmalloc(h, &pl.d_lo, pl.n_tasks));
@@ -454,6 +467,10 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
     case HCCMF_OPT_HOGWILD_ATOMIC:
       h->opt_atomic = value != 0;
       return HCCMF_OK;
+    case HCCMF_OPT_SYNC_PHASES:
+      if (value < 1) return fail(h, HCCMF_EINVAL, "sync phases must be >= 1");
+      h->opt_phases = value;
+      return HCCMF_OK;
     case HCCMF_OPT_DET_WAVE:
       h->opt_wave = value != 0;
       return HCCMF_OK;
@@ -496,6 +513,10 @@ hccmf_status hccmf_load_ratings(hccmf_t h, const int32_t* u, const int32_t* v, c
   dfree(h, h->d_in_u, h->nnz);
   dfree(h, h->d_in_v, h->nnz);
   dfree(h, h->d_in_r, h->nnz);
+  if (h->transposed) {  // back to the caller's orientation
+    std::swap(h->m, h->n);
+    h->transposed = false;
+  }
   h->state = 0;
   h->nnz = nnz;
   CU(h, dmalloc(h, &h->d_in_u, nnz));
@@ -529,12 +550,24 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   const int G = o->n_shards;
   if (G < 1) return fail(h, HCCMF_EINVAL, "n_shards must be >= 1");
   if (h->world > 1 && G != h->world) return fail(h, HCCMF_EINVAL, "n_shards must equal the world size");
-  if (G > h->m) return fail(h, HCCMF_EINVAL, "n_shards must be <= m");
   if (o->grid_rows < 1 || o->grid_cols < 1) return fail(h, HCCMF_EINVAL, "grid must be >= 1 x 1");
   if (o->storage != 0) return fail(h, HCCMF_EINVAL, "only fp32 storage (0) is implemented");
   if (o->strategy < HCCMF_DP0 || o->strategy > HCCMF_DP2) return fail(h, HCCMF_EINVAL, "bad strategy");
   if ((o->strategy != HCCMF_DP0) && !o->t_meas) return fail(h, HCCMF_EINVAL, "DP1/DP2 need t_meas");
+  if (o->grid_dim < 0 || o->grid_dim > 2) return fail(h, HCCMF_EINVAL, "grid_dim must be 0, 1 or 2");
   free_partition(h);
+  // row grid or column grid (L881-L886): a column grid is the row grid of R^T with
+  // the roles of P and Q swapped; only the caller-facing calls swap back
+  {
+    const int64_t rows_now = h->transposed ? h->n : h->m, cols_now = h->transposed ? h->m : h->n;
+    const bool want_t = o->grid_dim == 1 || (o->grid_dim == 2 && cols_now > rows_now);
+    if (want_t != h->transposed) {
+      std::swap(h->d_in_u, h->d_in_v);
+      std::swap(h->m, h->n);
+      h->transposed = want_t;
+    }
+  }
+  if (G > h->m) return fail(h, HCCMF_EINVAL, "n_shards must be <= the number of grid rows");
 
   // ---- a3 partition fractions (host planner, section 3.3)
   std::vector<double> x(G, 1.0 / G);
@@ -697,8 +730,10 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
 hccmf_status hccmf_init_factors(hccmf_t h, uint64_t seed) {
   ENTER(h);
   if (h->state < 2) return fail(h, HCCMF_ESTATE, "init_factors needs partition first");
-  CU(h, k_init_factors(seed, 3, h->m, h->k, h->d_perm_row, h->row0, h->rows, h->d_P, h->stream));
-  CU(h, k_init_factors(seed, 4, h->n, h->k, h->d_perm_col, 0, h->n, h->d_Q, h->stream));
+  // R5: users draw from tag 3, items from tag 4, whatever the grid orientation
+  const uint64_t trow = h->transposed ? 4 : 3, tcol = h->transposed ? 3 : 4;
+  CU(h, k_init_factors(seed, trow, h->m, h->k, h->d_perm_row, h->row0, h->rows, h->d_P, h->stream));
+  CU(h, k_init_factors(seed, tcol, h->n, h->k, h->d_perm_col, 0, h->n, h->d_Q, h->stream));
   h->q_ring_sched = -1;
   h->state = 3;
   return finish(h);
@@ -708,6 +743,7 @@ hccmf_status hccmf_set_factors(hccmf_t h, const float* P, const float* Q) {
   ENTER(h);
   if (h->state < 2) return fail(h, HCCMF_ESTATE, "set_factors needs partition first");
   if (!P || !Q) return fail(h, HCCMF_EINVAL, "P and Q are required");
+  if (h->transposed) std::swap(P, Q);
   const size_t mk = (size_t)h->m * h->k, nk = (size_t)h->n * h->k;
   float* tmp = nullptr;
   CU(h, cudaMallocAsync((void**)&tmp, sizeof(float) * std::max(mk, nk), h->stream));
@@ -756,10 +792,22 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     if (st != HCCMF_OK) return st;
   }
   const int nrep = h->shard_hi - h->shard_lo;
-  if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && !dist) {
+  auto replicate = [&]() -> hccmf_status {  // logical all-reduce: every shard starts from Q
     if (!h->d_Qrep) CU(h, dmalloc(h, &h->d_Qrep, (size_t)nk * nrep));
     for (int r = 0; r < nrep; ++r)
       CU(h, cudaMemcpyAsync(h->d_Qrep + (size_t)r * nk, h->d_Q, sizeof(float) * nk, cudaMemcpyDeviceToDevice, s));
+    return HCCMF_OK;
+  };
+  auto average = [&]() -> hccmf_status {  // the server's sync (L549-L557): Q = mean of the shards' Q
+    if (dist)
+      NC(h, ncclAllReduce(h->d_Q, h->d_Q, (size_t)nk, ncclFloat, ncclAvg, h->comm, s));
+    else
+      CU(h, k_average(h->d_Qrep, nrep, nk, h->d_Q, s));
+    return HCCMF_OK;
+  };
+  if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && !dist) {
+    st = replicate();
+    if (st != HCCMF_OK) return st;
   }
   CU(h, cudaMemsetAsync(h->d_counters, 0, sizeof(unsigned long long) * pl->launches.size(), s));
   SgdArgs a{};
@@ -777,8 +825,18 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   // a ring stage races only on its column group's items
   const int64_t hog_warps = auto_warps(h, eff_sync == HCCMF_SYNC_RING ? h->n / G : h->n);
   int stage = 0;
+  int phase = 0;
   for (size_t li = 0; li < pl->launches.size(); ++li) {
     const Launch& ln = pl->launches[li];
+    if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && ln.phase != phase) {  // sub-epoch sync (R22)
+      st = average();
+      if (st != HCCMF_OK) return st;
+      if (!dist) {
+        st = replicate();
+        if (st != HCCMF_OK) return st;
+      }
+      phase = ln.phase;
+    }
     if (dist && eff_sync == HCCMF_SYNC_RING) {
       while (stage < ln.stage) {
         st = ring_exchange(h, sched, stage++);
@@ -802,10 +860,8 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     h->q_ring_sched = sched;
   }
   if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG) {
-    if (dist)
-      NC(h, ncclAllReduce(h->d_Q, h->d_Q, (size_t)nk, ncclFloat, ncclAvg, h->comm, s));
-    else
-      CU(h, k_average(h->d_Qrep, nrep, nk, h->d_Q, s));
+    st = average();
+    if (st != HCCMF_OK) return st;
   }
   return finish(h);
 }
@@ -815,6 +871,7 @@ hccmf_status hccmf_rmse(hccmf_t h, const int32_t* u, const int32_t* v, const flo
   if (!out) return fail(h, HCCMF_EINVAL, "out is NULL");
   if (h->state < 3) return fail(h, HCCMF_ESTATE, "rmse needs factors");
   if (nt < 0 || (nt > 0 && (!u || !v || !r))) return fail(h, HCCMF_EINVAL, "bad test set");
+  if (h->transposed) std::swap(u, v);
   hccmf_status st = materialize_q(h);
   if (st != HCCMF_OK) return st;
   cudaStream_t s = h->stream;
@@ -856,6 +913,7 @@ hccmf_status hccmf_rmse(hccmf_t h, const int32_t* u, const int32_t* v, const flo
 hccmf_status hccmf_get_factors(hccmf_t h, float* P, float* Q) {
   ENTER(h);
   if (h->state < 3) return fail(h, HCCMF_ESTATE, "get_factors needs factors");
+  if (h->transposed) std::swap(P, Q);
   cudaStream_t s = h->stream;
   const size_t mk = (size_t)h->m * h->k, nk = (size_t)h->n * h->k;
   if (P) {
@@ -957,6 +1015,39 @@ hccmf_status hccmf_schedule(int32_t G, int32_t Br, int32_t Bc, int64_t n, int32_
   return HCCMF_OK;
 }
 
+hccmf_status hccmf_cost_model(int32_t p, int64_t m, int64_t n, int64_t nnz, int32_t k, const double* B,
+                              const double* Bbus, double B_server, int32_t t, int32_t q_only, int32_t elem_bytes,
+                              double lambda_sync, double* x, double* T_i, double* T_sync, double* T,
+                              int32_t* strategy) {
+  if (p < 1 || m < 1 || n < 1 || nnz < 0 || k < 1 || !B || !Bbus || !x || !T_i || !T_sync || !T || !strategy ||
+      !(B_server > 0.0) || t < 0 || elem_bytes < 1)
+    return fail(nullptr, HCCMF_EINVAL, "bad cost model arguments");
+  for (int i = 0; i < p; ++i)
+    if (!(B[i] > 0.0) || !(Bbus[i] > 0.0)) return fail(nullptr, HCCMF_EINVAL, "bandwidths must be > 0");
+  // section 3.2: bytes per rating 16k + 4 (L741-L742); parameters moved D k elem (R18)
+  const double D = q_only ? (double)n : (double)(m + n);
+  const double per_rating = 16.0 * k + 4.0;
+  std::vector<double> Te(p);
+  for (int i = 0; i < p; ++i) Te[i] = (double)nnz * per_rating / B[i];  // independent execution time
+  std::vector<double> xv;
+  plan_dp0(p, Te.data(), xv);  // Eq. 6
+  double Tmax = 0.0;
+  for (int i = 0; i < p; ++i) {
+    x[i] = xv[i];
+    T_i[i] = xv[i] * (double)nnz * per_rating / B[i] + 2.0 * elem_bytes * k * D / Bbus[i];  // Eq. 2
+    Tmax = std::max(Tmax, T_i[i]);
+  }
+  *T_sync = 3.0 * t * elem_bytes * k * D / B_server;  // Eq. 3
+  if (Tmax / *T_sync >= lambda_sync) {  // Eq. 5: synchronisation negligible -> balance (DP1)
+    *T = Tmax;
+    *strategy = HCCMF_DP1;
+  } else {  // hide the synchronisation (DP2)
+    *T = Tmax + *T_sync;
+    *strategy = HCCMF_DP2;
+  }
+  return HCCMF_OK;
+}
+
 hccmf_status hccmf_get_info(hccmf_t h, hccmf_info* o) {
   if (!h || !o) return fail(h, HCCMF_EINVAL, "NULL argument");
   memset(o, 0, sizeof(*o));
@@ -976,6 +1067,7 @@ hccmf_status hccmf_get_info(hccmf_t h, hccmf_info* o) {
   o->rank = h->rank;
   o->world = h->world;
   o->device_bytes = (int64_t)h->device_bytes;
+  o->transposed = h->transposed ? 1 : 0;
   return HCCMF_OK;
 }
 

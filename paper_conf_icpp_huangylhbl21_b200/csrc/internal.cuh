@@ -36,6 +36,7 @@ struct Launch {
   int64_t t0, nt;
   int32_t qrep;
   int32_t stage;
+  int32_t phase;  // all-reduce sub-epoch round (R22)
 };
 
 struct Plan {
@@ -45,6 +46,7 @@ struct Plan {
   int64_t n_tasks = 0;
   std::vector<Launch> launches;
   int32_t n_stages = 1;
+  int32_t phases = 1;
 };
 
 struct SgdArgs {
@@ -127,7 +129,7 @@ struct hccmf_ctx {
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 4, opt_heavy = 1024, opt_vec = 0, opt_wave = 1;
+  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 4, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1;
   bool sync_stream = true;
   size_t device_bytes = 0;
 
@@ -170,6 +172,7 @@ struct hccmf_ctx {
   int64_t* d_blk_off = nullptr;  // local block offsets (DET wavefront), nblk_local + 1
   int* d_progress = nullptr;     // wavefront progress counters, Br
 
+  bool transposed = false;  // column grid: internal rows are the caller's columns
   int q_ring_sched = -1;  // >= 0: distributed ring left only this rank's Q group valid
   std::vector<hccmf::Plan> plans;
 };

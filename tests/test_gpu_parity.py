@@ -320,3 +320,59 @@ def test_det_wavefront_equals_strata(pkg, orc, k, B):
     assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
     Po, Qo = prob.factors()
     assert max(np.abs(outs[0][0] - Po).max(), np.abs(outs[0][1] - Qo).max()) <= 1e-4
+
+
+def test_column_grid_is_the_transposed_row_grid(pkg, orc):
+    # f3 / L881-L886: a column grid = the row grid of R^T with P and Q swapped;
+    # only P would move between shards ("transmitting P only", L1216-L1218)
+    m, n, k, B, G = 300, 700, 16, 4, 2
+    (u, v, r), (tu, tv, tr) = synth.planted(m, n, 20000, 2000, seed=4)
+    rng = np.random.default_rng(1)
+    P0 = rng.uniform(0, 0.3, (m, k)).astype(np.float32)
+    Q0 = rng.uniform(0, 0.3, (n, k)).astype(np.float32)
+    prob = orc.Problem(n, m, k, 0.05, 0.01, v, u, r, G=G, Br=B, Bc=G * B, seed=8)  # R^T
+    prob.set_factors(Q0, P0)
+    mdl = pkg.Model(m, n, k, 0.05, 0.01)
+    mdl.load(u, v, r)
+    mdl.partition(G, (B, G * B), seed=8, grid_dim="cols")
+    assert mdl.info()["transposed"] == 1 and mdl.info()["m"] == n
+    _check_partition(mdl, prob)
+    mdl.set_factors(P0, Q0)
+    assert mdl.rmse(tu, tv, tr) == pytest.approx(prob.rmse(tv, tu, tr), rel=1e-6)
+    for _ in range(2):
+        mdl.train_epoch("det", "ring")
+        prob.epoch("det", "ring")
+    P, Q = mdl.factors()
+    Qo, Po = prob.factors()
+    assert max(np.abs(P - Po).max(), np.abs(Q - Qo).max()) <= 1e-4
+    # the paper's rule picks columns here (n > m); init is orientation-independent
+    a = pkg.Model(m, n, k)
+    a.load(u, v, r)
+    a.partition(1, (1, 1), seed=8, grid_dim="auto")
+    assert a.info()["transposed"] == 1
+    a.init(9)
+    b = pkg.Model(m, n, k)
+    b.load(u, v, r)
+    b.partition(1, (1, 1), seed=8, grid_dim="rows")
+    b.init(9)
+    (Pa, Qa), (Pb, Qb) = a.factors(), b.factors()
+    assert np.array_equal(Pa, Pb) and np.array_equal(Qa, Qb)
+
+
+@pytest.mark.parametrize("phases", [2, 4])
+def test_hogwild_allreduce_sub_epoch_sync_band_c2(pkg, orc, phases):
+    # R22 / SURVEY f4: all-reduce with `phases` rounds per epoch vs the oracle's
+    # phased replica schedule (serial inside each replica), 20 epochs, C2 full size
+    cfg = synth.CONFIGS["c2"]
+    (u, v, r), (tu, tv, tr) = synth.make(cfg)
+    G, Br = 2, 4
+    prob = orc.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=1, seed=cfg.seed)
+    prob.init(1)
+    mdl = _gpu_problem(pkg, cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=1, seed=cfg.seed)
+    mdl.set_option("sync_phases", phases)
+    mdl.init(1)
+    for _ in range(20):
+        prob.epoch_phased(phases)
+        mdl.train_epoch("hogwild", "allreduce")
+    want, got = prob.rmse(tu, tv, tr), mdl.rmse(tu, tv, tr)
+    assert abs(got - want) <= 0.005, (want, got)

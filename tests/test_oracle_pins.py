@@ -273,3 +273,31 @@ def test_init_range_and_scale(orc):
     pr = orc.perm(3, 1, m)
     P2, _ = orc.init(5, m, n, k, pr, np.arange(n, dtype=np.int32))
     assert np.array_equal(P2[pr], P)
+
+
+def test_phased_allreduce_pins(orc):
+    # R22: phases = 1 is the plain all-reduce epoch (bit-exact); any phase count keeps
+    # the all-reduce first-order limit (P step gamma, Q step gamma / G)
+    import synth
+    m, n, k, G = 12, 9, 3, 3
+    u, v, r = synth.tiny(m, n, 60, seed=31)
+    a = orc.Problem(m, n, k, 0.01, 0.1, u, v, r, G=G, Br=4, Bc=2, seed=3)
+    b = orc.Problem(m, n, k, 0.01, 0.1, u, v, r, G=G, Br=4, Bc=2, seed=3)
+    a.init(2)
+    b.init(2)
+    a.epoch("serial", "allreduce")
+    b.epoch_phased(1)
+    assert np.array_equal(a.P, b.P) and np.array_equal(a.Q, b.Q)
+    with pytest.raises(ValueError):
+        b.epoch_phased(3)  # 4 row blocks cannot be split in 3 rounds
+    rng = np.random.default_rng(8)
+    P0, Q0 = rng.uniform(0, 1, (m, k)), rng.uniform(0, 1, (n, k))
+    gaps = []
+    for gamma in (1e-2, 5e-3, 2.5e-3):
+        p = orc.Problem(m, n, k, gamma, 0.1, u, v, r, G=G, Br=4, Bc=2, seed=3)
+        p.set_factors(P0, Q0)
+        p.epoch_phased(4)
+        P1, Q1 = p.factors()
+        Pg, Qg = _gd_step(u, v, r, 0.1, P0, Q0, gamma, gamma / G)
+        gaps.append(max(np.abs(P1 - Pg).max(), np.abs(Q1 - Qg).max()))
+    assert 0.2 < gaps[1] / gaps[0] < 0.3 and 0.2 < gaps[2] / gaps[1] < 0.3
