@@ -139,7 +139,7 @@ typedef enum {
                                     (racing writers may overwrite: the paper's
                                     "coverage", L1680-L1686)                      */
     HCCMF_OPT_CONFLICT_RATIO = 6,/* auto Hogwild concurrency: at most n / value
-                                    rating groups in flight (default 4; 0 = no cap) */
+                                    rating groups in flight (default 3; 0 = no cap) */
     HCCMF_OPT_HEAVY_FIRST = 7,   /* Hogwild task order inside a block: tasks with more
                                     than `value` ratings run first, longest first
                                     (no late heavy user stretches the epoch); the
