@@ -376,3 +376,38 @@ def test_hogwild_allreduce_sub_epoch_sync_band_c2(pkg, orc, phases):
         mdl.train_epoch("hogwild", "allreduce")
     want, got = prob.rmse(tu, tv, tr), mdl.rmse(tu, tv, tr)
     assert abs(got - want) <= 0.005, (want, got)
+
+
+def test_distributed_handle_world1_matches_single(pkg, orc):
+    # the NCCL code paths (unique-id bootstrap through torch.distributed, ncclCommInitRank,
+    # ncclAllReduce(ncclAvg) for Q and {sum, count} of the RMSE, broadcasts in get_factors)
+    # on a one-rank communicator: results equal the single-process handle bit for bit
+    import os
+    import socket
+    import torch.distributed as dist
+    sock = socket.socket()
+    sock.bind(("127.0.0.1", 0))
+    port = sock.getsockname()[1]
+    sock.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=0, world_size=1)
+    try:
+        cfg = synth.CONFIGS["c1"]
+        (u, v, r), (tu, tv, tr) = synth.make(cfg)
+        outs = []
+        for distributed in (True, False):
+            mdl = pkg.Model(cfg.m, cfg.n, 128, 0.02, cfg.lam, dist=distributed, device=0)
+            mdl.load(u, v, r)
+            mdl.partition(1, (8, 8), seed=4)
+            mdl.init(3)
+            mdl.set_option("hogwild_warps", 1)  # k = 128: one group in one warp, deterministic
+            for sched, sync in (("det", "none"), ("det", "allreduce"), ("hogwild", "ring")):
+                mdl.train_epoch(sched, sync)
+            outs.append((mdl.factors(), mdl.rmse(tu, tv, tr), mdl.info()["world"]))
+            mdl.close()
+        (Pd, Qd), rd, wd = outs[0]
+        (Ps, Qs), rs, ws = outs[1]
+        assert wd == 1 and ws == 1
+        assert np.array_equal(Pd, Ps) and np.array_equal(Qd, Qs) and rd == rs
+    finally:
+        dist.destroy_process_group()
