@@ -46,7 +46,7 @@ def parse():
     ap.add_argument("--config", default="c3", choices=sorted(synth.CONFIGS))
     ap.add_argument("--sched", default="hogwild", choices=["hogwild", "det"])
     ap.add_argument("--sync", default=None, choices=["none", "ring", "allreduce"])
-    ap.add_argument("--grid", default=None, help="Br,Bc (default: hogwild 1,G ; det 64,64*G)")
+    ap.add_argument("--grid", default=None, help="Br,Bc (default: hogwild 1,4G (ring) or 1,ceil(|Q|/80MB); det 64,64G)")
     ap.add_argument("--warps", type=int, default=0)
     ap.add_argument("--task", type=int, default=0)
     ap.add_argument("--vec", type=int, default=0, help="float4 slots per lane (0 = library auto)")
@@ -228,7 +228,11 @@ def main():
     if args.grid:
         Br, Bc = (int(x) for x in args.grid.split(","))
     elif args.sched == "hogwild":
-        Br, Bc = 1, (G if sync == "ring" else 1)
+        # ring: 4 column blocks per group so each block's transfer overlaps the next
+        # block's compute (hidden synchronisation); one GPU: column-block-major phases
+        # whenever Q exceeds ~80 MB of L2 (C4: 320 MB -> 4 phases)
+        qmb = cfg.n * cfg.k * 4 / 80e6
+        Br, Bc = 1, (4 * G if sync == "ring" else max(1, round(qmb)))
     else:
         Br, Bc = 64, 64 * (G if sync == "ring" else 1)
 

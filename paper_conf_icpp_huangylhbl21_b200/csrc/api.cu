@@ -364,6 +364,30 @@ hccmf_status ring_exchange(hccmf_t h, int sched, int t) {
   return HCCMF_OK;
 }
 
+// Hidden synchronisation (L1143-L1172) with asynchronous computing-transmission
+// (L1251-L1269): HOGWILD ring stages are launched one column block at a time; as soon
+// as column block j of stage t is done, the comm stream ships it to shard s-1 and
+// receives column block j of the next group from s+1, overlapping the transfer with
+// the compute of blocks j+1.. of the same stage.  Stage t+1's block j waits only for
+// its own block's receive.
+hccmf_status ring_exchange_block(hccmf_t h, int t, int j, cudaStream_t cs) {
+  const int G = h->G, s = h->rank, c = h->Bc / G;
+  auto rows = [&](int g, int64_t* a, int64_t* b) {
+    const int64_t cb = (int64_t)g * c + j;
+    *a = ceil_div(cb * h->n, h->Bc);
+    *b = ceil_div((cb + 1) * h->n, h->Bc);
+  };
+  int64_t sa, sb, ra, rb;
+  rows((s + t) % G, &sa, &sb);
+  rows((s + t + 1) % G, &ra, &rb);
+  const int prev = (s - 1 + G) % G, next = (s + 1) % G;
+  NC(h, ncclGroupStart());
+  if (sb > sa) NC(h, ncclSend(h->d_Q + sa * h->k, (size_t)(sb - sa) * h->k, ncclFloat, prev, h->comm, cs));
+  if (rb > ra) NC(h, ncclRecv(h->d_Q + ra * h->k, (size_t)(rb - ra) * h->k, ncclFloat, next, h->comm, cs));
+  NC(h, ncclGroupEnd());
+  return HCCMF_OK;
+}
+
 // after ring epochs rank s holds only group s of Q: broadcast every group from its owner
 hccmf_status materialize_q(hccmf_t h) {
   if (h->world <= 1 || h->q_ring_sched < 0) return HCCMF_OK;
@@ -500,6 +524,12 @@ void hccmf_destroy(hccmf_t h) {
   dfree(h, h->d_in_r, h->nnz);
   dfree(h, h->d_partials, 2 * RMSE_BLOCKS);
   dfree(h, h->d_scalar, 2);
+  for (auto e : h->ev_done) cudaEventDestroy(e);
+  for (auto e : h->ev_recv) cudaEventDestroy(e);
+  if (h->comm_stream) {
+    cudaStreamSynchronize(h->comm_stream);
+    cudaStreamDestroy(h->comm_stream);
+  }
   if (h->comm) ncclCommDestroy(h->comm);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   delete h;
@@ -824,6 +854,21 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   const int L = sgd_lanes(h->k, (int)h->opt_vec);
   // a ring stage races only on its column group's items
   const int64_t hog_warps = auto_warps(h, eff_sync == HCCMF_SYNC_RING ? h->n / G : h->n);
+  if (dist && eff_sync == HCCMF_SYNC_RING && sched == HCCMF_SCHED_HOGWILD) {
+    const size_t ne = (size_t)G * (h->Bc / G);
+    if (pl->launches.size() != ne) return fail(h, HCCMF_EINVAL, "ring plan: one launch per column block expected");
+    if (!h->comm_stream) CU(h, cudaStreamCreateWithFlags(&h->comm_stream, cudaStreamNonBlocking));
+    while (h->ev_done.size() < ne) {
+      cudaEvent_t a0, a1;
+      CU(h, cudaEventCreateWithFlags(&a0, cudaEventDisableTiming));
+      CU(h, cudaEventCreateWithFlags(&a1, cudaEventDisableTiming));
+      h->ev_done.push_back(a0);
+      h->ev_recv.push_back(a1);
+    }
+    // the comm stream must not run ahead of work already queued on the compute stream
+    CU(h, cudaEventRecord(h->ev_done[0], s));
+    CU(h, cudaStreamWaitEvent(h->comm_stream, h->ev_done[0], 0));
+  }
   int stage = 0;
   int phase = 0;
   for (size_t li = 0; li < pl->launches.size(); ++li) {
@@ -837,7 +882,12 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
       }
       phase = ln.phase;
     }
-    if (dist && eff_sync == HCCMF_SYNC_RING) {
+    const bool pipelined = dist && eff_sync == HCCMF_SYNC_RING && sched == HCCMF_SCHED_HOGWILD;
+    int jblk = 0;  // column block of this launch inside its stage (HOGWILD ring plans: one each)
+    if (pipelined) {
+      jblk = (int)(li % (size_t)(h->Bc / G));
+      if (ln.stage > 0) CU(h, cudaStreamWaitEvent(s, h->ev_recv[(size_t)(ln.stage - 1) * (h->Bc / G) + jblk], 0));
+    } else if (dist && eff_sync == HCCMF_SYNC_RING) {
       while (stage < ln.stage) {
         st = ring_exchange(h, sched, stage++);
         if (st != HCCMF_OK) return st;
@@ -851,8 +901,21 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     // DET: one rating group per block of the stratum; HOGWILD: persistent grid
     const int64_t warps = (sched == HCCMF_SCHED_DET) ? (ln.nt * L + 31) / 32 : hog_warps;
     CU(h, launch_sgd(a, warps, s));
+    if (pipelined) {
+      const size_t e = (size_t)ln.stage * (h->Bc / G) + jblk;
+      CU(h, cudaEventRecord(h->ev_done[e], s));
+      CU(h, cudaStreamWaitEvent(h->comm_stream, h->ev_done[e], 0));
+      st = ring_exchange_block(h, ln.stage, jblk, h->comm_stream);
+      if (st != HCCMF_OK) return st;
+      CU(h, cudaEventRecord(h->ev_recv[e], h->comm_stream));
+    }
   }
-  if (dist && eff_sync == HCCMF_SYNC_RING) {
+  if (dist && eff_sync == HCCMF_SYNC_RING && sched == HCCMF_SCHED_HOGWILD) {
+    // every transfer of the last stage lands before the epoch ends (shard s holds group s)
+    const int c = h->Bc / G;
+    for (int j = 0; j < c; ++j) CU(h, cudaStreamWaitEvent(s, h->ev_recv[(size_t)(G - 1) * c + j], 0));
+    h->q_ring_sched = sched;
+  } else if (dist && eff_sync == HCCMF_SYNC_RING) {
     while (stage < pl->n_stages) {
       st = ring_exchange(h, sched, stage++);
       if (st != HCCMF_OK) return st;

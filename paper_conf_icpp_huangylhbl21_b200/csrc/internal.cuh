@@ -126,6 +126,8 @@ struct hccmf_ctx {
   bool own_stream = false;
   int32_t rank = 0, world = 1;
   ncclComm_t comm = nullptr;
+  cudaStream_t comm_stream = nullptr;           // ring transfers overlapped with compute
+  std::vector<cudaEvent_t> ev_done, ev_recv;    // per (stage, column block)
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
