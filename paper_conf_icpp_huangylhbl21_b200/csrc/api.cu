@@ -807,6 +807,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     a.gamma = h->gamma;
     a.lambda = h->lambda;
     a.vec_pref = (int32_t)h->opt_vec;
+    a.prefetch = 1;
     CU(h, launch_wave(a, h->d_blk_off, h->Br, h->d_progress, h->stream));
     return finish(h);
   }
@@ -851,6 +852,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   a.lambda = h->lambda;
   a.atomic_q = (sched == HCCMF_SCHED_HOGWILD && h->opt_atomic) ? 1 : 0;
   a.vec_pref = (int32_t)h->opt_vec;
+  a.prefetch = sched == HCCMF_SCHED_DET ? 1 : 0;
   const int L = sgd_lanes(h->k, (int)h->opt_vec);
   // a ring stage races only on its column group's items
   const int64_t hog_warps = auto_warps(h, eff_sync == HCCMF_SYNC_RING ? h->n / G : h->n);

@@ -64,6 +64,7 @@ struct SgdArgs {
   unsigned long long* counter;
   int32_t atomic_q;  // Hogwild: apply q_v increments with vector atomics
   int32_t vec_pref;  // float4 slots per lane (0 = auto)
+  int32_t prefetch;  // L2 bulk prefetch of the next window's p_u / q_v rows (DET blocks)
 };
 
 // launch the SGD kernel for a list of tasks; warps = concurrent warps wanted

@@ -285,6 +285,15 @@ struct WarpSgd {
     for (int i = 0; i < VEC; ++i) __stcg(const_cast<float4*>(r) + 32 * i, x[i]);
   }
 
+  // bulk L2 prefetch of one rating's p_u and q_v rows (cp.async.bulk.prefetch, sm_90+)
+  __device__ __forceinline__ void prefetch_rows(int u, int v) const {
+    const unsigned bytes = (unsigned)k4 * 16u;
+    const float4* pr = reinterpret_cast<const float4*>(a.P) + (int64_t)(u - a.row0) * k4;
+    const float4* qr = reinterpret_cast<const float4*>(a.Q) + (int64_t)v * k4;
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(pr), "r"(bytes) : "memory");
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(qr), "r"(bytes) : "memory");
+  }
+
   // all ratings of records [lo, lo + left), left >= 1, in order
   __device__ __forceinline__ void run(int64_t lo, int left) {
     auto ld = [&](const float4* r, float4 (&x)[VEC]) { this->ld(r, x); };
@@ -299,6 +308,10 @@ struct WarpSgd {
     float wr0 = 0.f, wr1 = 0.f;
     if (lane < left) wu0 = __ldcs(ru + lane), wv0 = __ldcs(rv + lane), wr0 = __ldcs(rr + lane);
     if (lane + 32 < left) wu1 = __ldcs(ru + 32 + lane), wv1 = __ldcs(rv + 32 + lane), wr1 = __ldcs(rr + 32 + lane);
+    if (a.prefetch) {  // DET: every rating of the next 64 pulls its p_u / q_v rows into L2 now
+      if (lane < left) prefetch_rows(wu0, wv0);
+      if (lane + 32 < left) prefetch_rows(wu1, wv1);
+    }
     int wb = 0;  // first rating of window 0
     int cu = __shfl_sync(FM, wu0, 0), cv = __shfl_sync(FM, wv0, 0);
     float cr = __shfl_sync(FM, wr0, 0);
@@ -317,7 +330,10 @@ struct WarpSgd {
           wu0 = wu1, wv0 = wv1, wr0 = wr1;
           wb += 32;
           const int idx = wb + 32 + lane;
-          if (idx < left) wu1 = __ldcs(ru + idx), wv1 = __ldcs(rv + idx), wr1 = __ldcs(rr + idx);
+          if (idx < left) {
+            wu1 = __ldcs(ru + idx), wv1 = __ldcs(rv + idx), wr1 = __ldcs(rr + idx);
+            if (a.prefetch) prefetch_rows(wu1, wv1);
+          }
         }
         const int src = j + 1 - wb;
         nu = __shfl_sync(FM, wu0, src);
