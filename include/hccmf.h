@@ -31,7 +31,9 @@
  *    HCCMF_ESTATE.
  *  - All work is issued on the handle's CUDA stream (its own, or the one given
  *    to hccmf_set_stream); every call returns after that stream is synchronised
- *    unless stated otherwise, so host timing around a call is meaningful.
+ *    unless stated otherwise, so host timing around a call is meaningful.  The
+ *    handle's own stream is a blocking stream (ordered after the legacy default
+ *    stream); with hccmf_set_stream the caller orders device inputs itself.
  *  - Not thread-safe per handle; distinct handles are independent.
  *  - There is no CPU fallback: without a CUDA device every call that needs one
  *    returns HCCMF_ECUDA.

@@ -3,6 +3,7 @@
 // launch plans for every (schedule, sync) pair, the ring / all-reduce Q
 // synchronisation over NCCL, and export.
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -56,17 +57,21 @@ hccmf_status fail(hccmf_t h, hccmf_status st, const char* fmt, ...) {
     CU(h, cudaSetDevice((h)->device));                \
   } while (0)
 
+// Every device buffer of a handle comes from the device's stream-ordered pool on the
+// handle's stream.  The pool keeps its mapped memory (release threshold = max, set in
+// make_ctx), so repeated jobs and the syncs inside one partition reuse it instead of
+// mapping and unmapping gigabytes (C3 partition: 550 -> see DESIGN.md section 8).
 template <typename T>
 cudaError_t dmalloc(hccmf_t h, T** p, size_t count) {
   const size_t bytes = sizeof(T) * (count ? count : 1);
-  cudaError_t e = cudaMalloc((void**)p, bytes);
+  cudaError_t e = cudaMallocAsync((void**)p, bytes, h->stream);
   if (e == cudaSuccess) h->device_bytes += bytes;
   return e;
 }
 template <typename T>
 void dfree(hccmf_t h, T*& p, size_t count) {
   if (p) {
-    cudaFree((void*)p);
+    cudaFreeAsync((void*)p, h->stream);
     h->device_bytes -= sizeof(T) * (count ? count : 1);
   }
   p = nullptr;
@@ -77,6 +82,24 @@ hccmf_status finish(hccmf_t h) {
   if (h->sync_stream) CU(h, cudaStreamSynchronize(h->stream));
   return HCCMF_OK;
 }
+
+// HCCMF_PROFILE=1: per-phase wall times of the preprocessing on stderr (syncs the stream)
+struct PhaseTimer {
+  bool on;
+  cudaStream_t st;
+  std::chrono::steady_clock::time_point t0;
+  explicit PhaseTimer(cudaStream_t s) : on(getenv("HCCMF_PROFILE") != nullptr), st(s) {
+    if (on) cudaStreamSynchronize(st);
+    t0 = std::chrono::steady_clock::now();
+  }
+  void mark(const char* what) {
+    if (!on) return;
+    cudaStreamSynchronize(st);
+    const auto t1 = std::chrono::steady_clock::now();
+    fprintf(stderr, "[hccmf] %-28s %9.3f ms\n", what, std::chrono::duration<double, std::milli>(t1 - t0).count());
+    t0 = t1;
+  }
+};
 
 int bitlen(uint64_t x) {  // bits needed to represent x (0 -> 0)
   int b = 0;
@@ -104,7 +127,9 @@ hccmf_status make_ctx(int64_t m, int64_t n, int32_t k, float gamma, float lambda
   h->lambda = lambda;
   h->device = device;
   cudaError_t e = cudaSetDevice(device);
-  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking);
+  // a blocking stream: the handle's work is ordered after the legacy default stream, so
+  // device inputs a caller produced there (e.g. with torch) are complete before we copy
+  if (e == cudaSuccess) e = cudaStreamCreate(&h->stream);
   if (e != cudaSuccess) {
     hccmf_status st = fail(nullptr, HCCMF_ECUDA, "no usable CUDA device: %s", cudaGetErrorString(e));
     cudaGetLastError();
@@ -112,8 +137,25 @@ hccmf_status make_ctx(int64_t m, int64_t n, int32_t k, float gamma, float lambda
     return st;
   }
   h->own_stream = true;
+  // Keep what the stream-ordered pool maps (a release threshold of 0 unmaps and remaps
+  // gigabytes at every stream synchronisation; HCCMF_TRIM=1 trims at destroy).
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess) {
+    uint64_t keep = UINT64_MAX;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+  }
+  cudaGetLastError();
   *out = h;
   return HCCMF_OK;
+}
+
+void trim_pool(hccmf_t h) {
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, h->device) == cudaSuccess) {
+    cudaStreamSynchronize(h->stream);
+    cudaMemPoolTrimTo(pool, 0);
+  }
+  cudaGetLastError();
 }
 
 // ----------------------------------------------------------- DP planners
@@ -531,6 +573,8 @@ void hccmf_destroy(hccmf_t h) {
     cudaStreamDestroy(h->comm_stream);
   }
   if (h->comm) ncclCommDestroy(h->comm);
+  if (getenv("HCCMF_TRIM")) trim_pool(h);
+  if (h->stream) cudaStreamSynchronize(h->stream);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   delete h;
 }
@@ -616,12 +660,14 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   const int64_t m = h->m, n = h->n, nnz = h->nnz;
   cudaStream_t st = h->stream;
 
+  PhaseTimer timer(h->stream);
   // ---- a2 shuffle
   CU(h, dmalloc(h, &h->d_perm_row, m));
   CU(h, dmalloc(h, &h->d_perm_col, n));
   CU(h, k_perm(h->seed, 1, m, h->d_perm_row, st));
   CU(h, k_perm(h->seed, 2, n, h->d_perm_col, st));
 
+  timer.mark("a2 shuffle");
   // ---- a3 row histogram, prefix, boundaries
   unsigned long long* dS = nullptr;
   CU(h, cudaMallocAsync((void**)&dS, sizeof(unsigned long long) * (m + 1), st));
@@ -651,6 +697,7 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   CU(h, cudaMallocAsync((void**)&dB, sizeof(int32_t) * (G + 1), st));
   CU(h, cudaMemcpyAsync(dB, h->bounds.data(), sizeof(int32_t) * (G + 1), cudaMemcpyHostToDevice, st));
 
+  timer.mark("a3 histogram+bounds");
   // ---- a4 geometry + stable sort
   BlockGeom g{};
   g.G = G;
@@ -674,7 +721,9 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   CU(h, dmalloc(h, &sv, nnz));
   CU(h, dmalloc(h, &sr, nnz));
   CU(h, cudaMallocAsync((void**)&dOff, sizeof(int64_t) * (nblk + 1), st));
+  timer.mark("a4 alloc records");
   CU(h, k_block_sort(g, dB, h->d_perm_row, h->d_perm_col, h->d_in_u, h->d_in_v, h->d_in_r, nnz, su, sv, sr, dOff, st));
+  timer.mark("a4 key+sort+decode");
   h->block_off.assign(nblk + 1, 0);
   CU(h, cudaMemcpyAsync(h->block_off.data(), dOff, sizeof(int64_t) * (nblk + 1), cudaMemcpyDeviceToHost, st));
   CU(h, cudaStreamSynchronize(st));
@@ -683,7 +732,7 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   dfree(h, h->d_in_u, nnz);
   dfree(h, h->d_in_v, nnz);
   dfree(h, h->d_in_r, nnz);
-
+  timer.mark("a4 offsets + free input");
   // ---- local shard(s)
   const int64_t bps = (int64_t)h->Br * h->Bc;
   if (h->world > 1) {
@@ -718,6 +767,7 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   h->row0 = h->bounds[h->shard_lo];
   h->rows = (int64_t)h->bounds[h->shard_hi] - h->row0;
 
+  timer.mark("local shard");
   // ---- Hogwild tasks: user-aligned runs of ~opt_task ratings inside each block
   std::vector<int64_t> loc_off(h->nblk_local + 1);
   for (int64_t j = 0; j <= h->nblk_local; ++j) loc_off[j] = h->block_off[h->blk0 + j] - h->rec0;
@@ -748,12 +798,14 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   }
   for (int64_t j = 0; j < h->nblk_local; ++j) h->blk_task_off[j + 1] += h->blk_task_off[j];
 
+  timer.mark("hogwild tasks");
   // ---- factors
   CU(h, dmalloc(h, &h->d_P, h->rows * h->k));
   CU(h, dmalloc(h, &h->d_Q, h->n * h->k));
   if (!h->d_partials) CU(h, dmalloc(h, &h->d_partials, 2 * RMSE_BLOCKS));
   h->q_ring_sched = -1;
   h->state = 2;
+  timer.mark("factors alloc");
   return finish(h);
 }
 

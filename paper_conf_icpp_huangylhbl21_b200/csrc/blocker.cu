@@ -4,6 +4,11 @@
 // PAPER.md section 3.1 preprocessing "shuffling, sorting, and data partition"
 // (L543-L548), row grid (L881-L895), row-sorted blocks (L1472-L1474).  Every
 // step is integer work and bit-exact against the oracle (tests/test_gpu_*).
+#include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
+
 #include <cub/cub.cuh>
 #include <thrust/iterator/counting_iterator.h>
 
@@ -321,34 +326,50 @@ cudaError_t k_bound_search(const unsigned long long* S, int64_t m, const int64_t
   return cudaGetLastError();
 }
 
+static void bs_mark(cudaStream_t st, const char* what) {
+  static bool on = getenv("HCCMF_PROFILE") != nullptr;
+  if (!on) return;
+  static auto t0 = std::chrono::steady_clock::now();
+  cudaStreamSynchronize(st);
+  auto t1 = std::chrono::steady_clock::now();
+  fprintf(stderr, "[hccmf]   %-26s %9.3f ms\n", what, std::chrono::duration<double, std::milli>(t1 - t0).count());
+  t0 = t1;
+}
+
 cudaError_t k_block_sort(const BlockGeom& g, const int32_t* bounds, const int32_t* perm_row, const int32_t* perm_col,
                          const int32_t* u, const int32_t* v, const float* r, int64_t nnz, int32_t* ou, int32_t* ov,
                          float* orr, int64_t* block_off, cudaStream_t st) {
+  bs_mark(st, "bs: enter");
   const int64_t nblk = (int64_t)g.G * g.Br * g.Bc;
   const int bits = g.bb + g.bu + g.bv;
   uint64_t *k0 = nullptr, *k1 = nullptr;
   CKR(dalloc(&k0, nnz, st));
   CKR(dalloc(&k1, nnz, st));
+  bs_mark(st, "bs: alloc keys");
   if (nnz) {
     block_key_kernel<<<grid_for(nnz), kT, 0, st>>>(g, bounds, perm_row, perm_col, u, v, nnz, k0);
     CKR(cudaGetLastError());
   }
+  bs_mark(st, "bs: key kernel");
   const uint64_t* ks = k0;
   if (nnz && bits > 0) {
     size_t tb = 0;
     void* tmp = nullptr;
-    CKR(cub::DeviceRadixSort::SortPairs(nullptr, tb, k0, k1, r, orr, nnz, 0, bits, st));
+    const int end_bit = bits;
+    CKR(cub::DeviceRadixSort::SortPairs(nullptr, tb, k0, k1, r, orr, nnz, 0, end_bit, st));
     CKR(cudaMallocAsync(&tmp, tb, st));
-    CKR(cub::DeviceRadixSort::SortPairs(tmp, tb, k0, k1, r, orr, nnz, 0, bits, st));
+    CKR(cub::DeviceRadixSort::SortPairs(tmp, tb, k0, k1, r, orr, nnz, 0, end_bit, st));
     cudaFreeAsync(tmp, st);
     ks = k1;
   } else if (nnz) {
     CKR(cudaMemcpyAsync(orr, r, sizeof(float) * nnz, cudaMemcpyDeviceToDevice, st));
   }
+  bs_mark(st, "bs: radix sort");
   if (nnz) {
     block_decode_kernel<<<grid_for(nnz), kT, 0, st>>>(g, bounds, ks, nnz, ou, ov);
     CKR(cudaGetLastError());
   }
+  bs_mark(st, "bs: decode");
   block_off_kernel<<<grid_for(nblk + 1), kT, 0, st>>>(ks, nnz, g.bu + g.bv, nblk, block_off);
   CKR(cudaGetLastError());
   cudaFreeAsync(k0, st);
@@ -362,8 +383,8 @@ cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, i
   *task_lo = nullptr;
   *task_hi = nullptr;
   if (nrec == 0) {
-    CKR(cudaMalloc(task_lo, sizeof(int64_t)));
-    CKR(cudaMalloc(task_hi, sizeof(int64_t)));
+    CKR(cudaMallocAsync((void**)task_lo, sizeof(int64_t), st));
+    CKR(cudaMallocAsync((void**)task_hi, sizeof(int64_t), st));
     return cudaSuccess;
   }
   unsigned char* flag = nullptr;
@@ -434,8 +455,8 @@ cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, i
   CKR(cudaMallocAsync(&tmp, tb, st));
   CKR(cub::DeviceRadixSort::SortPairs(tmp, tb, sk0, sk1, ix0, ix1, nt, 0, 64, st));
   cudaFreeAsync(tmp, st);
-  CKR(cudaMalloc(task_lo, sizeof(int64_t) * (nt ? nt : 1)));
-  CKR(cudaMalloc(task_hi, sizeof(int64_t) * (nt ? nt : 1)));
+  CKR(cudaMallocAsync((void**)task_lo, sizeof(int64_t) * (nt ? nt : 1), st));
+  CKR(cudaMallocAsync((void**)task_hi, sizeof(int64_t) * (nt ? nt : 1), st));
   permute_tasks_kernel<<<grid_for(nt), kT, 0, st>>>(ix1, nt, lo, hi, *task_lo, *task_hi);
   CKR(cudaGetLastError());
   for (void* p : {(void*)flag, (void*)runs, (void*)nsel, (void*)ccnt, (void*)coff, (void*)cpos, (void*)keep,
