@@ -157,12 +157,18 @@ typedef enum {
                                     only for warp i+1's previous stratum) when the
                                     B warps fit on the device; 0: one launch per
                                     stratum.  Same update order either way.       */
-    HCCMF_OPT_SYNC_PHASES = 10   /* ALLREDUCE_AVG + HOGWILD: rounds per epoch (>= 1,
+    HCCMF_OPT_SYNC_PHASES = 10,  /* ALLREDUCE_AVG + HOGWILD: rounds per epoch (>= 1,
                                     default 1; must divide grid_rows).  Round ph runs
                                     every shard's row blocks [ph Br/S, (ph+1) Br/S)
                                     on its Q copy, then averages Q: the paper's
                                     several pull-compute-push pipelines per epoch
                                     (L1251-L1269, Fig. 6; R22).         */
+    HCCMF_OPT_WIRE_FP16 = 11     /* 1: Q travels as IEEE binary16 (Strategy 2,
+                                    "Transmitting FP16 Data", L1234-L1249): ring
+                                    transfers and the all-reduce pack to half and
+                                    unpack to fp32; factors stay fp32 (R25).  The
+                                    logical-shard backend applies the same rounding
+                                    at every stage boundary.  Default 0.          */
 } hccmf_option;
 
 /* ------------------------------------------------------------------ lifecycle */

@@ -509,3 +509,86 @@ int orc_epoch_phased(int32_t G, int32_t Br, int32_t Bc, int32_t phases, const in
     free(Qsum);
     return 0;
 }
+
+/* ------------------------------------------------------------------------- */
+/* Strategy 2, "Transmitting FP16 Data" (L1234-L1249): Q travels as IEEE-754     */
+/* binary16.  orc_round_half returns the binary16 value nearest to x (ties to    */
+/* even), as a double: the pack -> unpack a transfer applies.  Written from the */
+/* format's definition (1 sign, 5 exponent bits with bias 15, 10 fraction bits, */
+/* subnormals below 2^-14, largest finite 65504); overflow gives +-inf.          */
+/* ------------------------------------------------------------------------- */
+double orc_round_half(double x)
+{
+    if (x != x) return x;
+    double a = fabs(x);
+    if (a == 0.0) return x;
+    if (a >= 65520.0) return x > 0 ? INFINITY : -INFINITY; /* 65504 + half an ulp (16) rounds up */
+    int e;
+    frexp(a, &e);                        /* a = f * 2^e, f in [0.5, 1) -> leading bit 2^(e-1) */
+    int lead = e - 1;
+    if (lead < -14) lead = -14;          /* subnormal range: fixed spacing 2^-24 */
+    double ulp = ldexp(1.0, lead - 10);
+    double q = a / ulp;                  /* exact: ulp is a power of two */
+    double fl = floor(q), rem = q - fl;
+    double r = fl;
+    if (rem > 0.5 || (rem == 0.5 && fmod(fl, 2.0) != 0.0)) r = fl + 1.0;
+    double y = r * ulp;
+    if (y >= 65520.0) y = INFINITY;
+    return x < 0 ? -y : y;
+}
+
+/* Ring / all-reduce epoch with FP16 transmission (R25).  RING: after
+ * stage t, the column group each shard held, (s+t) mod G, has been shipped as
+ * binary16 -> its Q rows are rounded.  ALLREDUCE: every shard's copy is rounded
+ * before the mean and the mean is rounded again (it comes back as binary16).
+ * Same grid rules as orc_epoch. */
+int orc_epoch_wire16(int32_t sched, int32_t sync, int32_t G, int32_t Br, int32_t Bc, const int64_t* off,
+                     int64_t n, int32_t k, double gamma, double lambda, const int32_t* ru, const int32_t* rv,
+                     const float* rr, double* P, double* Q)
+{
+    if (sync == 1) {
+        if (Bc % G != 0) return -1;
+        int32_t c = Bc / G;
+        if (sched == 0 && c != Br) return -1;
+        for (int32_t t = 0; t < G; ++t) {
+            for (int32_t s = 0; s < G; ++s) {
+                int32_t g = (s + t) % G;
+                if (sched == 0) {
+                    det_square(s, c, Br, Bc, g * c, off, k, gamma, lambda, ru, rv, rr, P, Q);
+                } else {
+                    for (int32_t j = 0; j < c; ++j)
+                        for (int32_t rb = 0; rb < Br; ++rb) {
+                            int64_t blk = ((int64_t)s * Br + rb) * Bc + g * c + j;
+                            orc_run(off[blk], off[blk + 1], k, gamma, lambda, ru, rv, rr, P, Q);
+                        }
+                }
+            }
+            for (int32_t g = 0; g < G; ++g) { /* every group moved once at the end of stage t */
+                int64_t a = ((int64_t)g * c * n + Bc - 1) / Bc, b = ((int64_t)(g + 1) * c * n + Bc - 1) / Bc;
+                for (int64_t i = a * k; i < b * k; ++i) Q[i] = orc_round_half(Q[i]);
+            }
+        }
+        return 0;
+    }
+    if (sync == 2) {
+        if (sched == 0 && Br != Bc) return -1;
+        size_t qn = (size_t)n * (size_t)k;
+        double* Qs = (double*)malloc(sizeof(double) * qn);
+        double* Qsum = (double*)calloc(qn, sizeof(double));
+        for (int32_t s = 0; s < G; ++s) {
+            memcpy(Qs, Q, sizeof(double) * qn);
+            if (sched == 0) {
+                det_square(s, Br, Br, Bc, 0, off, k, gamma, lambda, ru, rv, rr, P, Qs);
+            } else {
+                int64_t lo = off[(int64_t)s * Br * Bc], hi = off[(int64_t)(s + 1) * Br * Bc];
+                orc_run(lo, hi, k, gamma, lambda, ru, rv, rr, P, Qs);
+            }
+            for (size_t i = 0; i < qn; ++i) Qsum[i] += orc_round_half(Qs[i]);
+        }
+        for (size_t i = 0; i < qn; ++i) Q[i] = orc_round_half(Qsum[i] / (double)G);
+        free(Qs);
+        free(Qsum);
+        return 0;
+    }
+    return -1;
+}

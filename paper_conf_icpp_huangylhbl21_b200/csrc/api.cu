@@ -392,6 +392,44 @@ void ring_group_cols(hccmf_t h, int sched, int g, int64_t* a, int64_t* b) {
   ring_cols(h->n, h->G, h->Br, h->Bc, sched, g, a, b);
 }
 
+hccmf_status wire_reserve(hccmf_t h, size_t halves) {  // send + recv staging, binary16
+  const size_t bytes = 2 * halves * 2;
+  if (h->wire_bytes >= bytes) return HCCMF_OK;
+  if (h->d_wire) cudaFreeAsync(h->d_wire, h->stream);
+  h->d_wire = nullptr;
+  h->wire_bytes = 0;
+  CU(h, cudaMallocAsync(&h->d_wire, bytes, h->stream));
+  h->wire_bytes = bytes;
+  return HCCMF_OK;
+}
+
+// one ring transfer of Q rows [sa, sb) to `prev` and [ra, rb) from `next`, fp32 or binary16
+hccmf_status ring_transfer(hccmf_t h, int64_t sa, int64_t sb, int64_t ra, int64_t rb, int prev, int next,
+                           cudaStream_t cs) {
+  const size_t ns = (size_t)(sb - sa) * h->k, nr = (size_t)(rb - ra) * h->k;
+  if (!h->opt_wire16) {
+    NC(h, ncclGroupStart());
+    if (ns) NC(h, ncclSend(h->d_Q + sa * h->k, ns, ncclFloat, prev, h->comm, cs));
+    if (nr) NC(h, ncclRecv(h->d_Q + ra * h->k, nr, ncclFloat, next, h->comm, cs));
+    NC(h, ncclGroupEnd());
+    return HCCMF_OK;
+  }
+  // Strategy 2: pack to binary16, ship half the bytes, unpack (all on the comm stream)
+  const size_t cap = (size_t)h->n * h->k;
+  hccmf_status st = wire_reserve(h, cap);
+  if (st != HCCMF_OK) return st;
+  CU(h, cudaStreamSynchronize(h->stream));  // staging allocation ordered before its use on cs
+  char* sendb = static_cast<char*>(h->d_wire);
+  char* recvb = sendb + cap * 2;
+  CU(h, k_pack_half(h->d_Q + sa * h->k, sendb, (int64_t)ns, cs));
+  NC(h, ncclGroupStart());
+  if (ns) NC(h, ncclSend(sendb, ns, ncclHalf, prev, h->comm, cs));
+  if (nr) NC(h, ncclRecv(recvb, nr, ncclHalf, next, h->comm, cs));
+  NC(h, ncclGroupEnd());
+  CU(h, k_unpack_half(recvb, h->d_Q + ra * h->k, (int64_t)nr, cs));
+  return HCCMF_OK;
+}
+
 hccmf_status ring_exchange(hccmf_t h, int sched, int t) {
   const int G = h->G, s = h->rank;
   const int g_send = (s + t) % G, g_recv = (s + t + 1) % G;
@@ -399,11 +437,7 @@ hccmf_status ring_exchange(hccmf_t h, int sched, int t) {
   ring_group_cols(h, sched, g_send, &sa, &sb);
   ring_group_cols(h, sched, g_recv, &ra, &rb);
   const int prev = (s - 1 + G) % G, next = (s + 1) % G;
-  NC(h, ncclGroupStart());
-  if (sb > sa) NC(h, ncclSend(h->d_Q + sa * h->k, (size_t)(sb - sa) * h->k, ncclFloat, prev, h->comm, h->stream));
-  if (rb > ra) NC(h, ncclRecv(h->d_Q + ra * h->k, (size_t)(rb - ra) * h->k, ncclFloat, next, h->comm, h->stream));
-  NC(h, ncclGroupEnd());
-  return HCCMF_OK;
+  return ring_transfer(h, sa, sb, ra, rb, prev, next, h->stream);
 }
 
 // Hidden synchronisation (L1143-L1172) with asynchronous computing-transmission
@@ -423,11 +457,7 @@ hccmf_status ring_exchange_block(hccmf_t h, int t, int j, cudaStream_t cs) {
   rows((s + t) % G, &sa, &sb);
   rows((s + t + 1) % G, &ra, &rb);
   const int prev = (s - 1 + G) % G, next = (s + 1) % G;
-  NC(h, ncclGroupStart());
-  if (sb > sa) NC(h, ncclSend(h->d_Q + sa * h->k, (size_t)(sb - sa) * h->k, ncclFloat, prev, h->comm, cs));
-  if (rb > ra) NC(h, ncclRecv(h->d_Q + ra * h->k, (size_t)(rb - ra) * h->k, ncclFloat, next, h->comm, cs));
-  NC(h, ncclGroupEnd());
-  return HCCMF_OK;
+  return ring_transfer(h, sa, sb, ra, rb, prev, next, cs);
 }
 
 // after ring epochs rank s holds only group s of Q: broadcast every group from its owner
@@ -533,6 +563,9 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
     case HCCMF_OPT_HOGWILD_ATOMIC:
       h->opt_atomic = value != 0;
       return HCCMF_OK;
+    case HCCMF_OPT_WIRE_FP16:
+      h->opt_wire16 = value != 0;
+      return HCCMF_OK;
     case HCCMF_OPT_SYNC_PHASES:
       if (value < 1) return fail(h, HCCMF_EINVAL, "sync phases must be >= 1");
       h->opt_phases = value;
@@ -566,6 +599,7 @@ void hccmf_destroy(hccmf_t h) {
   dfree(h, h->d_in_r, h->nnz);
   dfree(h, h->d_partials, 2 * RMSE_BLOCKS);
   dfree(h, h->d_scalar, 2);
+  if (h->d_wire) cudaFreeAsync(h->d_wire, h->stream);
   for (auto e : h->ev_done) cudaEventDestroy(e);
   for (auto e : h->ev_recv) cudaEventDestroy(e);
   if (h->comm_stream) {
@@ -882,12 +916,24 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     return HCCMF_OK;
   };
   auto average = [&]() -> hccmf_status {  // the server's sync (L549-L557): Q = mean of the shards' Q
-    if (dist)
+    if (dist && h->opt_wire16) {  // Strategy 2: the copies travel and come back as binary16
+      hccmf_status w = wire_reserve(h, (size_t)nk);
+      if (w != HCCMF_OK) return w;
+      CU(h, k_pack_half(h->d_Q, h->d_wire, nk, s));
+      NC(h, ncclAllReduce(h->d_wire, h->d_wire, (size_t)nk, ncclHalf, ncclAvg, h->comm, s));
+      CU(h, k_unpack_half(h->d_wire, h->d_Q, nk, s));
+    } else if (dist) {
       NC(h, ncclAllReduce(h->d_Q, h->d_Q, (size_t)nk, ncclFloat, ncclAvg, h->comm, s));
-    else
+    } else if (h->opt_wire16) {
+      CU(h, k_average_half(h->d_Qrep, nrep, nk, h->d_Q, s));
+    } else {
       CU(h, k_average(h->d_Qrep, nrep, nk, h->d_Q, s));
+    }
     return HCCMF_OK;
   };
+  // logical ring + Strategy 2: every column group moves once per stage, i.e. all of Q
+  // passes through binary16 at each stage boundary
+  const bool logical_wire = !dist && eff_sync == HCCMF_SYNC_RING && h->opt_wire16;
   if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && !dist) {
     st = replicate();
     if (st != HCCMF_OK) return st;
@@ -946,6 +992,8 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
         st = ring_exchange(h, sched, stage++);
         if (st != HCCMF_OK) return st;
       }
+    } else if (logical_wire) {
+      for (; stage < ln.stage; ++stage) CU(h, k_round_half(h->d_Q, nk, s));
     }
     a.Q = (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && !dist) ? h->d_Qrep + (size_t)ln.qrep * nk : h->d_Q;
     a.task_lo = pl->d_lo + ln.t0;
@@ -976,6 +1024,8 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     }
     h->q_ring_sched = sched;
   }
+  if (logical_wire)
+    for (; stage < pl->n_stages; ++stage) CU(h, k_round_half(h->d_Q, nk, s));
   if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG) {
     st = average();
     if (st != HCCMF_OK) return st;

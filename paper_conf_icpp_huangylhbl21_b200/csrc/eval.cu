@@ -1,4 +1,6 @@
 // eval.cu -- a0 factor init, a8 RMSE, a9 export (un-permute), Q replica average.
+#include <cuda_fp16.h>
+
 #include "internal.cuh"
 
 namespace hccmf {
@@ -133,7 +135,49 @@ __global__ void average_kernel(const float* reps, int32_t G, int64_t count, floa
   }
 }
 
+// Strategy 2 (L1234-L1249): Q on the wire as IEEE binary16 (round to nearest even).
+__global__ void round_half_kernel(float* x, int64_t count) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < count; e += (int64_t)gridDim.x * blockDim.x)
+    x[e] = __half2float(__float2half_rn(x[e]));
+}
+__global__ void pack_half_kernel(const float* x, __half* y, int64_t count) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < count; e += (int64_t)gridDim.x * blockDim.x)
+    y[e] = __float2half_rn(x[e]);
+}
+__global__ void unpack_half_kernel(const __half* y, float* x, int64_t count) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < count; e += (int64_t)gridDim.x * blockDim.x)
+    x[e] = __half2float(y[e]);
+}
+// replicas rounded to binary16, mean in fp64, mean rounded to binary16 (one rounding)
+__global__ void average_half_kernel(const float* reps, int32_t G, int64_t count, float* out) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < count; e += (int64_t)gridDim.x * blockDim.x) {
+    double s = 0.0;
+    for (int g = 0; g < G; ++g) s += (double)__half2float(__float2half_rn(reps[(int64_t)g * count + e]));
+    out[e] = __half2float(__double2half(s / (double)G));
+  }
+}
+
 }  // namespace
+
+cudaError_t k_round_half(float* x, int64_t count, cudaStream_t st) {
+  if (count <= 0) return cudaSuccess;
+  round_half_kernel<<<grid_for(count), kT, 0, st>>>(x, count);
+  return cudaGetLastError();
+}
+cudaError_t k_pack_half(const float* x, void* y, int64_t count, cudaStream_t st) {
+  if (count <= 0) return cudaSuccess;
+  pack_half_kernel<<<grid_for(count), kT, 0, st>>>(x, reinterpret_cast<__half*>(y), count);
+  return cudaGetLastError();
+}
+cudaError_t k_unpack_half(const void* y, float* x, int64_t count, cudaStream_t st) {
+  if (count <= 0) return cudaSuccess;
+  unpack_half_kernel<<<grid_for(count), kT, 0, st>>>(reinterpret_cast<const __half*>(y), x, count);
+  return cudaGetLastError();
+}
+cudaError_t k_average_half(const float* reps, int32_t G, int64_t count, float* out, cudaStream_t st) {
+  average_half_kernel<<<grid_for(count), kT, 0, st>>>(reps, G, count, out);
+  return cudaGetLastError();
+}
 
 cudaError_t k_init_factors(uint64_t seed, uint64_t tag, int64_t rows_total, int32_t k, const int32_t* perm,
                            int64_t row0, int64_t rows, float* X, cudaStream_t st) {

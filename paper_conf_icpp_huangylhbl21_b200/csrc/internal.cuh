@@ -113,6 +113,10 @@ cudaError_t k_rmse(const int32_t* tu, const int32_t* tv, const float* tr, int64_
                    const int32_t* perm_col, const float* P, int64_t row0, int64_t rows, const float* Q, int32_t k,
                    double* partials /*2*RMSE_BLOCKS*/, double* out2 /*sum, count*/, cudaStream_t st);
 cudaError_t k_average(const float* reps, int32_t G, int64_t count, float* out, cudaStream_t st);
+cudaError_t k_round_half(float* x, int64_t count, cudaStream_t st);
+cudaError_t k_pack_half(const float* x, void* y /* __half */, int64_t count, cudaStream_t st);
+cudaError_t k_unpack_half(const void* y /* __half */, float* x, int64_t count, cudaStream_t st);
+cudaError_t k_average_half(const float* reps, int32_t G, int64_t count, float* out, cudaStream_t st);
 constexpr int RMSE_BLOCKS = 592;
 
 }  // namespace hccmf
@@ -129,10 +133,12 @@ struct hccmf_ctx {
   ncclComm_t comm = nullptr;
   cudaStream_t comm_stream = nullptr;           // ring transfers overlapped with compute
   std::vector<cudaEvent_t> ev_done, ev_recv;    // per (stage, column block)
+  void* d_wire = nullptr;                       // binary16 staging (send | recv) for Strategy 2
+  size_t wire_bytes = 0;
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 3, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1;
+  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 3, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1, opt_wire16 = 0;
   bool sync_stream = true;
   size_t device_bytes = 0;
 

@@ -411,3 +411,46 @@ def test_distributed_handle_world1_matches_single(pkg, orc):
         assert np.array_equal(Pd, Ps) and np.array_equal(Qd, Qs) and rd == rs
     finally:
         dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("sync,G,Br,Bc", [("ring", 2, 4, 8), ("ring", 3, 3, 9), ("allreduce", 2, 4, 4)])
+def test_det_wire_fp16_logical_shards(pkg, orc, sync, G, Br, Bc):
+    # Strategy 2 (L1234-L1249, R25): Q crosses every shard boundary as binary16.
+    # Bar: the fp32-vs-fp64 1e-4 plus one binary16 rounding flip (2^-10 |x|) where the
+    # two sides' values straddle a binary16 rounding boundary.
+    cfg = synth.CONFIGS["c1"]
+    (u, v, r), _ = synth.make(cfg)
+    k, gamma = 16, 0.05
+    prob = orc.Problem(cfg.m, cfg.n, k, gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=Bc, seed=5)
+    prob.init(8)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    mdl = _gpu_problem(pkg, cfg.m, cfg.n, k, gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=Bc, seed=5)
+    mdl.set_option("wire_fp16", 1)
+    mdl.set_factors(P0, Q0)
+    for _ in range(2):
+        mdl.train_epoch("det", sync)
+        prob.epoch_wire16("det", sync)
+    P, Q = mdl.factors()
+    Po, Qo = prob.factors()
+    assert np.all(np.abs(Q - Qo) <= 1e-4 + 2.0 ** -10 * np.abs(Qo))
+    assert np.all(np.abs(P - Po) <= 1e-4 + 2.0 ** -10 * np.abs(Po))
+    # every Q value left the last transfer as a binary16 number
+    assert np.array_equal(Q.astype(np.float16).astype(np.float32), Q)
+
+
+def test_hogwild_ring_wire_fp16_band_c2(pkg, orc):
+    # the paper's claim that FP16 transmission does not cost accuracy, on C2 at 20 epochs
+    cfg = synth.CONFIGS["c2"]
+    (u, v, r), (tu, tv, tr) = synth.make(cfg)
+    G, Bc = 4, 8
+    prob = orc.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=G, Br=1, Bc=Bc, seed=cfg.seed)
+    prob.init(1)
+    mdl = _gpu_problem(pkg, cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=G, Br=1, Bc=Bc, seed=cfg.seed)
+    mdl.set_option("wire_fp16", 1)
+    mdl.init(1)
+    for _ in range(20):
+        prob.epoch_wire16("serial", "ring")
+        mdl.train_epoch("hogwild", "ring")
+    want, got = prob.rmse(tu, tv, tr), mdl.rmse(tu, tv, tr)
+    assert abs(got - want) <= 0.005, (want, got)

@@ -301,3 +301,47 @@ def test_phased_allreduce_pins(orc):
         Pg, Qg = _gd_step(u, v, r, 0.1, P0, Q0, gamma, gamma / G)
         gaps.append(max(np.abs(P1 - Pg).max(), np.abs(Q1 - Qg).max()))
     assert 0.2 < gaps[1] / gaps[0] < 0.3 and 0.2 < gaps[2] / gaps[1] < 0.3
+
+
+def test_round_half_matches_ieee_binary16(orc):
+    # Strategy 2 (L1234-L1249): the oracle's binary16 rounding against numpy's
+    # IEEE-754 half conversion (round to nearest even) on hand-picked and random values
+    cases = [0.0, -0.0, 1.0, 1 / 3, 0.1, 65504.0, 65519.0, 65520.0, 70000.0, 2.0 ** -24, 2.0 ** -25,
+             3 * 2.0 ** -26, 2.0 ** -14, 1 + 2.0 ** -11, 1 + 3 * 2.0 ** -11, -2.5e-5, 6.1e-5, 1e-8]
+    rng = np.random.default_rng(0)
+    cases += list(rng.normal(0, 1, 2000)) + list(rng.uniform(-1e-4, 1e-4, 500)) + list(rng.uniform(-7e4, 7e4, 500))
+    for x in cases:
+        with np.errstate(over="ignore"):
+            want = float(np.float16(x))
+        got = orc.round_half(x)
+        assert (got == want) or (np.isinf(got) and np.isinf(want) and np.sign(got) == np.sign(want)), (x, got, want)
+
+
+def test_wire16_epoch_pins(orc):
+    # with every Q value already a binary16 number and gamma -> 0 the wire is lossless:
+    # the wire16 epoch equals the fp64 epoch; with real updates it differs by at most
+    # one binary16 rounding per transfer (relative 2^-11 per stage)
+    import synth
+    m, n, k, G = 12, 10, 4, 2
+    u, v, r = synth.tiny(m, n, 70, seed=41)
+    rng = np.random.default_rng(3)
+    P0 = rng.uniform(0, 1, (m, k))
+    Q0 = np.array([[float(np.float16(x)) for x in row] for row in rng.uniform(0, 1, (n, k))])
+    for sync, Br, Bc in (("ring", 2, 4), ("allreduce", 2, 2)):
+        a = orc.Problem(m, n, k, 0.0, 0.0, u, v, r, G=G, Br=Br, Bc=Bc, seed=5)
+        b = orc.Problem(m, n, k, 0.0, 0.0, u, v, r, G=G, Br=Br, Bc=Bc, seed=5)
+        a.set_factors(P0, Q0)
+        b.set_factors(P0, Q0)
+        a.epoch("det", sync)
+        b.epoch_wire16("det", sync)
+        assert np.array_equal(a.Q, b.Q) and np.array_equal(a.P, b.P)
+        a = orc.Problem(m, n, k, 0.05, 0.01, u, v, r, G=G, Br=Br, Bc=Bc, seed=5)
+        b = orc.Problem(m, n, k, 0.05, 0.01, u, v, r, G=G, Br=Br, Bc=Bc, seed=5)
+        a.set_factors(P0, Q0)
+        b.set_factors(P0, Q0)
+        a.epoch("det", sync)
+        b.epoch_wire16("det", sync)
+        assert not np.array_equal(a.Q, b.Q)
+        assert np.abs(a.Q - b.Q).max() <= 4 * 2.0 ** -11 * np.abs(a.Q).max()
+        # every transmitted value is a binary16 number
+        assert all(float(np.float16(x)) == x for x in b.Q.ravel())
