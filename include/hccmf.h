@@ -163,12 +163,15 @@ typedef enum {
                                     on its Q copy, then averages Q: the paper's
                                     several pull-compute-push pipelines per epoch
                                     (L1251-L1269, Fig. 6; R22).         */
-    HCCMF_OPT_WIRE_FP16 = 11     /* 1: Q travels as IEEE binary16 (Strategy 2,
+    HCCMF_OPT_WIRE_FP16 = 11,    /* 1: Q travels as IEEE binary16 (Strategy 2,
                                     "Transmitting FP16 Data", L1234-L1249): ring
                                     transfers and the all-reduce pack to half and
                                     unpack to fp32; factors stay fp32 (R25).  The
                                     logical-shard backend applies the same rounding
                                     at every stage boundary.  Default 0.          */
+    HCCMF_OPT_L2_PERSIST = 12    /* 1: during a Hogwild epoch Q is an L2 persisting
+                                    access-policy window on the launch stream
+                                    (removed afterwards).  Default 0.             */
 } hccmf_option;
 
 /* ------------------------------------------------------------------ lifecycle */

@@ -563,6 +563,9 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
     case HCCMF_OPT_HOGWILD_ATOMIC:
       h->opt_atomic = value != 0;
       return HCCMF_OK;
+    case HCCMF_OPT_L2_PERSIST:
+      h->opt_l2persist = value != 0;
+      return HCCMF_OK;
     case HCCMF_OPT_WIRE_FP16:
       h->opt_wire16 = value != 0;
       return HCCMF_OK;
@@ -969,6 +972,28 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     CU(h, cudaEventRecord(h->ev_done[0], s));
     CU(h, cudaStreamWaitEvent(h->comm_stream, h->ev_done[0], 0));
   }
+  // Keep Q resident in L2 across the epoch: a persisting access-policy
+  // window over Q on the launch stream, so the 1.2 GB record stream and the P rows
+  // do not evict q_v lines between a group's load and its red.
+  const bool persist = h->opt_l2persist && sched == HCCMF_SCHED_HOGWILD;
+  if (persist) {
+    int max_win = 0, max_persist = 0;
+    cudaDeviceGetAttribute(&max_win, cudaDevAttrMaxAccessPolicyWindowSize, h->device);
+    cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, h->device);
+    const size_t qbytes = sizeof(float) * (size_t)nk;
+    const size_t win = std::min(qbytes, (size_t)std::max(0, max_win));
+    if (win > 0 && max_persist > 0) {
+      cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, std::min(win, (size_t)max_persist));
+      cudaStreamAttrValue v{};
+      v.accessPolicyWindow.base_ptr = h->d_Q;
+      v.accessPolicyWindow.num_bytes = win;
+      v.accessPolicyWindow.hitRatio = std::min(1.0f, (float)max_persist / (float)win);
+      v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+      v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+      cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v);
+    }
+    cudaGetLastError();
+  }
   int stage = 0;
   int phase = 0;
   for (size_t li = 0; li < pl->launches.size(); ++li) {
@@ -1023,6 +1048,12 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
       if (st != HCCMF_OK) return st;
     }
     h->q_ring_sched = sched;
+  }
+  if (persist) {  // drop the window again: the stream may be the caller's
+    cudaStreamAttrValue v{};
+    v.accessPolicyWindow.num_bytes = 0;
+    cudaStreamSetAttribute(s, cudaStreamAttributeAccessPolicyWindow, &v);
+    cudaGetLastError();
   }
   if (logical_wire)
     for (; stage < pl->n_stages; ++stage) CU(h, k_round_half(h->d_Q, nk, s));

@@ -138,7 +138,7 @@ struct hccmf_ctx {
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 3, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1, opt_wire16 = 0;
+  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 3, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1, opt_wire16 = 0, opt_l2persist = 0;
   bool sync_stream = true;
   size_t device_bytes = 0;
 

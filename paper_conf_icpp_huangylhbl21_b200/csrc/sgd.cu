@@ -408,7 +408,10 @@ struct WarpSgd {
 };
 
 template <int VEC, bool ATOMIC>
-__global__ void __launch_bounds__(kThreads) sgd_warp_kernel(SgdArgs a) {
+#ifndef HCCMF_WARP_MINB
+#define HCCMF_WARP_MINB 1
+#endif
+__global__ void __launch_bounds__(kThreads, HCCMF_WARP_MINB) sgd_warp_kernel(SgdArgs a) {
   constexpr unsigned FM = 0xffffffffu;
   WarpSgd<VEC, ATOMIC> w(a);
   unsigned long long tn = 0;

@@ -30,6 +30,7 @@ ap.add_argument("--vec", default="0")
 ap.add_argument("--repeat", type=int, default=1)
 ap.add_argument("--heavy", type=int, default=-1)
 ap.add_argument("--sched", default="hogwild")
+ap.add_argument("--persist", type=int, default=0)
 
 ap.add_argument("--every", action="store_true", help="test RMSE after every epoch")
 args = ap.parse_args()
@@ -43,6 +44,7 @@ mdl = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam)
 mdl.set_stream(st)
 mdl.set_option("task_ratings", args.task)
 mdl.set_option("heavy_first", args.heavy)
+mdl.set_option("l2_persist", args.persist)
 
 mdl.load(u, v, r)
 mdl.partition(1, (Br, Bc), seed=cfg.seed)
