@@ -569,6 +569,10 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
     case HCCMF_OPT_WIRE_FP16:
       h->opt_wire16 = value != 0;
       return HCCMF_OK;
+    case HCCMF_OPT_PREFETCH_DEPTH:
+      if (value < 1 || value > 4) return fail(h, HCCMF_EINVAL, "prefetch depth must be in [1, 4]");
+      h->opt_depth = value;
+      return HCCMF_OK;
     case HCCMF_OPT_SYNC_PHASES:
       if (value < 1) return fail(h, HCCMF_EINVAL, "sync phases must be >= 1");
       h->opt_phases = value;
@@ -954,6 +958,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   a.atomic_q = (sched == HCCMF_SCHED_HOGWILD && h->opt_atomic) ? 1 : 0;
   a.vec_pref = (int32_t)h->opt_vec;
   a.prefetch = sched == HCCMF_SCHED_DET ? 1 : 0;
+  a.depth = sched == HCCMF_SCHED_HOGWILD ? (int32_t)h->opt_depth : 1;
   const int L = sgd_lanes(h->k, (int)h->opt_vec);
   // a ring stage races only on its column group's items
   const int64_t hog_warps = auto_warps(h, eff_sync == HCCMF_SYNC_RING ? h->n / G : h->n);

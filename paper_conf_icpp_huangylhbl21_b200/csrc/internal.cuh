@@ -65,6 +65,7 @@ struct SgdArgs {
   int32_t atomic_q;  // Hogwild: apply q_v increments with vector atomics
   int32_t vec_pref;  // float4 slots per lane (0 = auto)
   int32_t prefetch;  // L2 bulk prefetch of the next window's p_u / q_v rows (DET blocks)
+  int32_t depth;     // q_v prefetch distance in ratings (warp-per-rating Hogwild kernel)
 };
 
 // launch the SGD kernel for a list of tasks; warps = concurrent warps wanted
@@ -138,7 +139,7 @@ struct hccmf_ctx {
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 3, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1, opt_wire16 = 0, opt_l2persist = 0;
+  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 3, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1, opt_wire16 = 0, opt_l2persist = 0, opt_depth = 1;
   bool sync_stream = true;
   size_t device_bytes = 0;
 

@@ -21,6 +21,10 @@
 //    q_{v(j+1)} == q_{v(j)} is forwarded from registers (serial read-after-write).
 //  * 32-bit row offsets and a compile-time full-vector geometry keep the per-rating
 //    instruction count low (profiles/).
+//  * the warp-per-rating Hogwild loop (k = 128 j) takes its records from a per-warp
+//    shared-memory ring filled by cp.async one window of 32 ahead (one broadcast
+//    LDS.128 per rating) and carries each row address from its prefetch to its red;
+//    an optional deeper q prefetch (D = 2..4) keeps D + 1 rows in flight.
 #include <algorithm>
 #include <type_traits>
 
@@ -294,6 +298,147 @@ struct WarpSgd {
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(qr), "r"(bytes) : "memory");
   }
 
+  // ---- Hogwild hot loop with a shared-memory record ring ----
+  // The warp's next 64 records sit in a per-warp ring of {u, v, r, -} entries filled by
+  // cp.async (4-byte copies, one window of 32 records per commit group, one window
+  // ahead), so the record of rating j+1 is ONE broadcast LDS.128 instead of three
+  // shuffles out of rotating register windows.  Row addresses are formed once with a
+  // 32x32->64 multiply-add and carried from the prefetch to the update and the red.
+  __device__ __forceinline__ const float4* qptr(int v) const {
+    return reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Qb) +
+                                           (unsigned long long)(unsigned)v * (unsigned)(k4 * 16));
+  }
+  __device__ __forceinline__ const float4* pptr(int u) const {
+    return reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Pb) +
+                                           (unsigned long long)(unsigned)u * (unsigned)(k4 * 16));
+  }
+  static __device__ __forceinline__ void cp4(const void* dst_smem, const void* src) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(d), "l"(src) : "memory");
+  }
+  // window w (records 32w .. 32w+31 of the task) -> ring half w & 1
+  __device__ __forceinline__ void stage(int4* ring, const int32_t* ru, const int32_t* rv, const float* rr, int w,
+                                        int left) const {
+    const int idx = w * 32 + lane;
+    if (idx < left) {
+      int4* e = ring + ((w & 1) << 5) + lane;
+      cp4(&e->x, ru + idx);
+      cp4(&e->y, rv + idx);
+      cp4(&e->z, rr + idx);
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  }
+  static __device__ __forceinline__ void wait_all() {
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
+    __syncwarp();
+  }
+
+  __device__ __forceinline__ void run_ring(int4* ring, int64_t lo, int left) {
+    const int32_t* ru = a.ru + lo;
+    const int32_t* rv = a.rv + lo;
+    const float* rr = a.rr + lo;
+    stage(ring, ru, rv, rr, 0, left);
+    wait_all();
+    stage(ring, ru, rv, rr, 1, left);  // one window in flight from here on
+    int4 rec = ring[0];
+    int cu = rec.x, cv = rec.y;
+    float cr = __int_as_float(rec.z);
+    const float4* pc = pptr(cu);
+    const float4* qc_p = qptr(cv);
+    float4 p[VEC], pn[VEC], qa[VEC], qb[VEC];
+    ld(pc, p);
+    ld(qc_p, qa);
+
+    // one step: update rating j (q in qc at qc_p), prefetch rating j+1 (q into qn)
+    auto step = [&](int j, float4 (&qc)[VEC], float4 (&qn)[VEC], auto has_next_tag, auto may_cross_tag) {
+      constexpr bool HAS_NEXT = decltype(has_next_tag)::value;
+      constexpr bool MAY_CROSS = decltype(may_cross_tag)::value;
+      int nu = 0, nv = 0;
+      float nr = 0.f;
+      bool fwd = false, newp = false;
+      const float4* qn_p = qc_p;
+      if (HAS_NEXT) {
+        const int jn = j + 1;
+        if (MAY_CROSS && (jn & 31) == 0) {  // entering window jn/32: it is complete; refill the other half
+          wait_all();
+          stage(ring, ru, rv, rr, (jn >> 5) + 1, left);
+        }
+        rec = ring[jn & 63];
+        nu = rec.x;
+        nv = rec.y;
+        nr = __int_as_float(rec.z);
+        fwd = nv == cv;
+        newp = nu != cu;
+        if (!fwd) {
+          qn_p = qptr(nv);
+          ld(qn_p, qn);
+        }
+        if (newp) ld(pptr(nu), pn);
+      }
+      float d0 = 0.f, d1 = 0.f, d2 = 0.f, d3 = 0.f;
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) {
+        d0 = fmaf(p[i].x, qc[i].x, d0);
+        d1 = fmaf(p[i].y, qc[i].y, d1);
+        d2 = fmaf(p[i].z, qc[i].z, d2);
+        d3 = fmaf(p[i].w, qc[i].w, d3);
+      }
+      float d = (d0 + d1) + (d2 + d3);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
+      const float ge = g * (cr - d);
+      float4 dq[VEC];
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) {
+        dq[i] = f4_fma(ge, p[i], f4_scale(ngl, qc[i]));
+        p[i] = f4_fma(ge, qc[i], f4_scale(c1, p[i]));
+      }
+      if (ATOMIC) {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i)
+          asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(qc_p + 32 * i),
+                       "f"(dq[i].x), "f"(dq[i].y), "f"(dq[i].z), "f"(dq[i].w)
+                       : "memory");
+      } else {
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) dq[i] = f4_add(qc[i], dq[i]);
+        st(qc_p, dq);
+      }
+      if (HAS_NEXT) {
+        if (fwd) {  // same item next (duplicates): serial read-after-write from registers
+#pragma unroll
+          for (int i = 0; i < VEC; ++i) qn[i] = ATOMIC ? f4_add(qc[i], dq[i]) : dq[i];
+        }
+        if (newp) {
+          st(pc, p);
+          pc = pptr(nu);
+#pragma unroll
+          for (int i = 0; i < VEC; ++i) p[i] = pn[i];
+        }
+        cu = nu;
+        cv = nv;
+        cr = nr;
+        qc_p = qn_p;
+      } else {
+        st(pc, p);
+      }
+    };
+    using T = std::true_type;
+    using F = std::false_type;
+    int j = 0;
+    for (; left - j >= 3; j += 2) {  // j even: only the odd step can enter a new window
+      step(j, qa, qb, T{}, F{});
+      step(j + 1, qb, qa, T{}, T{});
+    }
+    if (left - j == 2) {
+      step(j, qa, qb, T{}, F{});
+      step(j + 1, qb, qa, F{}, F{});
+    } else {
+      step(j, qa, qb, F{}, F{});
+    }
+    wait_all();  // no copy may still target the ring when the next task stages
+  }
+
   // all ratings of records [lo, lo + left), left >= 1, in order
   __device__ __forceinline__ void run(int64_t lo, int left) {
     auto ld = [&](const float4* r, float4 (&x)[VEC]) { this->ld(r, x); };
@@ -405,15 +550,126 @@ struct WarpSgd {
       step(j, qa, qb, F{});
     }
   }
+
+  // Deeper pipeline (D >= 2, Hogwild): the q row of rating j + D is requested while
+  // rating j is updated, from a ring of D + 1 register rows (the loop is unrolled
+  // D + 1 times so every slot index is static).  Every pending row whose load was
+  // issued before this warp's own update of the same item gets the increment added
+  // in registers, so one warp alone is exactly serial; p_u keeps the 1-deep prefetch
+  // (a user change is rare next to a rating).
+  template <int D>
+  __device__ __forceinline__ void run_deep(int64_t lo, int left) {
+    constexpr int R = D + 1;
+    const int32_t* ru = a.ru + lo;
+    const int32_t* rv = a.rv + lo;
+    const float* rr = a.rr + lo;
+    int wu0 = 0, wv0 = 0, wu1 = 0, wv1 = 0;
+    float wr0 = 0.f, wr1 = 0.f;
+    if (lane < left) wu0 = __ldcs(ru + lane), wv0 = __ldcs(rv + lane), wr0 = __ldcs(rr + lane);
+    if (lane + 32 < left) wu1 = __ldcs(ru + 32 + lane), wv1 = __ldcs(rv + 32 + lane), wr1 = __ldcs(rr + 32 + lane);
+    int wb = 0;
+    int su[R], sv[R];
+    float sr[R];
+    float4 q[R][VEC], p[VEC], pn[VEC];
+#pragma unroll
+    for (int s = 0; s < R; ++s) {
+      su[s] = sv[s] = 0;
+      sr[s] = 0.f;
+    }
+#pragma unroll
+    for (int s = 0; s < D; ++s) {
+      if (s < left) {
+        su[s] = __shfl_sync(FM, wu0, s);
+        sv[s] = __shfl_sync(FM, wv0, s);
+        sr[s] = __shfl_sync(FM, wr0, s);
+        ld(qrow(sv[s]), q[s]);
+      }
+    }
+    ld(prow(su[0]), p);
+    for (int j0 = 0; j0 < left; j0 += R) {
+#pragma unroll
+      for (int c = 0; c < R; ++c) {
+        const int j = j0 + c;
+        if (j >= left) break;
+        const int ns = (c + D) % R;  // slot of rating j + D
+        const int jn = j + D;
+        if (jn < left) {
+          if (jn - wb == 32) {  // slide the record window
+            wu0 = wu1, wv0 = wv1, wr0 = wr1;
+            wb += 32;
+            const int idx = wb + 32 + lane;
+            if (idx < left) wu1 = __ldcs(ru + idx), wv1 = __ldcs(rv + idx), wr1 = __ldcs(rr + idx);
+          }
+          const int src = jn - wb;
+          su[ns] = __shfl_sync(FM, wu0, src);
+          sv[ns] = __shfl_sync(FM, wv0, src);
+          sr[ns] = __shfl_sync(FM, wr0, src);
+          ld(qrow(sv[ns]), q[ns]);
+        }
+        const int cn = (c + 1) % R;
+        const bool has_next = j + 1 < left;
+        const bool newp = has_next && su[cn] != su[c];
+        if (newp) ld(prow(su[cn]), pn);
+        float d0 = 0.f, d1 = 0.f, d2 = 0.f, d3 = 0.f;
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) {
+          d0 = fmaf(p[i].x, q[c][i].x, d0);
+          d1 = fmaf(p[i].y, q[c][i].y, d1);
+          d2 = fmaf(p[i].z, q[c][i].z, d2);
+          d3 = fmaf(p[i].w, q[c][i].w, d3);
+        }
+        float d = (d0 + d1) + (d2 + d3);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
+        const float ge = g * (sr[c] - d);
+        float4 dq[VEC];
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) {
+          dq[i] = f4_fma(ge, p[i], f4_scale(ngl, q[c][i]));
+          p[i] = f4_fma(ge, q[c][i], f4_scale(c1, p[i]));
+        }
+        const float4* qw = qrow(sv[c]);
+        if (ATOMIC) {
+#pragma unroll
+          for (int i = 0; i < VEC; ++i)
+            asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(qw + 32 * i),
+                         "f"(dq[i].x), "f"(dq[i].y), "f"(dq[i].z), "f"(dq[i].w)
+                         : "memory");
+        } else {
+#pragma unroll
+          for (int i = 0; i < VEC; ++i) dq[i] = f4_add(q[c][i], dq[i]);
+          st(qw, dq);
+        }
+        // pending rows j+1 .. j+D were all requested before this update
+#pragma unroll
+        for (int t = 1; t <= D; ++t) {
+          const int s = (c + t) % R;
+          if (j + t < left && sv[s] == sv[c]) {
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) q[s][i] = ATOMIC ? f4_add(q[s][i], dq[i]) : dq[i];
+          }
+        }
+        if (!has_next || newp) {
+          st(prow(su[c]), p);
+          if (newp) {
+#pragma unroll
+            for (int i = 0; i < VEC; ++i) p[i] = pn[i];
+          }
+        }
+      }
+    }
+  }
 };
 
-template <int VEC, bool ATOMIC>
 #ifndef HCCMF_WARP_MINB
 #define HCCMF_WARP_MINB 1
 #endif
-__global__ void __launch_bounds__(kThreads, HCCMF_WARP_MINB) sgd_warp_kernel(SgdArgs a) {
+template <int VEC, bool ATOMIC, int D>
+__global__ void __launch_bounds__(kThreads, (VEC == 1 ? 4 : HCCMF_WARP_MINB)) sgd_warp_kernel(SgdArgs a) {
   constexpr unsigned FM = 0xffffffffu;
   WarpSgd<VEC, ATOMIC> w(a);
+  __shared__ int4 sring[kThreads / 32][64];
+  int4* ring = sring[threadIdx.x >> 5];
   unsigned long long tn = 0;
   if (w.lane == 0) tn = atomicAdd(a.counter, 1ull);
   tn = __shfl_sync(FM, tn, 0);
@@ -422,7 +678,10 @@ __global__ void __launch_bounds__(kThreads, HCCMF_WARP_MINB) sgd_warp_kernel(Sgd
     const int left = (int)(a.task_hi[tn] - lo);
     unsigned long long tn2 = 0;
     if (w.lane == 0) tn2 = atomicAdd(a.counter, 1ull);  // next task id, fetched one task ahead
-    w.run(lo, left);
+    if (D == 1)
+      w.run_ring(ring, lo, left);
+    else
+      w.template run_deep<D>(lo, left);
     tn = __shfl_sync(FM, tn2, 0);
   }
 }
@@ -473,11 +732,18 @@ cudaError_t launch_t(const SgdArgs& a, int64_t warps, cudaStream_t st) {
   const int threads = w < kThreads / 32 ? (int)w * 32 : kThreads;
   const int64_t blocks = (w * 32 + threads - 1) / threads;
   if (L == 32 && FULL) {  // warp-per-rating specialisation
-    if (a.atomic_q)
-      sgd_warp_kernel<VEC, true><<<(unsigned)blocks, threads, 0, st>>>(a);
-    else
-      sgd_warp_kernel<VEC, false><<<(unsigned)blocks, threads, 0, st>>>(a);
-    return cudaGetLastError();
+    const int depth = a.depth < 1 ? 1 : a.depth;
+#define WARP_CASE(DD)                                                   \
+  if (depth == DD) {                                                    \
+    if (a.atomic_q)                                                     \
+      sgd_warp_kernel<VEC, true, DD><<<(unsigned)blocks, threads, 0, st>>>(a);  \
+    else                                                                \
+      sgd_warp_kernel<VEC, false, DD><<<(unsigned)blocks, threads, 0, st>>>(a); \
+    return cudaGetLastError();                                          \
+  }
+    WARP_CASE(1) WARP_CASE(2) WARP_CASE(3) WARP_CASE(4)
+#undef WARP_CASE
+    return cudaErrorInvalidValue;
   }
   if (a.atomic_q)
     sgd_kernel<L, VEC, FULL, true><<<(unsigned)blocks, threads, 0, st>>>(a);

@@ -229,8 +229,9 @@ def test_det_logical_shards_parity(pkg, orc, sync, G, Br, Bc):
 
 # ------------------------------------------------------- a6 Hogwild
 @pytest.mark.parametrize("atomic", [0, 1])
-@pytest.mark.parametrize("k", [128, 256])
-def test_hogwild_single_group_is_the_serial_oracle(pkg, orc, atomic, k):
+@pytest.mark.parametrize("k,task,depth", [(128, 64, 1), (256, 64, 1), (128, 1000, 1), (128, 1000, 2),
+                                          (128, 100, 3), (128, 1000, 4)])
+def test_hogwild_single_group_is_the_serial_oracle(pkg, orc, atomic, k, task, depth):
     # One warp = one rating group (k >= 128) walks the tasks in record order: the
     # Hogwild kernel then IS the oracle's serial epoch (task builder, user runs,
     # p_u carry, q forwarding and same-thread red->load ordering all pinned).
@@ -241,7 +242,9 @@ def test_hogwild_single_group_is_the_serial_oracle(pkg, orc, atomic, k):
     P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
     prob.set_factors(P0, Q0)
     mdl = pkg.Model(cfg.m, cfg.n, k, 0.02, cfg.lam)
-    mdl.set_option("task_ratings", 64)
+    mdl.set_option("task_ratings", task)  # > 64: the record ring wraps inside a task
+    mdl.set_option("prefetch_depth", depth)
+    mdl.set_option("heavy_first", -1)  # record order = the oracle's serial order
     mdl.load(u, v, r)
     mdl.partition(1, (1, 1), seed=3)
     mdl.set_option("hogwild_warps", 1)

@@ -31,6 +31,7 @@ ap.add_argument("--repeat", type=int, default=1)
 ap.add_argument("--heavy", type=int, default=-1)
 ap.add_argument("--sched", default="hogwild")
 ap.add_argument("--persist", type=int, default=0)
+ap.add_argument("--depth", default="1")
 
 ap.add_argument("--every", action="store_true", help="test RMSE after every epoch")
 args = ap.parse_args()
@@ -49,9 +50,11 @@ mdl.set_option("l2_persist", args.persist)
 mdl.load(u, v, r)
 mdl.partition(1, (Br, Bc), seed=cfg.seed)
 dtu, dtv, dtr = (torch.from_numpy(x).cuda() for x in (tu, tv, tr))
-for at, vec, w in [(a_, v_, w_) for a_ in (int(x) for x in args.atomic.split(","))
-                   for v_ in (int(x) for x in args.vec.split(",")) for w_ in (int(x) for x in args.warps.split(",")) for _ in range(args.repeat)]:
+for at, vec, w, dp in [(a_, v_, w_, d_) for a_ in (int(x) for x in args.atomic.split(","))
+                       for v_ in (int(x) for x in args.vec.split(",")) for w_ in (int(x) for x in args.warps.split(","))
+                       for d_ in (int(x) for x in args.depth.split(",")) for _ in range(args.repeat)]:
     if True:
+        mdl.set_option("prefetch_depth", dp)
         mdl.set_option("vec", vec)
         mdl.set_option("hogwild_atomic", at)
         mdl.set_option("hogwild_warps", w)
@@ -68,5 +71,5 @@ for at, vec, w in [(a_, v_, w_) for a_ in (int(x) for x in args.atomic.split(","
                 rms.append(round(mdl.rmse(dtu, dtv, dtr), 5))
         rm = rms[-1]
         tmin = min(ts[1:] if len(ts) > 1 else ts)
-        print(json.dumps({"config": cfg.name, "atomic": at, "vec": vec, "warps": w, "epoch_ms": tmin,
+        print(json.dumps({"config": cfg.name, "depth": dp, "atomic": at, "vec": vec, "warps": w, "epoch_ms": tmin,
                           "gupd_s": cfg.nnz / tmin / 1e6, "test_rmse": rm, "per_epoch": rms}), flush=True)
