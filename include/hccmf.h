@@ -100,7 +100,13 @@ typedef struct {
     const double* t_meas; /* optional [G] measured compute time per shard, s       */
     double t_sync;        /* DP2: per-shard sync time, s                            */
     uint64_t seed;        /* a2 ID shuffle seed; 0 = identity permutation          */
-    int32_t storage;      /* 0 = fp32 factors (the only value accepted this round) */
+    int32_t storage;      /* 0 = fp32 factors; 1 = Q stored as IEEE binary16 while
+                             an epoch runs (fp32 arithmetic, P stays fp32): every
+                             q_v write keeps the nearest binary16 value (DESIGN.md
+                             R26).  Needs one rating per warp
+                             (k a multiple of 128): train_epoch returns EINVAL
+                             otherwise.  Q read back (rmse, get_factors) holds
+                             binary16 values.                                    */
     int32_t grid_dim;     /* 0 (default): row grid, shards of users, only Q moves;
                              1: column grid, shards of items, only P moves (Strategy 1
                              "transmitting P only", L1216-L1218); 2: the paper's rule

@@ -66,6 +66,7 @@ def lib():
             "orc_epoch_phased": (ctypes.c_int, [i32, i32, i32, i32, P, i64, i32, f64, f64, P, P, P, P, P]),
             "orc_round_half": (f64, [f64]),
             "orc_epoch_wire16": (ctypes.c_int, [i32, i32, i32, i32, i32, P, i64, i32, f64, f64, P, P, P, P, P]),
+            "orc_epoch_q16": (ctypes.c_int, [i32, i32, i32, i32, i32, P, i64, i32, f64, f64, P, P, P, P, P, i32]),
             "orc_cost_model": (i32, [i32, i64, i64, i64, i32, P, P, f64, i32, i32, i32, f64, P, P, P, P]),
         }
         for name, (res, args) in sig.items():
@@ -238,6 +239,16 @@ def epoch_wire16(sched, sync, G, Br, Bc, off, n, k, gamma, lam, ru, rv, rr, P, Q
         raise ValueError("oracle wire16 epoch: invalid grid or sync")
 
 
+def epoch_q16(sched, sync, G, Br, Bc, off, n, k, gamma, lam, ru, rv, rr, P, Q, add16=False):
+    """Epoch with Q stored in binary16 (every q_v write rounded; add16: the write is a
+    binary16 add of the rounded increment, as atomic Hogwild does; R26)."""
+    off = np.ascontiguousarray(off, dtype=np.int64)
+    rc = lib().orc_epoch_q16(SCHED[sched], SYNC[sync], G, Br, Bc, _p(off), n, P.shape[1], gamma, lam, _p(ru),
+                             _p(rv), _p(rr), _p(P), _p(Q), int(bool(add16)))
+    if rc != 0:
+        raise ValueError("oracle q16 epoch: invalid grid for this schedule")
+
+
 def rmse(tu, tv, tr, perm_row, perm_col, P, Q) -> float:
     tu, tv, tr = _i32(tu), _i32(tv), _f32(tr)
     return float(lib().orc_rmse(len(tu), _p(tu), _p(tv), _p(tr), P.shape[1], _p(_i32(perm_row)),
@@ -286,6 +297,10 @@ class Problem:
     def epoch(self, sched="det", sync="none"):
         epoch(sched, sync, self.G, self.Br, self.Bc, self.off, self.n, self.k, self.gamma, self.lam,
               self.ru, self.rv, self.rr, self.P, self.Q)
+
+    def epoch_q16(self, sched="det", sync="none", add16=False):
+        epoch_q16(sched, sync, self.G, self.Br, self.Bc, self.off, self.n, self.k, self.gamma, self.lam,
+                  self.ru, self.rv, self.rr, self.P, self.Q, add16)
 
     def epoch_wire16(self, sched="det", sync="ring"):
         epoch_wire16(sched, sync, self.G, self.Br, self.Bc, self.off, self.n, self.k, self.gamma, self.lam,

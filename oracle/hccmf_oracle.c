@@ -296,6 +296,17 @@ void orc_init(uint64_t seed, int64_t m, int64_t n, int32_t k, const int32_t* per
 /*   q' = q + gamma (e p - lambda q)      (p = value before this update)       */
 /* Returns e.                                                                  */
 /* ------------------------------------------------------------------------- */
+double orc_round_half(double x);
+
+/* Storage of Q (R26).  0: Q as computed (fp64 here).   */
+/* 1: Q is stored in IEEE binary16: every write of q_v keeps the binary16 value   */
+/* nearest to the update's result (orc_round_half), and an epoch starts from Q    */
+/* rounded to binary16.  2: as 1, but the write is a binary16 ADD of the          */
+/* increment: q <- rn16(q + rn16(gamma (e p - lambda q))) (Hogwild's component-   */
+/* wise atomic add on binary16 words).  P is never rounded.  Set per call by      */
+/* orc_epoch_q16.                                                                 */
+static int g_q16 = 0;
+
 double orc_sgd_update(int32_t k, double gamma, double lambda, double* p, double* q, double r)
 {
     double d = 0.0;
@@ -304,7 +315,12 @@ double orc_sgd_update(int32_t k, double gamma, double lambda, double* p, double*
     for (int32_t j = 0; j < k; ++j) {
         double pj = p[j], qj = q[j];
         p[j] = pj + gamma * (e * qj - lambda * pj);
-        q[j] = qj + gamma * (e * pj - lambda * qj);
+        if (g_q16 == 2)
+            q[j] = orc_round_half(qj + orc_round_half(gamma * (e * pj - lambda * qj)));
+        else if (g_q16 == 1)
+            q[j] = orc_round_half(qj + gamma * (e * pj - lambda * qj));
+        else
+            q[j] = qj + gamma * (e * pj - lambda * qj);
     }
     return e;
 }
@@ -591,4 +607,20 @@ int orc_epoch_wire16(int32_t sched, int32_t sync, int32_t G, int32_t Br, int32_t
         return 0;
     }
     return -1;
+}
+
+/* orc_epoch with Q stored in binary16 (storage = 1, R26): Q is rounded
+ * to binary16 first (the epoch starts from stored values), then every q_v write
+ * is rounded (orc_sgd_update; add16 = 1: as a binary16 add of the rounded
+ * increment).  Same schedules, grids and return codes. */
+int orc_epoch_q16(int32_t sched, int32_t sync, int32_t G, int32_t Br, int32_t Bc, const int64_t* off,
+                  int64_t n, int32_t k, double gamma, double lambda, const int32_t* ru, const int32_t* rv,
+                  const float* rr, double* P, double* Q, int32_t add16)
+{
+    size_t qn = (size_t)n * (size_t)k;
+    for (size_t i = 0; i < qn; ++i) Q[i] = orc_round_half(Q[i]);
+    g_q16 = add16 ? 2 : 1;
+    int rc = orc_epoch(sched, sync, G, Br, Bc, off, n, k, gamma, lambda, ru, rv, rr, P, Q);
+    g_q16 = 0;
+    return rc;
 }

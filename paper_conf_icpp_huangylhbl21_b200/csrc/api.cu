@@ -221,6 +221,7 @@ void free_partition(hccmf_t h) {
   dfree(h, h->d_P, h->rows * h->k);
   dfree(h, h->d_Q, h->n * h->k);
   dfree(h, h->d_Qrep, (size_t)h->n * h->k * (h->shard_hi - h->shard_lo));
+  dfree(h, h->d_Qh, (size_t)h->n * h->k);
   dfree(h, h->d_counters, h->n_counters);
   h->n_counters = 0;
   dfree(h, h->d_blk_off, h->nblk_local + 1);
@@ -666,7 +667,7 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   if (G < 1) return fail(h, HCCMF_EINVAL, "n_shards must be >= 1");
   if (h->world > 1 && G != h->world) return fail(h, HCCMF_EINVAL, "n_shards must equal the world size");
   if (o->grid_rows < 1 || o->grid_cols < 1) return fail(h, HCCMF_EINVAL, "grid must be >= 1 x 1");
-  if (o->storage != 0) return fail(h, HCCMF_EINVAL, "only fp32 storage (0) is implemented");
+  if (o->storage != 0 && o->storage != 1) return fail(h, HCCMF_EINVAL, "storage must be 0 (fp32) or 1 (binary16 Q)");
   if (o->strategy < HCCMF_DP0 || o->strategy > HCCMF_DP2) return fail(h, HCCMF_EINVAL, "bad strategy");
   if ((o->strategy != HCCMF_DP0) && !o->t_meas) return fail(h, HCCMF_EINVAL, "DP1/DP2 need t_meas");
   if (o->grid_dim < 0 || o->grid_dim > 2) return fail(h, HCCMF_EINVAL, "grid_dim must be 0, 1 or 2");
@@ -698,6 +699,7 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   h->Br = o->grid_rows;
   h->Bc = o->grid_cols;
   h->seed = o->seed;
+  h->storage = o->storage;
   const int64_t m = h->m, n = h->n, nnz = h->nnz;
   cudaStream_t st = h->stream;
 
@@ -886,7 +888,13 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   if (sched != HCCMF_SCHED_DET && sched != HCCMF_SCHED_HOGWILD) return fail(h, HCCMF_EINVAL, "bad schedule");
   if (sync < HCCMF_SYNC_NONE || sync > HCCMF_SYNC_ALLREDUCE_AVG) return fail(h, HCCMF_EINVAL, "bad sync");
   const int G = h->G;
-  if (sched == HCCMF_SCHED_DET && G == 1 && h->opt_wave && h->Br == h->Bc && h->Br > 1 &&
+  if (h->storage == 1) {  // binary16 Q lives in the warp-per-rating kernel (one rating per warp)
+    int L = 0, VEC = 0;
+    sgd_geometry(h->k, (int)h->opt_vec, &L, &VEC);
+    if (L != 32 || L * VEC * 4 != h->k)
+      return fail(h, HCCMF_EINVAL, "binary16 Q storage needs one rating per warp (k a multiple of 128, vec = k/128)");
+  }
+  if (sched == HCCMF_SCHED_DET && G == 1 && h->opt_wave && h->storage == 0 && h->Br == h->Bc && h->Br > 1 &&
       wave_supported(h->k, (int)h->opt_vec, h->Br)) {
     // DET as one wavefront kernel: same order of updates as the strata (R19)
     SgdArgs a{};
@@ -941,6 +949,30 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   // logical ring + Strategy 2: every column group moves once per stage, i.e. all of Q
   // passes through binary16 at each stage boundary
   const bool logical_wire = !dist && eff_sync == HCCMF_SYNC_RING && h->opt_wire16;
+  // Storage = 1 (R26): while launches run, the binary16 copy d_Qh of rows [qh_a, qh_b)
+  // of the fp32 matrix qh_of is the authoritative Q; it is rounded in before the first
+  // launch that needs it and written back (exactly: binary16 values are fp32 values)
+  // before anything else reads or moves Q (a ring transfer, an average, the next
+  // replica, the end of the epoch).
+  float* qh_of = nullptr;
+  int64_t qh_a = 0, qh_b = 0;
+  if (h->storage == 1 && !h->d_Qh) CU(h, dmalloc(h, &h->d_Qh, (size_t)nk));
+  auto qh_flush = [&]() -> hccmf_status {
+    if (qh_of && qh_b > qh_a)
+      CU(h, k_unpack_half(h->d_Qh + qh_a * h->k, qh_of + qh_a * h->k, (qh_b - qh_a) * h->k, s));
+    qh_of = nullptr;
+    return HCCMF_OK;
+  };
+  auto qh_enter = [&](float* q, int64_t a0, int64_t b0) -> hccmf_status {
+    if (qh_of == q && qh_a == a0 && qh_b == b0) return HCCMF_OK;
+    hccmf_status f = qh_flush();
+    if (f != HCCMF_OK) return f;
+    if (b0 > a0) CU(h, k_pack_half(q + a0 * h->k, h->d_Qh + a0 * h->k, (b0 - a0) * h->k, s));
+    qh_of = q;
+    qh_a = a0;
+    qh_b = b0;
+    return HCCMF_OK;
+  };
   if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && !dist) {
     st = replicate();
     if (st != HCCMF_OK) return st;
@@ -958,7 +990,8 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   a.atomic_q = (sched == HCCMF_SCHED_HOGWILD && h->opt_atomic) ? 1 : 0;
   a.vec_pref = (int32_t)h->opt_vec;
   a.prefetch = sched == HCCMF_SCHED_DET ? 1 : 0;
-  a.depth = sched == HCCMF_SCHED_HOGWILD ? (int32_t)h->opt_depth : 1;
+  a.depth = (sched == HCCMF_SCHED_HOGWILD && h->storage == 0) ? (int32_t)h->opt_depth : 1;
+  a.qhalf = h->storage == 1 ? 1 : 0;
   const int L = sgd_lanes(h->k, (int)h->opt_vec);
   // a ring stage races only on its column group's items
   const int64_t hog_warps = auto_warps(h, eff_sync == HCCMF_SYNC_RING ? h->n / G : h->n);
@@ -1004,6 +1037,8 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   for (size_t li = 0; li < pl->launches.size(); ++li) {
     const Launch& ln = pl->launches[li];
     if (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && ln.phase != phase) {  // sub-epoch sync (R22)
+      st = qh_flush();
+      if (st != HCCMF_OK) return st;
       st = average();
       if (st != HCCMF_OK) return st;
       if (!dist) {
@@ -1018,14 +1053,34 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
       jblk = (int)(li % (size_t)(h->Bc / G));
       if (ln.stage > 0) CU(h, cudaStreamWaitEvent(s, h->ev_recv[(size_t)(ln.stage - 1) * (h->Bc / G) + jblk], 0));
     } else if (dist && eff_sync == HCCMF_SYNC_RING) {
+      if (stage < ln.stage) {
+        st = qh_flush();
+        if (st != HCCMF_OK) return st;
+      }
       while (stage < ln.stage) {
         st = ring_exchange(h, sched, stage++);
         if (st != HCCMF_OK) return st;
       }
-    } else if (logical_wire) {
-      for (; stage < ln.stage; ++stage) CU(h, k_round_half(h->d_Q, nk, s));
+    } else if (logical_wire) {  // binary16 storage: Q is already binary16, the rounding is the identity
+      for (; stage < ln.stage; ++stage)
+        if (h->storage == 0) CU(h, k_round_half(h->d_Q, nk, s));
     }
     a.Q = (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && !dist) ? h->d_Qrep + (size_t)ln.qrep * nk : h->d_Q;
+    if (h->storage == 1) {
+      // rows this launch may touch: its column block (pipelined ring), its column group
+      // (stage-wise ring), else all of Q
+      int64_t ra = 0, rb = h->n;
+      if (pipelined) {
+        const int64_t cb = (int64_t)((h->rank + ln.stage) % G) * (h->Bc / G) + jblk;
+        ra = ceil_div(cb * h->n, h->Bc);
+        rb = ceil_div((cb + 1) * h->n, h->Bc);
+      } else if (dist && eff_sync == HCCMF_SYNC_RING) {
+        ring_group_cols(h, sched, (h->rank + ln.stage) % G, &ra, &rb);
+      }
+      st = qh_enter(a.Q, ra, rb);
+      if (st != HCCMF_OK) return st;
+      a.Q = reinterpret_cast<float*>(h->d_Qh);
+    }
     a.task_lo = pl->d_lo + ln.t0;
     a.task_hi = pl->d_hi + ln.t0;
     a.n_tasks = ln.nt;
@@ -1034,6 +1089,8 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     const int64_t warps = (sched == HCCMF_SCHED_DET) ? (ln.nt * L + 31) / 32 : hog_warps;
     CU(h, launch_sgd(a, warps, s));
     if (pipelined) {
+      st = qh_flush();  // the block travels as fp32 (or binary16 wire) right after its launch
+      if (st != HCCMF_OK) return st;
       const size_t e = (size_t)ln.stage * (h->Bc / G) + jblk;
       CU(h, cudaEventRecord(h->ev_done[e], s));
       CU(h, cudaStreamWaitEvent(h->comm_stream, h->ev_done[e], 0));
@@ -1042,6 +1099,8 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
       CU(h, cudaEventRecord(h->ev_recv[e], h->comm_stream));
     }
   }
+  st = qh_flush();
+  if (st != HCCMF_OK) return st;
   if (dist && eff_sync == HCCMF_SYNC_RING && sched == HCCMF_SCHED_HOGWILD) {
     // every transfer of the last stage lands before the epoch ends (shard s holds group s)
     const int c = h->Bc / G;

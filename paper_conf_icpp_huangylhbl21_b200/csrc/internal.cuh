@@ -66,6 +66,7 @@ struct SgdArgs {
   int32_t vec_pref;  // float4 slots per lane (0 = auto)
   int32_t prefetch;  // L2 bulk prefetch of the next window's p_u / q_v rows (DET blocks)
   int32_t depth;     // q_v prefetch distance in ratings (warp-per-rating Hogwild kernel)
+  int32_t qhalf;     // Q is IEEE binary16 (storage = 1; warp-per-rating kernel only)
 };
 
 // launch the SGD kernel for a list of tasks; warps = concurrent warps wanted
@@ -175,6 +176,8 @@ struct hccmf_ctx {
   float* d_P = nullptr;
   float* d_Q = nullptr;
   float* d_Qrep = nullptr;  // logical all-reduce replicas
+  int32_t storage = 0;      // 1: Q held in binary16 while an epoch runs (R26)
+  uint16_t* d_Qh = nullptr; // n x k binary16 copy of Q, authoritative inside an epoch (storage = 1)
   unsigned long long* d_counters = nullptr;
   int64_t n_counters = 0;
   double* d_partials = nullptr;

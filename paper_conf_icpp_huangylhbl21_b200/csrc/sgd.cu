@@ -25,6 +25,8 @@
 //    shared-memory ring filled by cp.async one window of 32 ahead (one broadcast
 //    LDS.128 per rating) and carries each row address from its prefetch to its red;
 //    an optional deeper q prefetch (D = 2..4) keeps D + 1 rows in flight.
+#include <cuda_fp16.h>
+
 #include <algorithm>
 #include <type_traits>
 
@@ -77,6 +79,16 @@ __device__ __forceinline__ float4 f4_scale(float s, float4 a) {
 }
 __device__ __forceinline__ float4 f4_add(float4 a, float4 b) {
   return make_float4(a.x + b.x, a.y + b.y, a.z + b.z, a.w + b.w);
+}
+// four binary16 (two half2 words) <-> float4, round to nearest even (storage = 1)
+__device__ __forceinline__ uint2 f4_to_h4(float4 a) {
+  const __half2 lo = __floats2half2_rn(a.x, a.y), hi = __floats2half2_rn(a.z, a.w);
+  return make_uint2(*reinterpret_cast<const unsigned*>(&lo), *reinterpret_cast<const unsigned*>(&hi));
+}
+__device__ __forceinline__ float4 h4_to_f4(uint2 r) {
+  const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&r.x));
+  const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&r.y));
+  return make_float4(lo.x, lo.y, hi.x, hi.y);
 }
 
 template <int L, int VEC, bool FULL, bool ATOMIC>
@@ -304,13 +316,55 @@ struct WarpSgd {
   // ahead), so the record of rating j+1 is ONE broadcast LDS.128 instead of three
   // shuffles out of rotating register windows.  Row addresses are formed once with a
   // 32x32->64 multiply-add and carried from the prefetch to the update and the red.
-  __device__ __forceinline__ const float4* qptr(int v) const {
-    return reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Qb) +
-                                           (unsigned long long)(unsigned)v * (unsigned)(k4 * 16));
+  // q_v row addresses as bytes: fp32 rows of k*4 bytes (lane slot i at +512 i), or
+  // binary16 rows of k*2 bytes (QH, storage = 1: lane holds 4 halves = 8 bytes per
+  // slot, slot i at +256 i).  The lane offset is folded into the base.
+  template <bool QH>
+  __device__ __forceinline__ const char* qaddr(int v) const {
+    const char* base = QH ? reinterpret_cast<const char*>(a.Q) + lane * 8 : reinterpret_cast<const char*>(Qb);
+    return base + (unsigned long long)(unsigned)v * (unsigned)(QH ? k4 * 8 : k4 * 16);
   }
   __device__ __forceinline__ const float4* pptr(int u) const {
     return reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Pb) +
                                            (unsigned long long)(unsigned)u * (unsigned)(k4 * 16));
+  }
+  template <bool QH>
+  __device__ __forceinline__ void ldq(const char* q, float4 (&x)[VEC]) const {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) {
+      if (QH)
+        x[i] = h4_to_f4(__ldcg(reinterpret_cast<const uint2*>(q + 256 * i)));
+      else
+        x[i] = __ldcg(reinterpret_cast<const float4*>(q + 512 * i));
+    }
+  }
+  template <bool QH>
+  __device__ __forceinline__ void stq(const char* q, const float4 (&x)[VEC]) const {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) {
+      if (QH)
+        __stcg(reinterpret_cast<uint2*>(const_cast<char*>(q) + 256 * i), f4_to_h4(x[i]));
+      else
+        __stcg(reinterpret_cast<float4*>(const_cast<char*>(q) + 512 * i), x[i]);
+    }
+  }
+  // Hogwild!'s component-wise atomic add: red.global.add.v4.f32 (fp32 rows) or
+  // red.global.add.noftz.v2.f16x2 of the increment rounded to binary16 (QH)
+  template <bool QH>
+  __device__ __forceinline__ void redq(const char* q, const float4 (&d)[VEC]) const {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) {
+      if (QH) {
+        const uint2 h = f4_to_h4(d[i]);
+        asm volatile("red.relaxed.gpu.global.add.noftz.v2.f16x2 [%0], {%1, %2};" ::"l"(q + 256 * i), "r"(h.x),
+                     "r"(h.y)
+                     : "memory");
+      } else {
+        asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(q + 512 * i), "f"(d[i].x),
+                     "f"(d[i].y), "f"(d[i].z), "f"(d[i].w)
+                     : "memory");
+      }
+    }
   }
   static __device__ __forceinline__ void cp4(const void* dst_smem, const void* src) {
     const unsigned d = (unsigned)__cvta_generic_to_shared(dst_smem);
@@ -333,6 +387,7 @@ struct WarpSgd {
     __syncwarp();
   }
 
+  template <bool QH>
   __device__ __forceinline__ void run_ring(int4* ring, int64_t lo, int left) {
     const int32_t* ru = a.ru + lo;
     const int32_t* rv = a.rv + lo;
@@ -344,10 +399,10 @@ struct WarpSgd {
     int cu = rec.x, cv = rec.y;
     float cr = __int_as_float(rec.z);
     const float4* pc = pptr(cu);
-    const float4* qc_p = qptr(cv);
+    const char* qc_p = qaddr<QH>(cv);
     float4 p[VEC], pn[VEC], qa[VEC], qb[VEC];
     ld(pc, p);
-    ld(qc_p, qa);
+    ldq<QH>(qc_p, qa);
 
     // one step: update rating j (q in qc at qc_p), prefetch rating j+1 (q into qn)
     auto step = [&](int j, float4 (&qc)[VEC], float4 (&qn)[VEC], auto has_next_tag, auto may_cross_tag) {
@@ -356,7 +411,7 @@ struct WarpSgd {
       int nu = 0, nv = 0;
       float nr = 0.f;
       bool fwd = false, newp = false;
-      const float4* qn_p = qc_p;
+      const char* qn_p = qc_p;
       if (HAS_NEXT) {
         const int jn = j + 1;
         if (MAY_CROSS && (jn & 31) == 0) {  // entering window jn/32: it is complete; refill the other half
@@ -370,8 +425,8 @@ struct WarpSgd {
         fwd = nv == cv;
         newp = nu != cu;
         if (!fwd) {
-          qn_p = qptr(nv);
-          ld(qn_p, qn);
+          qn_p = qaddr<QH>(nv);
+          ldq<QH>(qn_p, qn);
         }
         if (newp) ld(pptr(nu), pn);
       }
@@ -394,20 +449,21 @@ struct WarpSgd {
         p[i] = f4_fma(ge, qc[i], f4_scale(c1, p[i]));
       }
       if (ATOMIC) {
-#pragma unroll
-        for (int i = 0; i < VEC; ++i)
-          asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(qc_p + 32 * i),
-                       "f"(dq[i].x), "f"(dq[i].y), "f"(dq[i].z), "f"(dq[i].w)
-                       : "memory");
+        redq<QH>(qc_p, dq);
       } else {
 #pragma unroll
         for (int i = 0; i < VEC; ++i) dq[i] = f4_add(qc[i], dq[i]);
-        st(qc_p, dq);
+        stq<QH>(qc_p, dq);
       }
       if (HAS_NEXT) {
         if (fwd) {  // same item next (duplicates): serial read-after-write from registers
 #pragma unroll
-          for (int i = 0; i < VEC; ++i) qn[i] = ATOMIC ? f4_add(qc[i], dq[i]) : dq[i];
+          for (int i = 0; i < VEC; ++i) {
+            if (QH)  // what memory now holds: rn16(q + rn16(dq)) (atomic) or rn16(q + dq) (store)
+              qn[i] = h4_to_f4(f4_to_h4(ATOMIC ? f4_add(qc[i], h4_to_f4(f4_to_h4(dq[i]))) : dq[i]));
+            else
+              qn[i] = ATOMIC ? f4_add(qc[i], dq[i]) : dq[i];
+          }
         }
         if (newp) {
           st(pc, p);
@@ -664,7 +720,7 @@ struct WarpSgd {
 #ifndef HCCMF_WARP_MINB
 #define HCCMF_WARP_MINB 1
 #endif
-template <int VEC, bool ATOMIC, int D>
+template <int VEC, bool ATOMIC, int D, bool QH>
 __global__ void __launch_bounds__(kThreads, (VEC == 1 ? 4 : HCCMF_WARP_MINB)) sgd_warp_kernel(SgdArgs a) {
   constexpr unsigned FM = 0xffffffffu;
   WarpSgd<VEC, ATOMIC> w(a);
@@ -678,8 +734,10 @@ __global__ void __launch_bounds__(kThreads, (VEC == 1 ? 4 : HCCMF_WARP_MINB)) sg
     const int left = (int)(a.task_hi[tn] - lo);
     unsigned long long tn2 = 0;
     if (w.lane == 0) tn2 = atomicAdd(a.counter, 1ull);  // next task id, fetched one task ahead
-    if (D == 1)
-      w.run_ring(ring, lo, left);
+    if (D == 1 && QH)
+      w.template run_ring<true>(ring, lo, left);
+    else if (D == 1)
+      w.template run_ring<false>(ring, lo, left);
     else
       w.template run_deep<D>(lo, left);
     tn = __shfl_sync(FM, tn2, 0);
@@ -733,18 +791,19 @@ cudaError_t launch_t(const SgdArgs& a, int64_t warps, cudaStream_t st) {
   const int64_t blocks = (w * 32 + threads - 1) / threads;
   if (L == 32 && FULL) {  // warp-per-rating specialisation
     const int depth = a.depth < 1 ? 1 : a.depth;
-#define WARP_CASE(DD)                                                   \
-  if (depth == DD) {                                                    \
-    if (a.atomic_q)                                                     \
-      sgd_warp_kernel<VEC, true, DD><<<(unsigned)blocks, threads, 0, st>>>(a);  \
-    else                                                                \
-      sgd_warp_kernel<VEC, false, DD><<<(unsigned)blocks, threads, 0, st>>>(a); \
-    return cudaGetLastError();                                          \
+#define WARP_CASE(DD, QQ)                                                     \
+  if (depth == DD && (a.qhalf != 0) == QQ) {                                  \
+    if (a.atomic_q)                                                           \
+      sgd_warp_kernel<VEC, true, DD, QQ><<<(unsigned)blocks, threads, 0, st>>>(a);  \
+    else                                                                      \
+      sgd_warp_kernel<VEC, false, DD, QQ><<<(unsigned)blocks, threads, 0, st>>>(a); \
+    return cudaGetLastError();                                                \
   }
-    WARP_CASE(1) WARP_CASE(2) WARP_CASE(3) WARP_CASE(4)
+    WARP_CASE(1, false) WARP_CASE(2, false) WARP_CASE(3, false) WARP_CASE(4, false) WARP_CASE(1, true)
 #undef WARP_CASE
     return cudaErrorInvalidValue;
   }
+  if (a.qhalf) return cudaErrorInvalidValue;  // binary16 Q: warp-per-rating geometry only
   if (a.atomic_q)
     sgd_kernel<L, VEC, FULL, true><<<(unsigned)blocks, threads, 0, st>>>(a);
   else

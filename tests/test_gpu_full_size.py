@@ -65,22 +65,24 @@ def test_c3_partition_bitexact_full_size(pkg, c3, B):
     assert _digest(mdl) == ref[key]
 
 
-@pytest.mark.parametrize("name,data", [("c3", "c3"), ("c2", None)])
-def test_hogwild_band_full_size(pkg, c3, name, data):
-    # bench.py's configuration: one shard, grid (1, 1), library defaults, init seed 1
+@pytest.mark.parametrize("name,data,storage", [("c3", "c3", "fp32"), ("c2", None, "fp32"), ("c3", "c3", "fp16")])
+def test_hogwild_band_full_size(pkg, c3, name, data, storage):
+    # bench.py's configuration: one shard, grid (1, 1), library defaults, init seed 1.
+    # storage fp16 (Q in binary16, R26) is held to the same band against the fp64 oracle.
     ref = _ref(name)
     cfg = synth.CONFIGS[name]
     (u, v, r), (tu, tv, tr) = c3 if data == "c3" else synth.make(cfg)
     mdl = pkg.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam)
     mdl.load(u, v, r)
-    mdl.partition(1, (1, 1), seed=cfg.seed)
+    mdl.partition(1, (1, 1), seed=cfg.seed, storage=storage)
     mdl.init(1)
     curve = [mdl.rmse(tu, tv, tr)]
     E = ref["epochs"]
     for _ in range(E):
         mdl.train_epoch("hogwild", "none")
         curve.append(mdl.rmse(tu, tv, tr))
-    assert curve[0] == pytest.approx(ref["test_rmse"][0], rel=1e-6)  # same init, same data
+    if storage == "fp32":
+        assert curve[0] == pytest.approx(ref["test_rmse"][0], rel=1e-6)  # same init, same data
     assert abs(curve[E] - ref["test_rmse"][E]) <= 0.005, (curve, ref["test_rmse"])
 
 

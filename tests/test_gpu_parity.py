@@ -457,3 +457,100 @@ def test_hogwild_ring_wire_fp16_band_c2(pkg, orc):
         mdl.train_epoch("hogwild", "ring")
     want, got = prob.rmse(tu, tv, tr), mdl.rmse(tu, tv, tr)
     assert abs(got - want) <= 0.005, (want, got)
+
+
+# ---------------------------------------- binary16 storage of Q (f1, R26)
+# Bar: 1e-4 + 2^-9 |x| (two binary16 ulps).  Both sides round every q_v write to
+# binary16, but the CUDA kernel rounds its fp32 result while the oracle rounds its
+# fp64 result; where the two straddle a rounding boundary the stored q differs by
+# one binary16 ulp (2^-10 |x| at most), and that difference is carried, contracted,
+# into later updates of the same item and its users.
+def _q16_bar(x):
+    return 1e-4 + np.abs(x) * 2.0 ** -9
+
+
+@pytest.mark.parametrize("k,B,epochs", [(128, 8, 1), (128, 8, 3), (256, 4, 1)])
+def test_det_epoch_parity_q16(pkg, orc, k, B, epochs):
+    cfg = synth.CONFIGS["c1"]
+    (u, v, r), (tu, tv, tr) = synth.make(cfg)
+    gamma = 0.02
+    prob = orc.Problem(cfg.m, cfg.n, k, gamma, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=11)
+    prob.init(2)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    mdl = pkg.Model(cfg.m, cfg.n, k, gamma, cfg.lam)
+    mdl.load(u, v, r)
+    mdl.partition(1, (B, B), seed=11, storage="fp16")
+    mdl.set_factors(P0, Q0)
+    for _ in range(epochs):
+        mdl.train_epoch("det", "none")
+        prob.epoch_q16("det", "none")
+    P, Q = mdl.factors()
+    Po, Qo = prob.factors()
+    assert np.array_equal(Q.astype(np.float16).astype(np.float32), Q)  # Q holds binary16 values
+    assert np.all(np.abs(P - Po) <= _q16_bar(Po)), np.abs(P - Po).max()
+    assert np.all(np.abs(Q - Qo) <= _q16_bar(Qo)), np.abs(Q - Qo).max()
+    assert mdl.rmse(tu, tv, tr) == pytest.approx(prob.rmse(tu, tv, tr), abs=1e-4)
+
+
+@pytest.mark.parametrize("atomic", [0, 1])
+def test_hogwild_single_group_q16(pkg, orc, atomic):
+    # one warp walks the tasks in record order: the binary16 Hogwild kernel is then the
+    # oracle's serial epoch with binary16 Q (atomic: the increment is itself rounded
+    # to binary16 before the add, one more rounding than the oracle's)
+    cfg = synth.CONFIGS["c1"]
+    (u, v, r), _ = synth.make(cfg)
+    k = 128
+    prob = orc.Problem(cfg.m, cfg.n, k, 0.02, cfg.lam, u, v, r, G=1, Br=1, Bc=1, seed=3)
+    prob.init(4)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    mdl = pkg.Model(cfg.m, cfg.n, k, 0.02, cfg.lam)
+    mdl.set_option("task_ratings", 300)
+    mdl.set_option("heavy_first", -1)
+    mdl.load(u, v, r)
+    mdl.partition(1, (1, 1), seed=3, storage="fp16")
+    mdl.set_option("hogwild_warps", 1)
+    mdl.set_option("hogwild_atomic", atomic)
+    mdl.set_factors(P0, Q0)
+    for _ in range(2):
+        mdl.train_epoch("hogwild", "none")
+        prob.epoch_q16("serial", "none", add16=bool(atomic))
+    P, Q = mdl.factors()
+    Po, Qo = prob.factors()
+    assert np.all(np.abs(P - Po) <= _q16_bar(Po)), np.abs(P - Po).max()
+    assert np.all(np.abs(Q - Qo) <= _q16_bar(Qo)), np.abs(Q - Qo).max()
+
+
+@pytest.mark.parametrize("sync,G,Br,Bc", [("ring", 2, 4, 8), ("allreduce", 2, 4, 4)])
+def test_det_logical_shards_parity_q16(pkg, orc, sync, G, Br, Bc):
+    cfg = synth.CONFIGS["c1"]
+    (u, v, r), _ = synth.make(cfg)
+    k, gamma = 128, 0.02
+    prob = orc.Problem(cfg.m, cfg.n, k, gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=Bc, seed=5)
+    prob.init(8)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    mdl = pkg.Model(cfg.m, cfg.n, k, gamma, cfg.lam)
+    mdl.load(u, v, r)
+    mdl.partition(G, (Br, Bc), seed=5, storage="fp16")
+    mdl.set_factors(P0, Q0)
+    for _ in range(2):
+        mdl.train_epoch("det", sync)
+        prob.epoch_q16("det", sync)
+    P, Q = mdl.factors()
+    Po, Qo = prob.factors()
+    assert np.all(np.abs(P - Po) <= _q16_bar(Po)), np.abs(P - Po).max()
+    assert np.all(np.abs(Q - Qo) <= _q16_bar(Qo)), np.abs(Q - Qo).max()
+
+
+def test_q16_storage_rejects_unsupported_geometry(pkg):
+    cfg = synth.CONFIGS["c1"]
+    (u, v, r), _ = synth.make(cfg)
+    mdl = pkg.Model(cfg.m, cfg.n, 16, cfg.gamma, cfg.lam)
+    mdl.load(u, v, r)
+    mdl.partition(1, (1, 1), seed=1, storage="fp16")
+    mdl.init(1)
+    with pytest.raises(pkg.HccmfError) as ei:
+        mdl.train_epoch("hogwild", "none")
+    assert ei.value.code == pkg.EINVAL

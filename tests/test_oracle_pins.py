@@ -345,3 +345,68 @@ def test_wire16_epoch_pins(orc):
         assert np.abs(a.Q - b.Q).max() <= 4 * 2.0 ** -11 * np.abs(a.Q).max()
         # every transmitted value is a binary16 number
         assert all(float(np.float16(x)) == x for x in b.Q.ravel())
+
+
+def test_q16_storage_single_update_hand_computed(orc):
+    # Binary16 storage of Q (R26): Q is rounded first, every q write is
+    # rounded, P never.  Fig. 1 rating (0, 0, 5.0), p = (2.37, 0), q = (2.09, 0.69),
+    # lambda = 0.01.  By hand: rn16(2.09) = 1070 * 2^-9 = 2.08984375,
+    # rn16(0.69) = 1413 * 2^-11 = 0.68994140625;  e = 5 - 2.37 * 2.08984375 = 0.0470703125.
+    #  gamma = 0.005: q0 = 2.08984375 + 0.005*(0.0470703125*2.37 - 0.0208984375)
+    #                    = 2.090297041015625 -> 1070.23 ulps -> 2.08984375 (the step is lost)
+    #                 q1 = 0.68994140625 - 0.005*0.0068994140625 = 0.68990690917...
+    #                    -> 1412.93 ulps -> 0.68994140625 (lost too: SURVEY H6)
+    #                 p0 = 2.37 + 0.005*(0.0470703125*2.08984375 - 0.0237) = 2.370373347991943...
+    #                 p1 = 0.005*0.0470703125*0.68994140625 = 0.000162378787994384765625
+    #  gamma = 0.1:   q0 = 2.08984375 + 0.0090658203125 = 2.0989095703125 -> 1074.64 -> 2.099609375
+    #                 q1 = 0.68994140625 - 0.00068994140625 = 0.68925146484375 -> 1411.59 -> 0.689453125
+    u, v, r = np.array([0], np.int32), np.array([0], np.int32), np.array([5.0], np.float32)
+    for gamma, want_p, want_q in ((0.005, [2.370373347991943, 0.000162378787994384765625],
+                                   [2.08984375, 0.68994140625]),
+                                  (0.1, [2.37 + 0.1 * 0.074669598388671875, 0.1 * 0.032475757598876953125],
+                                   [2.099609375, 0.689453125])):
+        prob = orc.Problem(1, 1, 2, gamma, 0.01, u, v, r, seed=0)
+        prob.set_factors(np.array([[2.37, 0.0]]), np.array([[2.09, 0.69]]))
+        prob.epoch_q16("serial", "none")
+        P, Q = prob.factors()
+        assert list(Q[0]) == want_q  # exact: binary16 values
+        assert P[0] == pytest.approx(want_p, abs=1e-15)
+    # add16 (binary16 add of the rounded increment): gamma = 0.1, increments by hand
+    # 0.0090658203125 -> rn16 = 1188.3 * 2^-17 -> 1188 * 2^-17 = 0.0090637207..., and
+    # -0.00068994140625 -> -1446.9 * 2^-21 -> -1447 * 2^-21 = -0.000689983367919921875;
+    # q0 = rn16(2.08984375 + 0.009063720703125) = rn16(2.098907470703125) = 1074.64 -> 2.099609375
+    # q1 = rn16(0.68994140625 - 0.000689983367919921875) = 1411.59 ulps -> 0.689453125
+    # (same stored values here: the rounded increment moves each sum by < 0.01 ulp)
+    prob = orc.Problem(1, 1, 2, 0.1, 0.01, u, v, r, seed=0)
+    prob.set_factors(np.array([[2.37, 0.0]]), np.array([[2.09, 0.69]]))
+    prob.epoch_q16("serial", "none", add16=True)
+    assert list(prob.factors()[1][0]) == [2.099609375, 0.689453125]
+    assert float(np.float16(0.0090658203125)) == 1188 * 2.0 ** -17
+    assert float(np.float16(-0.00068994140625)) == -1447 * 2.0 ** -21
+
+
+def test_q16_storage_epoch_invariants(orc):
+    # every stored q is a binary16 number, P is not rounded, and the binary16 epoch stays
+    # within a few binary16 ulps of the fp64 epoch on a small problem
+    import synth
+    m, n, k = 30, 20, 8
+    u, v, r = synth.tiny(m, n, 300, seed=7)
+    rng = np.random.default_rng(5)
+    P0, Q0 = rng.uniform(0, 1, (m, k)), rng.uniform(0, 1, (n, k))
+    for sched, sync, G, Br, Bc in (("det", "none", 1, 3, 3), ("serial", "none", 1, 1, 1),
+                                    ("det", "ring", 2, 2, 4), ("det", "allreduce", 2, 3, 3)):
+        a = orc.Problem(m, n, k, 0.01, 0.05, u, v, r, G=G, Br=Br, Bc=Bc, seed=9)
+        b = orc.Problem(m, n, k, 0.01, 0.05, u, v, r, G=G, Br=Br, Bc=Bc, seed=9)
+        a.set_factors(P0, Q0)
+        b.set_factors(P0, Q0)
+        a.epoch(sched, sync)
+        b.epoch_q16(sched, sync)
+        if sync != "allreduce":  # the mean of binary16 copies is not itself rounded
+            assert all(float(np.float16(x)) == x for x in b.Q.ravel())
+        assert not all(float(np.float16(x)) == x for x in b.P.ravel())
+        assert 0 < np.abs(a.Q - b.Q).max() <= 8 * 2.0 ** -11 * np.abs(a.Q).max()
+        assert np.abs(a.P - b.P).max() <= 8 * 2.0 ** -11 * np.abs(a.P).max()
+        c = orc.Problem(m, n, k, 0.01, 0.05, u, v, r, G=G, Br=Br, Bc=Bc, seed=9)
+        c.set_factors(P0, Q0)
+        c.epoch_q16(sched, sync, add16=True)
+        assert 0 < np.abs(b.Q - c.Q).max() <= 8 * 2.0 ** -11 * np.abs(b.Q).max()

@@ -32,6 +32,7 @@ ap.add_argument("--heavy", type=int, default=-1)
 ap.add_argument("--sched", default="hogwild")
 ap.add_argument("--persist", type=int, default=0)
 ap.add_argument("--depth", default="1")
+ap.add_argument("--storage", default="fp32")
 
 ap.add_argument("--every", action="store_true", help="test RMSE after every epoch")
 args = ap.parse_args()
@@ -48,7 +49,7 @@ mdl.set_option("heavy_first", args.heavy)
 mdl.set_option("l2_persist", args.persist)
 
 mdl.load(u, v, r)
-mdl.partition(1, (Br, Bc), seed=cfg.seed)
+mdl.partition(1, (Br, Bc), seed=cfg.seed, storage=args.storage)
 dtu, dtv, dtr = (torch.from_numpy(x).cuda() for x in (tu, tv, tr))
 for at, vec, w, dp in [(a_, v_, w_, d_) for a_ in (int(x) for x in args.atomic.split(","))
                        for v_ in (int(x) for x in args.vec.split(",")) for w_ in (int(x) for x in args.warps.split(","))
@@ -71,5 +72,5 @@ for at, vec, w, dp in [(a_, v_, w_, d_) for a_ in (int(x) for x in args.atomic.s
                 rms.append(round(mdl.rmse(dtu, dtv, dtr), 5))
         rm = rms[-1]
         tmin = min(ts[1:] if len(ts) > 1 else ts)
-        print(json.dumps({"config": cfg.name, "depth": dp, "atomic": at, "vec": vec, "warps": w, "epoch_ms": tmin,
+        print(json.dumps({"config": cfg.name, "storage": args.storage, "depth": dp, "atomic": at, "vec": vec, "warps": w, "epoch_ms": tmin,
                           "gupd_s": cfg.nnz / tmin / 1e6, "test_rmse": rm, "per_epoch": rms}), flush=True)
