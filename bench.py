@@ -54,6 +54,10 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--storage", default="fp32", choices=["fp32", "fp16"],
+                    help="Q storage of the headline number (fp16 = binary16 Q, fp32 math, R26)")
+    ap.add_argument("--no-fp16-leg", action="store_true",
+                    help="skip the secondary binary16-Q measurement added to the JSON line")
     return ap.parse_args()
 
 
@@ -272,59 +276,67 @@ def main():
     if on_device:  # keep a host-free copy only where it fits; free the generator's 37 GB first
         del du, dv, dr
         torch.cuda.empty_cache()
-    mdl.partition(G, (Br, Bc), "DP0", seed=cfg.seed)
+    mdl.partition(G, (Br, Bc), "DP0", seed=cfg.seed, storage=args.storage)
     mdl.init(1)
     t_prep = time.perf_counter() - t_prep
     info = mdl.info()
     if not on_device:
         del du, dv, dr
-    rm0 = mdl.rmse(dtu, dtv, dtr)
-    mdl.set_option("sync_stream", 0)
-
-    def step(ev=None):
-        if ev is not None:
-            ev[0].record(stream)
-        mdl.train_epoch(args.sched, sync)
-        if ev is not None:
-            ev[1].record(stream)
-        return mdl.rmse(dtu, dtv, dtr)
-
-    curve = [rm0] + [step() for _ in range(args.warmup)]
-    kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    clocks = Clocks(local)
-    clocks.start()
-    time.sleep(0.3)
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    t_start.record(stream)
-    rms = [step(kev[i]) for i in range(args.steps)]
-    t_end.record(stream)
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
-    clk = clocks.stop()
-    ms = t_start.elapsed_time(t_end)
-    k_ms = [a.elapsed_time(b) for a, b in kev]
-    if world > 1:
-        t = torch.tensor([ms, float(np.mean(k_ms))], device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms, kmean = t.tolist()
-    else:
-        kmean = float(np.mean(k_ms))
-    value = nnz * args.steps / (ms / 1e3)
-
-    # roofline of the dominant kernel (the SGD epoch): north_star bytes/update = 12 + 16k
     peak, peak_src = hbm_peak()
-    b_upd = 12 + 16 * cfg.k
     local_nnz = info["local_nnz"]
-    achieved = local_nnz * b_upd / (kmean / 1e3) / 1e9
-    traffic = ncu_traffic(args.config, args.sched)
-    roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-            "traffic": traffic, "kernel": "sgd_kernel (a5/a6 epoch incl. Q sync)", "bytes_per_update": b_upd,
-            "updates_per_launch": local_nnz, "kernel_ms": kmean, "kernel_share_of_step": kmean / (ms / args.steps),
-            "peak_source": peak_src}
+
+    def measure(storage):
+        """W warm-up + K timed steps (epoch + Q sync + test RMSE) from a fresh init(1)."""
+        rm0 = mdl.rmse(dtu, dtv, dtr)
+        mdl.set_option("sync_stream", 0)
+
+        def step(ev=None):
+            if ev is not None:
+                ev[0].record(stream)
+            mdl.train_epoch(args.sched, sync)
+            if ev is not None:
+                ev[1].record(stream)
+            return mdl.rmse(dtu, dtv, dtr)
+
+        curve = [rm0] + [step() for _ in range(args.warmup)]
+        kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in range(args.steps)]
+        t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        clocks = Clocks(local)
+        clocks.start()
+        time.sleep(0.3)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t_start.record(stream)
+        rms = [step(kev[i]) for i in range(args.steps)]
+        t_end.record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        clk = clocks.stop()
+        mdl.set_option("sync_stream", 1)
+        ms = t_start.elapsed_time(t_end)
+        k_ms = [a.elapsed_time(b) for a, b in kev]
+        if world > 1:
+            t = torch.tensor([ms, float(np.mean(k_ms))], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms, kmean = t.tolist()
+        else:
+            kmean = float(np.mean(k_ms))
+        # roofline of the dominant kernel (the SGD epoch): north_star bytes/update = record
+        # (12 B) + read and write of p_u and q_v: 12 + 16k (fp32), 12 + 12k (binary16 Q)
+        b_upd = 12 + (16 if storage == "fp32" else 12) * cfg.k
+        achieved = local_nnz * b_upd / (kmean / 1e3) / 1e9
+        roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": ncu_traffic(args.config + ("" if storage == "fp32" else "-fp16"), args.sched),
+                "kernel": "sgd_warp_kernel (a5/a6 epoch incl. Q sync%s)"
+                          % ("" if storage == "fp32" else ", binary16 round-in/write-back of Q"),
+                "bytes_per_update": b_upd, "updates_per_launch": local_nnz, "kernel_ms": kmean,
+                "kernel_share_of_step": kmean / (ms / args.steps), "peak_source": peak_src}
+        return nnz * args.steps / (ms / 1e3), ms, roof, clk, curve + rms
+
+    value, ms, roof, clk, curve = measure(args.storage)
 
     out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
@@ -339,10 +351,23 @@ def main():
            "roofline": roof, "clocks": clk,
            "gpu_launches": args.steps * ((Bc if args.sched == "hogwild" else Br) * (G if sync == "ring" else 1)
                                          + 3),
-           "rmse": epochs_to_rmse(args.config, curve + rms),
+           "rmse": epochs_to_rmse(args.config, curve),
            "prep_s": t_prep, "gen_s": t_gen,
            "paper_context": {"netflix_hcc_updates_per_s": 2228476993,
                              "hardware": "2x Xeon Gold 6242 + RTX 2080 + RTX 2080S (Table 4, L2001)"}}
+    out["config"]["storage"] = args.storage
+    if args.storage == "fp16":
+        out["gpu_launches"] += args.steps * 2  # round-in / write-back of Q per launch
+    # secondary leg: the same workload with Q stored in binary16 (R26),
+    # fp32 arithmetic; same steps, same clocks rule; reported beside the fp32 headline
+    if args.storage == "fp32" and cfg.k % 128 == 0 and not args.no_fp16_leg:
+        mdl.set_option("storage", 1)
+        mdl.init(1)
+        v16, ms16, roof16, clk16, curve16 = measure("fp16")
+        out["storage_fp16"] = {"value": v16, "unit": UNIT, "ms_per_step": ms16 / args.steps, "roofline": roof16,
+                               "clocks": clk16, "rmse": epochs_to_rmse(args.config, curve16),
+                               "note": "Q held as IEEE binary16 during epochs (fp32 math, P fp32); "
+                                       "same band vs the fp64 oracle"}
 
     mdl.close()  # free HBM before the e2e jobs build their own handles
     # ---- e2e: the whole job through the public API from pinned host buffers
@@ -371,7 +396,7 @@ def main():
             if args.vec:
                 m2.set_option("vec", args.vec)
             m2.load(pin[0], pin[1], pin[2])
-            m2.partition(G, (Br, Bc), "DP0", seed=cfg.seed)
+            m2.partition(G, (Br, Bc), "DP0", seed=cfg.seed, storage=args.storage)
             m2.init(1)
             for _ in range(E):
                 m2.train_epoch(args.sched, sync)

@@ -178,13 +178,16 @@ typedef enum {
     HCCMF_OPT_L2_PERSIST = 12,   /* 1: during a Hogwild epoch Q is an L2 persisting
                                     access-policy window on the launch stream
                                     (removed afterwards).  Default 0.             */
-    HCCMF_OPT_PREFETCH_DEPTH = 13 /* Hogwild, one rating per warp (k = 128 j): the
+    HCCMF_OPT_PREFETCH_DEPTH = 13,/* Hogwild, one rating per warp (k = 128 j): the
                                     q_v row of rating j + D is requested while
                                     rating j is updated (1..4; default 1).  Loads
                                     issued before a warp's own update of the same
                                     item are corrected in registers, so a single
                                     warp stays serial; across warps D widens the
                                     read-to-write window (R14).         */
+    HCCMF_OPT_STORAGE = 14       /* Q storage from the next epoch on: 0 fp32, 1
+                                    binary16 (the partition option `storage`,
+                                    changeable without re-partitioning).          */
 } hccmf_option;
 
 /* ------------------------------------------------------------------ lifecycle */

@@ -570,6 +570,10 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
     case HCCMF_OPT_WIRE_FP16:
       h->opt_wire16 = value != 0;
       return HCCMF_OK;
+    case HCCMF_OPT_STORAGE:
+      if (value != 0 && value != 1) return fail(h, HCCMF_EINVAL, "storage must be 0 (fp32) or 1 (binary16 Q)");
+      h->storage = (int32_t)value;
+      return HCCMF_OK;
     case HCCMF_OPT_PREFETCH_DEPTH:
       if (value < 1 || value > 4) return fail(h, HCCMF_EINVAL, "prefetch depth must be in [1, 4]");
       h->opt_depth = value;

@@ -279,6 +279,7 @@ struct WarpSgd {
   float g, c1, ngl;
   const float4* __restrict__ Pb;
   const float4* __restrict__ Qb;
+  const char* Qhb;  // binary16 Q (storage = 1): lane's 4 halves of slot 0
 
   __device__ WarpSgd(const SgdArgs& args) : a(args) {
     lane = threadIdx.x & 31;
@@ -288,6 +289,7 @@ struct WarpSgd {
     ngl = -a.gamma * a.lambda;
     Pb = reinterpret_cast<const float4*>(a.P) + lane - (int64_t)a.row0 * k4;
     Qb = reinterpret_cast<const float4*>(a.Q) + lane;
+    Qhb = reinterpret_cast<const char*>(a.Q) + lane * 8;
   }
   // 32-bit row offsets: m_local * k/4 and n * k/4 < 2^31
   __device__ __forceinline__ const float4* prow(int u) const { return Pb + (int64_t)(u * k4); }
@@ -321,43 +323,44 @@ struct WarpSgd {
   // slot, slot i at +256 i).  The lane offset is folded into the base.
   template <bool QH>
   __device__ __forceinline__ const char* qaddr(int v) const {
-    const char* base = QH ? reinterpret_cast<const char*>(a.Q) + lane * 8 : reinterpret_cast<const char*>(Qb);
+    const char* base = QH ? Qhb : reinterpret_cast<const char*>(Qb);
     return base + (unsigned long long)(unsigned)v * (unsigned)(QH ? k4 * 8 : k4 * 16);
   }
   __device__ __forceinline__ const float4* pptr(int u) const {
     return reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Pb) +
                                            (unsigned long long)(unsigned)u * (unsigned)(k4 * 16));
   }
+  // q registers hold the row as stored (float4, or 4 binary16 in a uint2 for QH) and are
+  // widened only where used, so a prefetched load is not waited on by its conversion
   template <bool QH>
-  __device__ __forceinline__ void ldq(const char* q, float4 (&x)[VEC]) const {
-#pragma unroll
-    for (int i = 0; i < VEC; ++i) {
-      if (QH)
-        x[i] = h4_to_f4(__ldcg(reinterpret_cast<const uint2*>(q + 256 * i)));
-      else
-        x[i] = __ldcg(reinterpret_cast<const float4*>(q + 512 * i));
-    }
+  using QReg = typename std::conditional<QH, uint2, float4>::type;
+  template <bool QH>
+  static __device__ __forceinline__ float4 widen(const QReg<QH>& x) {
+    if constexpr (QH) return h4_to_f4(x); else return x;
   }
   template <bool QH>
-  __device__ __forceinline__ void stq(const char* q, const float4 (&x)[VEC]) const {
+  static __device__ __forceinline__ QReg<QH> narrow(const float4& x) {
+    if constexpr (QH) return f4_to_h4(x); else return x;
+  }
+  template <bool QH>
+  __device__ __forceinline__ void ldq(const char* q, QReg<QH> (&x)[VEC]) const {
 #pragma unroll
-    for (int i = 0; i < VEC; ++i) {
-      if (QH)
-        __stcg(reinterpret_cast<uint2*>(const_cast<char*>(q) + 256 * i), f4_to_h4(x[i]));
-      else
-        __stcg(reinterpret_cast<float4*>(const_cast<char*>(q) + 512 * i), x[i]);
-    }
+    for (int i = 0; i < VEC; ++i) x[i] = __ldcg(reinterpret_cast<const QReg<QH>*>(q + (QH ? 256 : 512) * i));
+  }
+  template <bool QH>
+  __device__ __forceinline__ void stq(const char* q, const QReg<QH> (&x)[VEC]) const {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) __stcg(reinterpret_cast<QReg<QH>*>(const_cast<char*>(q) + (QH ? 256 : 512) * i), x[i]);
   }
   // Hogwild!'s component-wise atomic add: red.global.add.v4.f32 (fp32 rows) or
   // red.global.add.noftz.v2.f16x2 of the increment rounded to binary16 (QH)
   template <bool QH>
-  __device__ __forceinline__ void redq(const char* q, const float4 (&d)[VEC]) const {
+  __device__ __forceinline__ void redq(const char* q, const QReg<QH> (&d)[VEC]) const {
 #pragma unroll
     for (int i = 0; i < VEC; ++i) {
-      if (QH) {
-        const uint2 h = f4_to_h4(d[i]);
-        asm volatile("red.relaxed.gpu.global.add.noftz.v2.f16x2 [%0], {%1, %2};" ::"l"(q + 256 * i), "r"(h.x),
-                     "r"(h.y)
+      if constexpr (QH) {
+        asm volatile("red.relaxed.gpu.global.add.noftz.v2.f16x2 [%0], {%1, %2};" ::"l"(q + 256 * i), "r"(d[i].x),
+                     "r"(d[i].y)
                      : "memory");
       } else {
         asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(q + 512 * i), "f"(d[i].x),
@@ -389,6 +392,7 @@ struct WarpSgd {
 
   template <bool QH>
   __device__ __forceinline__ void run_ring(int4* ring, int64_t lo, int left) {
+    using QR = QReg<QH>;
     const int32_t* ru = a.ru + lo;
     const int32_t* rv = a.rv + lo;
     const float* rr = a.rr + lo;
@@ -400,12 +404,13 @@ struct WarpSgd {
     float cr = __int_as_float(rec.z);
     const float4* pc = pptr(cu);
     const char* qc_p = qaddr<QH>(cv);
-    float4 p[VEC], pn[VEC], qa[VEC], qb[VEC];
+    float4 p[VEC], pn[VEC];
+    QR qa[VEC], qb[VEC];
     ld(pc, p);
     ldq<QH>(qc_p, qa);
 
-    // one step: update rating j (q in qc at qc_p), prefetch rating j+1 (q into qn)
-    auto step = [&](int j, float4 (&qc)[VEC], float4 (&qn)[VEC], auto has_next_tag, auto may_cross_tag) {
+    // one step: update rating j (q in qc_raw at qc_p), prefetch rating j+1 (q into qn)
+    auto step = [&](int j, QR (&qc_raw)[VEC], QR (&qn)[VEC], auto has_next_tag, auto may_cross_tag) {
       constexpr bool HAS_NEXT = decltype(has_next_tag)::value;
       constexpr bool MAY_CROSS = decltype(may_cross_tag)::value;
       int nu = 0, nv = 0;
@@ -430,6 +435,9 @@ struct WarpSgd {
         }
         if (newp) ld(pptr(nu), pn);
       }
+      float4 qc[VEC];
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) qc[i] = widen<QH>(qc_raw[i]);
       float d0 = 0.f, d1 = 0.f, d2 = 0.f, d3 = 0.f;
 #pragma unroll
       for (int i = 0; i < VEC; ++i) {
@@ -442,28 +450,21 @@ struct WarpSgd {
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
       const float ge = g * (cr - d);
-      float4 dq[VEC];
+      QR w[VEC];  // what is written: the increment (atomic) or the new row (store), as stored
 #pragma unroll
       for (int i = 0; i < VEC; ++i) {
-        dq[i] = f4_fma(ge, p[i], f4_scale(ngl, qc[i]));
+        const float4 dq = f4_fma(ge, p[i], f4_scale(ngl, qc[i]));
         p[i] = f4_fma(ge, qc[i], f4_scale(c1, p[i]));
+        w[i] = narrow<QH>(ATOMIC ? dq : f4_add(qc[i], dq));
       }
-      if (ATOMIC) {
-        redq<QH>(qc_p, dq);
-      } else {
-#pragma unroll
-        for (int i = 0; i < VEC; ++i) dq[i] = f4_add(qc[i], dq[i]);
-        stq<QH>(qc_p, dq);
-      }
+      if (ATOMIC)
+        redq<QH>(qc_p, w);
+      else
+        stq<QH>(qc_p, w);
       if (HAS_NEXT) {
-        if (fwd) {  // same item next (duplicates): serial read-after-write from registers
+        if (fwd) {  // same item next (duplicates): what memory now holds, from registers
 #pragma unroll
-          for (int i = 0; i < VEC; ++i) {
-            if (QH)  // what memory now holds: rn16(q + rn16(dq)) (atomic) or rn16(q + dq) (store)
-              qn[i] = h4_to_f4(f4_to_h4(ATOMIC ? f4_add(qc[i], h4_to_f4(f4_to_h4(dq[i]))) : dq[i]));
-            else
-              qn[i] = ATOMIC ? f4_add(qc[i], dq[i]) : dq[i];
-          }
+          for (int i = 0; i < VEC; ++i) qn[i] = ATOMIC ? narrow<QH>(f4_add(qc[i], widen<QH>(w[i]))) : w[i];
         }
         if (newp) {
           st(pc, p);
