@@ -33,6 +33,7 @@ import numpy as np  # noqa: E402
 import synth  # noqa: E402
 
 METRIC = "rating updates/sec (whole box)"
+STORAGE = {"fp32": 0, "fp16": 1, "fp16sr": 2}
 UNIT = "updates/s"
 FALLBACK_HBM_GBS = 6650.0
 DEVICE_GEN_NNZ = 1_000_000_000
@@ -54,10 +55,11 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
-    ap.add_argument("--storage", default="fp32", choices=["fp32", "fp16"],
-                    help="Q storage of the headline number (fp16 = binary16 Q, fp32 math, R26)")
-    ap.add_argument("--no-fp16-leg", action="store_true",
-                    help="skip the secondary binary16-Q measurement added to the JSON line")
+    ap.add_argument("--storage", default="fp32", choices=["fp32", "fp16", "fp16sr"],
+                    help="Q storage of the headline number (fp16 = binary16 Q, fp32 math, R26; "
+                         "fp16sr = with stochastic rounding, R27)")
+    ap.add_argument("--fp16-leg", default="fp16sr", choices=["fp16", "fp16sr", "none"],
+                    help="secondary binary16-Q measurement added to the JSON line")
     return ap.parse_args()
 
 
@@ -329,7 +331,7 @@ def main():
         b_upd = 12 + (16 if storage == "fp32" else 12) * cfg.k
         achieved = local_nnz * b_upd / (kmean / 1e3) / 1e9
         roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": ncu_traffic(args.config + ("" if storage == "fp32" else "-fp16"), args.sched),
+                "traffic": ncu_traffic(args.config + ("" if storage == "fp32" else "-" + storage), args.sched),
                 "kernel": "sgd_warp_kernel (a5/a6 epoch incl. Q sync%s)"
                           % ("" if storage == "fp32" else ", binary16 round-in/write-back of Q"),
                 "bytes_per_update": b_upd, "updates_per_launch": local_nnz, "kernel_ms": kmean,
@@ -356,18 +358,21 @@ def main():
            "paper_context": {"netflix_hcc_updates_per_s": 2228476993,
                              "hardware": "2x Xeon Gold 6242 + RTX 2080 + RTX 2080S (Table 4, L2001)"}}
     out["config"]["storage"] = args.storage
-    if args.storage == "fp16":
+    if args.storage != "fp32":
         out["gpu_launches"] += args.steps * 2  # round-in / write-back of Q per launch
     # secondary leg: the same workload with Q stored in binary16 (R26),
     # fp32 arithmetic; same steps, same clocks rule; reported beside the fp32 headline
-    if args.storage == "fp32" and cfg.k % 128 == 0 and not args.no_fp16_leg:
-        mdl.set_option("storage", 1)
+    if args.storage == "fp32" and cfg.k % 128 == 0 and args.fp16_leg != "none":
+        mdl.set_option("storage", STORAGE[args.fp16_leg])
         mdl.init(1)
-        v16, ms16, roof16, clk16, curve16 = measure("fp16")
-        out["storage_fp16"] = {"value": v16, "unit": UNIT, "ms_per_step": ms16 / args.steps, "roofline": roof16,
+        v16, ms16, roof16, clk16, curve16 = measure(args.fp16_leg)
+        out["storage_fp16"] = {"storage": args.fp16_leg, "value": v16, "unit": UNIT,
+                               "ms_per_step": ms16 / args.steps, "roofline": roof16,
                                "clocks": clk16, "rmse": epochs_to_rmse(args.config, curve16),
-                               "note": "Q held as IEEE binary16 during epochs (fp32 math, P fp32); "
-                                       "same band vs the fp64 oracle"}
+                               "note": "Q held as IEEE binary16 during epochs (fp32 math, P fp32)%s; "
+                                       "same band vs the fp64 oracle"
+                                       % (", stochastic rounding of every q write" if args.fp16_leg == "fp16sr"
+                                          else "")}
 
     mdl.close()  # free HBM before the e2e jobs build their own handles
     # ---- e2e: the whole job through the public API from pinned host buffers

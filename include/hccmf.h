@@ -106,7 +106,10 @@ typedef struct {
                              R26).  Needs one rating per warp
                              (k a multiple of 128): train_epoch returns EINVAL
                              otherwise.  Q read back (rmse, get_factors) holds
-                             binary16 values.                                    */
+                             binary16 values.  2 = as 1 with stochastic rounding
+                             of every q_v write (unbiased; random bits from a
+                             counter-based hash of (record, epoch, element pair),
+                             DESIGN.md R27).                                     */
     int32_t grid_dim;     /* 0 (default): row grid, shards of users, only Q moves;
                              1: column grid, shards of items, only P moves (Strategy 1
                              "transmitting P only", L1216-L1218); 2: the paper's rule
@@ -186,7 +189,8 @@ typedef enum {
                                     warp stays serial; across warps D widens the
                                     read-to-write window (R14).         */
     HCCMF_OPT_STORAGE = 14       /* Q storage from the next epoch on: 0 fp32, 1
-                                    binary16 (the partition option `storage`,
+                                    binary16, 2 binary16 with stochastic rounding
+                                    (the partition option `storage`,
                                     changeable without re-partitioning).          */
 } hccmf_option;
 

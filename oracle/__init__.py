@@ -66,7 +66,10 @@ def lib():
             "orc_epoch_phased": (ctypes.c_int, [i32, i32, i32, i32, P, i64, i32, f64, f64, P, P, P, P, P]),
             "orc_round_half": (f64, [f64]),
             "orc_epoch_wire16": (ctypes.c_int, [i32, i32, i32, i32, i32, P, i64, i32, f64, f64, P, P, P, P, P]),
-            "orc_epoch_q16": (ctypes.c_int, [i32, i32, i32, i32, i32, P, i64, i32, f64, f64, P, P, P, P, P, i32]),
+            "orc_epoch_q16": (ctypes.c_int, [i32, i32, i32, i32, i32, P, i64, i32, f64, f64, P, P, P, P, P, i32, i32,
+                                             ctypes.c_uint32]),
+            "orc_round_half_sr": (f64, [f64, ctypes.c_uint32]),
+            "orc_sr_word": (ctypes.c_uint32, [i64, ctypes.c_uint32, ctypes.c_uint32]),
             "orc_cost_model": (i32, [i32, i64, i64, i64, i32, P, P, f64, i32, i32, i32, f64, P, P, P, P]),
         }
         for name, (res, args) in sig.items():
@@ -230,6 +233,14 @@ def round_half(x: float) -> float:
     return float(lib().orc_round_half(float(x)))
 
 
+def round_half_sr(x: float, r13: int) -> float:
+    return float(lib().orc_round_half_sr(float(x), int(r13)))
+
+
+def sr_word(i: int, t: int, c: int) -> int:
+    return int(lib().orc_sr_word(int(i), int(t), int(c)))
+
+
 def epoch_wire16(sched, sync, G, Br, Bc, off, n, k, gamma, lam, ru, rv, rr, P, Q):
     """Ring / all-reduce epoch with FP16 transmission of Q (Strategy 2, R25)."""
     off = np.ascontiguousarray(off, dtype=np.int64)
@@ -239,12 +250,13 @@ def epoch_wire16(sched, sync, G, Br, Bc, off, n, k, gamma, lam, ru, rv, rr, P, Q
         raise ValueError("oracle wire16 epoch: invalid grid or sync")
 
 
-def epoch_q16(sched, sync, G, Br, Bc, off, n, k, gamma, lam, ru, rv, rr, P, Q, add16=False):
+def epoch_q16(sched, sync, G, Br, Bc, off, n, k, gamma, lam, ru, rv, rr, P, Q, add16=False, sr=False, t=0):
     """Epoch with Q stored in binary16 (every q_v write rounded; add16: the write is a
-    binary16 add of the rounded increment, as atomic Hogwild does; R26)."""
+    binary16 add of the rounded increment, as atomic Hogwild does; R26; sr:
+    stochastic rounding with the random words of epoch t, R27)."""
     off = np.ascontiguousarray(off, dtype=np.int64)
     rc = lib().orc_epoch_q16(SCHED[sched], SYNC[sync], G, Br, Bc, _p(off), n, P.shape[1], gamma, lam, _p(ru),
-                             _p(rv), _p(rr), _p(P), _p(Q), int(bool(add16)))
+                             _p(rv), _p(rr), _p(P), _p(Q), int(bool(add16)), int(bool(sr)), int(t))
     if rc != 0:
         raise ValueError("oracle q16 epoch: invalid grid for this schedule")
 
@@ -298,9 +310,9 @@ class Problem:
         epoch(sched, sync, self.G, self.Br, self.Bc, self.off, self.n, self.k, self.gamma, self.lam,
               self.ru, self.rv, self.rr, self.P, self.Q)
 
-    def epoch_q16(self, sched="det", sync="none", add16=False):
+    def epoch_q16(self, sched="det", sync="none", add16=False, sr=False, t=0):
         epoch_q16(sched, sync, self.G, self.Br, self.Bc, self.off, self.n, self.k, self.gamma, self.lam,
-                  self.ru, self.rv, self.rr, self.P, self.Q, add16)
+                  self.ru, self.rv, self.rr, self.P, self.Q, add16, sr, t)
 
     def epoch_wire16(self, sched="det", sync="ring"):
         epoch_wire16(sched, sync, self.G, self.Br, self.Bc, self.off, self.n, self.k, self.gamma, self.lam,

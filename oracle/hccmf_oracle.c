@@ -306,6 +306,43 @@ double orc_round_half(double x);
 /* wise atomic add on binary16 words).  P is never rounded.  Set per call by      */
 /* orc_epoch_q16.                                                                 */
 static int g_q16 = 0;
+static uint32_t g_sr_epoch = 0; /* mode 3 (stochastic rounding): epoch t of the random words */
+static int64_t g_sr_rec = 0;    /* mode 3: global index of the record being updated          */
+
+/* Stochastic rounding to binary16 (storage = 2, R27), from its definition:
+ * y = sign(x) * floor((|x| + R13 * ulp / 2^13) / ulp) * ulp, with ulp the binary16 spacing
+ * at |x| (2^(e-10) for |x| in [2^e, 2^(e+1)), e >= -14; 2^-24 below 2^-14) and R13 in
+ * [0, 2^13) random: the result is one of the two binary16 neighbours of x, the upper
+ * one with probability (fraction of x past the lower one) quantised to 2^-13 ulp. */
+double orc_round_half_sr(double x, uint32_t r13)
+{
+    if (x != x) return x;
+    double a = fabs(x);
+    if (a == 0.0) return x;
+    int e;
+    frexp(a, &e);
+    int lead = e - 1;
+    if (lead < -14) lead = -14;
+    double ulp = ldexp(1.0, lead - 10);
+    double y = floor((a + (double)(r13 & 0x1FFFu) * ulp / 8192.0) / ulp) * ulp;
+    if (y >= 65536.0) y = INFINITY;
+    return x < 0 ? -y : y;
+}
+
+/* The random word of element pair c (elements 2c, 2c+1) for the q write of record i in
+ * epoch t (R27): lowbias32(i*0x9E3779B1 + t*0x85EBCA77 + c*0xC2B2AE3D mod 2^32), with
+ * lowbias32 the 32-bit finaliser of C. Wellons (xorshift-multiply, 2 rounds).  Element 2c
+ * takes bits 12:0, element 2c+1 bits 28:16. */
+uint32_t orc_sr_word(int64_t i, uint32_t t, uint32_t c)
+{
+    uint32_t x = (uint32_t)i * 0x9E3779B1u + t * 0x85EBCA77u + c * 0xC2B2AE3Du;
+    x ^= x >> 16;
+    x *= 0x7FEB352Du;
+    x ^= x >> 15;
+    x *= 0x846CA68Bu;
+    x ^= x >> 16;
+    return x;
+}
 
 double orc_sgd_update(int32_t k, double gamma, double lambda, double* p, double* q, double r)
 {
@@ -315,7 +352,10 @@ double orc_sgd_update(int32_t k, double gamma, double lambda, double* p, double*
     for (int32_t j = 0; j < k; ++j) {
         double pj = p[j], qj = q[j];
         p[j] = pj + gamma * (e * qj - lambda * pj);
-        if (g_q16 == 2)
+        if (g_q16 == 3) {
+            uint32_t w = orc_sr_word(g_sr_rec, g_sr_epoch, (uint32_t)(j / 2));
+            q[j] = orc_round_half_sr(qj + gamma * (e * pj - lambda * qj), (j % 2 == 0) ? (w & 0x1FFFu) : ((w >> 16) & 0x1FFFu));
+        } else if (g_q16 == 2)
             q[j] = orc_round_half(qj + orc_round_half(gamma * (e * pj - lambda * qj)));
         else if (g_q16 == 1)
             q[j] = orc_round_half(qj + gamma * (e * pj - lambda * qj));
@@ -329,8 +369,10 @@ double orc_sgd_update(int32_t k, double gamma, double lambda, double* p, double*
 void orc_run(int64_t lo, int64_t hi, int32_t k, double gamma, double lambda, const int32_t* ru,
              const int32_t* rv, const float* rr, double* P, double* Q)
 {
-    for (int64_t i = lo; i < hi; ++i)
+    for (int64_t i = lo; i < hi; ++i) {
+        g_sr_rec = i;
         orc_sgd_update(k, gamma, lambda, P + (int64_t)ru[i] * k, Q + (int64_t)rv[i] * k, (double)rr[i]);
+    }
 }
 
 /* One epoch in the canonical serialisation of a schedule (R19).
@@ -612,14 +654,17 @@ int orc_epoch_wire16(int32_t sched, int32_t sync, int32_t G, int32_t Br, int32_t
 /* orc_epoch with Q stored in binary16 (storage = 1, R26): Q is rounded
  * to binary16 first (the epoch starts from stored values), then every q_v write
  * is rounded (orc_sgd_update; add16 = 1: as a binary16 add of the rounded
- * increment).  Same schedules, grids and return codes. */
+ * increment; sr = 1: stochastically rounded with the random words of epoch t,
+ * storage = 2, R27).  Same schedules, grids and return codes.  Record indices are
+ * positions in the sorted record array (global order). */
 int orc_epoch_q16(int32_t sched, int32_t sync, int32_t G, int32_t Br, int32_t Bc, const int64_t* off,
                   int64_t n, int32_t k, double gamma, double lambda, const int32_t* ru, const int32_t* rv,
-                  const float* rr, double* P, double* Q, int32_t add16)
+                  const float* rr, double* P, double* Q, int32_t add16, int32_t sr, uint32_t t)
 {
     size_t qn = (size_t)n * (size_t)k;
     for (size_t i = 0; i < qn; ++i) Q[i] = orc_round_half(Q[i]);
-    g_q16 = add16 ? 2 : 1;
+    g_q16 = sr ? 3 : (add16 ? 2 : 1);
+    g_sr_epoch = t;
     int rc = orc_epoch(sched, sync, G, Br, Bc, off, n, k, gamma, lambda, ru, rv, rr, P, Q);
     g_q16 = 0;
     return rc;

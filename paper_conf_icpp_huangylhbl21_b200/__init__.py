@@ -234,12 +234,13 @@ class Model:
     def partition(self, n_shards=1, grid=(1, 1), strategy="DP0", seed=0, x=None, t_meas=None, t_sync=0.0,
                   grid_dim="rows", storage="fp32"):
         """grid_dim: "rows" (shards of users, Q moves), "cols" (shards of items, P moves) or
-        "auto" (the paper's rule, L884-L886).  storage: "fp32", or "fp16" = Q held in IEEE
-        binary16 during epochs, fp32 arithmetic (R26; k a multiple of 128)."""
+        "auto" (the paper's rule, L884-L886).  storage: "fp32"; "fp16" = Q held in IEEE
+        binary16 during epochs, fp32 arithmetic, round to nearest (R26; k a multiple
+        of 128); "fp16sr" = the same with stochastic rounding of every q write (R27)."""
         px, kx = _buf(x, np.float64)
         pt, kt = _buf(t_meas, np.float64)
         o = PartitionOpts(int(n_shards), int(grid[0]), int(grid[1]), DP[strategy] if isinstance(strategy, str)
-                          else int(strategy), px, pt, float(t_sync), int(seed), {"fp32": 0, "fp16": 1}[storage],
+                          else int(strategy), px, pt, float(t_sync), int(seed), {"fp32": 0, "fp16": 1, "fp16sr": 2}[storage],
                           {"rows": 0, "cols": 1, "auto": 2}[grid_dim])
         self._check(lib().hccmf_partition(self._h, ctypes.byref(o)))
         self.G, self.grid = int(n_shards), (int(grid[0]), int(grid[1]))

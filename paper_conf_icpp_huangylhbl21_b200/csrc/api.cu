@@ -571,7 +571,7 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
       h->opt_wire16 = value != 0;
       return HCCMF_OK;
     case HCCMF_OPT_STORAGE:
-      if (value != 0 && value != 1) return fail(h, HCCMF_EINVAL, "storage must be 0 (fp32) or 1 (binary16 Q)");
+      if (value < 0 || value > 2) return fail(h, HCCMF_EINVAL, "storage must be 0 (fp32), 1 (binary16 Q) or 2 (binary16 Q, stochastic rounding)");
       h->storage = (int32_t)value;
       return HCCMF_OK;
     case HCCMF_OPT_PREFETCH_DEPTH:
@@ -671,7 +671,7 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   if (G < 1) return fail(h, HCCMF_EINVAL, "n_shards must be >= 1");
   if (h->world > 1 && G != h->world) return fail(h, HCCMF_EINVAL, "n_shards must equal the world size");
   if (o->grid_rows < 1 || o->grid_cols < 1) return fail(h, HCCMF_EINVAL, "grid must be >= 1 x 1");
-  if (o->storage != 0 && o->storage != 1) return fail(h, HCCMF_EINVAL, "storage must be 0 (fp32) or 1 (binary16 Q)");
+  if (o->storage < 0 || o->storage > 2) return fail(h, HCCMF_EINVAL, "storage must be 0 (fp32), 1 (binary16 Q) or 2 (binary16 Q, stochastic rounding)");
   if (o->strategy < HCCMF_DP0 || o->strategy > HCCMF_DP2) return fail(h, HCCMF_EINVAL, "bad strategy");
   if ((o->strategy != HCCMF_DP0) && !o->t_meas) return fail(h, HCCMF_EINVAL, "DP1/DP2 need t_meas");
   if (o->grid_dim < 0 || o->grid_dim > 2) return fail(h, HCCMF_EINVAL, "grid_dim must be 0, 1 or 2");
@@ -865,6 +865,7 @@ hccmf_status hccmf_init_factors(hccmf_t h, uint64_t seed) {
   CU(h, k_init_factors(seed, tcol, h->n, h->k, h->d_perm_col, 0, h->n, h->d_Q, h->stream));
   h->q_ring_sched = -1;
   h->state = 3;
+  h->epoch = 0;
   return finish(h);
 }
 
@@ -883,6 +884,7 @@ hccmf_status hccmf_set_factors(hccmf_t h, const float* P, const float* Q) {
   cudaFreeAsync(tmp, h->stream);
   h->q_ring_sched = -1;
   h->state = 3;
+  h->epoch = 0;
   return finish(h);
 }
 
@@ -892,7 +894,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   if (sched != HCCMF_SCHED_DET && sched != HCCMF_SCHED_HOGWILD) return fail(h, HCCMF_EINVAL, "bad schedule");
   if (sync < HCCMF_SYNC_NONE || sync > HCCMF_SYNC_ALLREDUCE_AVG) return fail(h, HCCMF_EINVAL, "bad sync");
   const int G = h->G;
-  if (h->storage == 1) {  // binary16 Q lives in the warp-per-rating kernel (one rating per warp)
+  if (h->storage >= 1) {  // binary16 Q lives in the warp-per-rating kernel (one rating per warp)
     int L = 0, VEC = 0;
     sgd_geometry(h->k, (int)h->opt_vec, &L, &VEC);
     if (L != 32 || L * VEC * 4 != h->k)
@@ -914,6 +916,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     a.vec_pref = (int32_t)h->opt_vec;
     a.prefetch = 1;
     CU(h, launch_wave(a, h->d_blk_off, h->Br, h->d_progress, h->stream));
+    ++h->epoch;
     return finish(h);
   }
   Plan* pl = nullptr;
@@ -960,7 +963,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   // replica, the end of the epoch).
   float* qh_of = nullptr;
   int64_t qh_a = 0, qh_b = 0;
-  if (h->storage == 1 && !h->d_Qh) CU(h, dmalloc(h, &h->d_Qh, (size_t)nk));
+  if (h->storage >= 1 && !h->d_Qh) CU(h, dmalloc(h, &h->d_Qh, (size_t)nk));
   auto qh_flush = [&]() -> hccmf_status {
     if (qh_of && qh_b > qh_a)
       CU(h, k_unpack_half(h->d_Qh + qh_a * h->k, qh_of + qh_a * h->k, (qh_b - qh_a) * h->k, s));
@@ -995,7 +998,9 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   a.vec_pref = (int32_t)h->opt_vec;
   a.prefetch = sched == HCCMF_SCHED_DET ? 1 : 0;
   a.depth = (sched == HCCMF_SCHED_HOGWILD && h->storage == 0) ? (int32_t)h->opt_depth : 1;
-  a.qhalf = h->storage == 1 ? 1 : 0;
+  a.qhalf = h->storage;
+  a.rec0 = h->rec0;
+  a.epoch = h->epoch;
   const int L = sgd_lanes(h->k, (int)h->opt_vec);
   // a ring stage races only on its column group's items
   const int64_t hog_warps = auto_warps(h, eff_sync == HCCMF_SYNC_RING ? h->n / G : h->n);
@@ -1070,7 +1075,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
         if (h->storage == 0) CU(h, k_round_half(h->d_Q, nk, s));
     }
     a.Q = (eff_sync == HCCMF_SYNC_ALLREDUCE_AVG && !dist) ? h->d_Qrep + (size_t)ln.qrep * nk : h->d_Q;
-    if (h->storage == 1) {
+    if (h->storage >= 1) {
       // rows this launch may touch: its column block (pipelined ring), its column group
       // (stage-wise ring), else all of Q
       int64_t ra = 0, rb = h->n;
@@ -1129,6 +1134,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     st = average();
     if (st != HCCMF_OK) return st;
   }
+  ++h->epoch;
   return finish(h);
 }
 

@@ -66,7 +66,9 @@ struct SgdArgs {
   int32_t vec_pref;  // float4 slots per lane (0 = auto)
   int32_t prefetch;  // L2 bulk prefetch of the next window's p_u / q_v rows (DET blocks)
   int32_t depth;     // q_v prefetch distance in ratings (warp-per-rating Hogwild kernel)
-  int32_t qhalf;     // Q is IEEE binary16 (storage = 1; warp-per-rating kernel only)
+  int32_t qhalf;     // Q is IEEE binary16: 1 round to nearest, 2 stochastic rounding (R26, R27)
+  int64_t rec0;      // global index of local record 0 (SR random words)
+  unsigned epoch;    // epochs since the factors were set (SR random words)
 };
 
 // launch the SGD kernel for a list of tasks; warps = concurrent warps wanted
@@ -176,7 +178,8 @@ struct hccmf_ctx {
   float* d_P = nullptr;
   float* d_Q = nullptr;
   float* d_Qrep = nullptr;  // logical all-reduce replicas
-  int32_t storage = 0;      // 1: Q held in binary16 while an epoch runs (R26)
+  int32_t storage = 0;      // 1: Q held in binary16 while an epoch runs (R26); 2: with stochastic rounding (R27)
+  uint32_t epoch = 0;       // train_epoch calls since init_factors / set_factors
   uint16_t* d_Qh = nullptr; // n x k binary16 copy of Q, authoritative inside an epoch (storage = 1)
   unsigned long long* d_counters = nullptr;
   int64_t n_counters = 0;

@@ -85,6 +85,30 @@ __device__ __forceinline__ uint2 f4_to_h4(float4 a) {
   const __half2 lo = __floats2half2_rn(a.x, a.y), hi = __floats2half2_rn(a.z, a.w);
   return make_uint2(*reinterpret_cast<const unsigned*>(&lo), *reinterpret_cast<const unsigned*>(&hi));
 }
+// Stochastic rounding (storage = 2, R27).  The random word of element pair c
+// (elements 2c, 2c+1) of the q_v write by the update of record i (global index in the
+// sorted order) in epoch t is r = lowbias32(i*0x9E3779B1 + t*0x85EBCA77 + c*0xC2B2AE3D)
+// (mod 2^32; lowbias32 = C. Wellons' 32-bit finaliser); element 2c is rounded with
+// r[12:0], element 2c+1 with r[28:16] by cvt.rs.f16x2.f32 (sm_100a F2FP.RS):
+// y = sign(x) floor((|x| + R13 ulp / 2^13) / ulp) ulp, ulp = the binary16 spacing at |x|.
+__device__ __forceinline__ unsigned lowbias32(unsigned x) {
+  x ^= x >> 16;
+  x *= 0x7FEB352Du;
+  x ^= x >> 15;
+  x *= 0x846CA68Bu;
+  x ^= x >> 16;
+  return x;
+}
+__device__ __forceinline__ unsigned cvt_rs_h2(float hi, float lo, unsigned r) {
+  unsigned d;
+  asm("cvt.rs.f16x2.f32 %0, %1, %2, %3;" : "=r"(d) : "f"(hi), "f"(lo), "r"(r));
+  return d;
+}
+__device__ __forceinline__ unsigned hsub2_bits(unsigned a, unsigned b) {  // a - b, binary16 x2, RN
+  unsigned d;
+  asm("sub.rn.f16x2 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b));
+  return d;
+}
 __device__ __forceinline__ float4 h4_to_f4(uint2 r) {
   const float2 lo = __half22float2(*reinterpret_cast<const __half2*>(&r.x));
   const float2 hi = __half22float2(*reinterpret_cast<const __half2*>(&r.y));
@@ -390,9 +414,13 @@ struct WarpSgd {
     __syncwarp();
   }
 
-  template <bool QH>
+  template <bool QH, bool SR = false>
   __device__ __forceinline__ void run_ring(int4* ring, int64_t lo, int left) {
+    static_assert(!SR || QH, "stochastic rounding needs binary16 storage");
     using QR = QReg<QH>;
+    // SR: random word base of rating j = (rec0 + lo + j) * A + t * B (mod 2^32)
+    const unsigned rb0 = (unsigned)(a.rec0 + lo) * 0x9E3779B1u + a.epoch * 0x85EBCA77u +
+                         (unsigned)(2 * lane) * 0xC2B2AE3Du;
     const int32_t* ru = a.ru + lo;
     const int32_t* rv = a.rv + lo;
     const float* rr = a.rr + lo;
@@ -451,11 +479,25 @@ struct WarpSgd {
       for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
       const float ge = g * (cr - d);
       QR w[VEC];  // what is written: the increment (atomic) or the new row (store), as stored
+      QR snew[VEC];  // SR: the new row as stored
 #pragma unroll
       for (int i = 0; i < VEC; ++i) {
-        const float4 dq = f4_fma(ge, p[i], f4_scale(ngl, qc[i]));
+        if constexpr (SR) {
+          // q' = q + dq = c1 q + (g e) p, stochastically rounded to binary16; the atomic
+          // increment is q' - q, exact in binary16 (both on q's grid), so a serial run
+          // stores exactly q'
+          const float4 qq = f4_fma(ge, p[i], f4_scale(c1, qc[i]));
+          const unsigned r = rb0 + (unsigned)j * 0x9E3779B1u + (unsigned)(64 * i) * 0xC2B2AE3Du;
+          uint2 hs;
+          hs.x = cvt_rs_h2(qq.y, qq.x, lowbias32(r));
+          hs.y = cvt_rs_h2(qq.w, qq.z, lowbias32(r + 0xC2B2AE3Du));
+          snew[i] = hs;
+          w[i] = ATOMIC ? make_uint2(hsub2_bits(hs.x, qc_raw[i].x), hsub2_bits(hs.y, qc_raw[i].y)) : hs;
+        } else {
+          const float4 dq = f4_fma(ge, p[i], f4_scale(ngl, qc[i]));
+          w[i] = narrow<QH>(ATOMIC ? dq : f4_add(qc[i], dq));
+        }
         p[i] = f4_fma(ge, qc[i], f4_scale(c1, p[i]));
-        w[i] = narrow<QH>(ATOMIC ? dq : f4_add(qc[i], dq));
       }
       if (ATOMIC)
         redq<QH>(qc_p, w);
@@ -464,7 +506,12 @@ struct WarpSgd {
       if (HAS_NEXT) {
         if (fwd) {  // same item next (duplicates): what memory now holds, from registers
 #pragma unroll
-          for (int i = 0; i < VEC; ++i) qn[i] = ATOMIC ? narrow<QH>(f4_add(qc[i], widen<QH>(w[i]))) : w[i];
+          for (int i = 0; i < VEC; ++i) {
+            if constexpr (SR)
+              qn[i] = snew[i];
+            else
+              qn[i] = ATOMIC ? narrow<QH>(f4_add(qc[i], widen<QH>(w[i]))) : w[i];
+          }
         }
         if (newp) {
           st(pc, p);
@@ -721,7 +768,7 @@ struct WarpSgd {
 #ifndef HCCMF_WARP_MINB
 #define HCCMF_WARP_MINB 1
 #endif
-template <int VEC, bool ATOMIC, int D, bool QH>
+template <int VEC, bool ATOMIC, int D, int QM>  // QM: 0 fp32 Q, 1 binary16 RN, 2 binary16 SR
 __global__ void __launch_bounds__(kThreads, (VEC == 1 ? 4 : HCCMF_WARP_MINB)) sgd_warp_kernel(SgdArgs a) {
   constexpr unsigned FM = 0xffffffffu;
   WarpSgd<VEC, ATOMIC> w(a);
@@ -735,7 +782,9 @@ __global__ void __launch_bounds__(kThreads, (VEC == 1 ? 4 : HCCMF_WARP_MINB)) sg
     const int left = (int)(a.task_hi[tn] - lo);
     unsigned long long tn2 = 0;
     if (w.lane == 0) tn2 = atomicAdd(a.counter, 1ull);  // next task id, fetched one task ahead
-    if (D == 1 && QH)
+    if (D == 1 && QM == 2)
+      w.template run_ring<true, true>(ring, lo, left);
+    else if (D == 1 && QM == 1)
       w.template run_ring<true>(ring, lo, left);
     else if (D == 1)
       w.template run_ring<false>(ring, lo, left);
@@ -793,14 +842,14 @@ cudaError_t launch_t(const SgdArgs& a, int64_t warps, cudaStream_t st) {
   if (L == 32 && FULL) {  // warp-per-rating specialisation
     const int depth = a.depth < 1 ? 1 : a.depth;
 #define WARP_CASE(DD, QQ)                                                     \
-  if (depth == DD && (a.qhalf != 0) == QQ) {                                  \
+  if (depth == DD && a.qhalf == QQ) {                                         \
     if (a.atomic_q)                                                           \
       sgd_warp_kernel<VEC, true, DD, QQ><<<(unsigned)blocks, threads, 0, st>>>(a);  \
     else                                                                      \
       sgd_warp_kernel<VEC, false, DD, QQ><<<(unsigned)blocks, threads, 0, st>>>(a); \
     return cudaGetLastError();                                                \
   }
-    WARP_CASE(1, false) WARP_CASE(2, false) WARP_CASE(3, false) WARP_CASE(4, false) WARP_CASE(1, true)
+    WARP_CASE(1, 0) WARP_CASE(2, 0) WARP_CASE(3, 0) WARP_CASE(4, 0) WARP_CASE(1, 1) WARP_CASE(1, 2)
 #undef WARP_CASE
     return cudaErrorInvalidValue;
   }

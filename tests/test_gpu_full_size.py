@@ -65,7 +65,8 @@ def test_c3_partition_bitexact_full_size(pkg, c3, B):
     assert _digest(mdl) == ref[key]
 
 
-@pytest.mark.parametrize("name,data,storage", [("c3", "c3", "fp32"), ("c2", None, "fp32"), ("c3", "c3", "fp16")])
+@pytest.mark.parametrize("name,data,storage", [("c3", "c3", "fp32"), ("c2", None, "fp32"), ("c3", "c3", "fp16"),
+                                                ("c3", "c3", "fp16sr")])
 def test_hogwild_band_full_size(pkg, c3, name, data, storage):
     # bench.py's configuration: one shard, grid (1, 1), library defaults, init seed 1.
     # storage fp16 (Q in binary16, R26) is held to the same band against the fp64 oracle.

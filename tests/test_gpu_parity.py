@@ -469,8 +469,9 @@ def _q16_bar(x):
     return 1e-4 + np.abs(x) * 2.0 ** -9
 
 
-@pytest.mark.parametrize("k,B,epochs", [(128, 8, 1), (128, 8, 3), (256, 4, 1)])
-def test_det_epoch_parity_q16(pkg, orc, k, B, epochs):
+@pytest.mark.parametrize("k,B,epochs,sr", [(128, 8, 1, False), (128, 8, 3, False), (256, 4, 1, False),
+                                           (128, 8, 1, True), (128, 8, 3, True), (256, 4, 2, True)])
+def test_det_epoch_parity_q16(pkg, orc, k, B, epochs, sr):
     cfg = synth.CONFIGS["c1"]
     (u, v, r), (tu, tv, tr) = synth.make(cfg)
     gamma = 0.02
@@ -480,11 +481,11 @@ def test_det_epoch_parity_q16(pkg, orc, k, B, epochs):
     prob.set_factors(P0, Q0)
     mdl = pkg.Model(cfg.m, cfg.n, k, gamma, cfg.lam)
     mdl.load(u, v, r)
-    mdl.partition(1, (B, B), seed=11, storage="fp16")
+    mdl.partition(1, (B, B), seed=11, storage="fp16sr" if sr else "fp16")
     mdl.set_factors(P0, Q0)
-    for _ in range(epochs):
+    for t in range(epochs):  # SR: the random words of epoch t (R27) are the same on both sides
         mdl.train_epoch("det", "none")
-        prob.epoch_q16("det", "none")
+        prob.epoch_q16("det", "none", sr=sr, t=t)
     P, Q = mdl.factors()
     Po, Qo = prob.factors()
     assert np.array_equal(Q.astype(np.float16).astype(np.float32), Q)  # Q holds binary16 values
@@ -493,8 +494,8 @@ def test_det_epoch_parity_q16(pkg, orc, k, B, epochs):
     assert mdl.rmse(tu, tv, tr) == pytest.approx(prob.rmse(tu, tv, tr), abs=1e-4)
 
 
-@pytest.mark.parametrize("atomic", [0, 1])
-def test_hogwild_single_group_q16(pkg, orc, atomic):
+@pytest.mark.parametrize("atomic,sr", [(0, False), (1, False), (0, True), (1, True)])
+def test_hogwild_single_group_q16(pkg, orc, atomic, sr):
     # one warp walks the tasks in record order: the binary16 Hogwild kernel is then the
     # oracle's serial epoch with binary16 Q (atomic: the increment is itself rounded
     # to binary16 before the add, one more rounding than the oracle's)
@@ -509,21 +510,22 @@ def test_hogwild_single_group_q16(pkg, orc, atomic):
     mdl.set_option("task_ratings", 300)
     mdl.set_option("heavy_first", -1)
     mdl.load(u, v, r)
-    mdl.partition(1, (1, 1), seed=3, storage="fp16")
+    mdl.partition(1, (1, 1), seed=3, storage="fp16sr" if sr else "fp16")
     mdl.set_option("hogwild_warps", 1)
     mdl.set_option("hogwild_atomic", atomic)
     mdl.set_factors(P0, Q0)
-    for _ in range(2):
+    for t in range(2):  # SR: serially, the atomic add of (SR(q + dq) - q) stores SR(q + dq)
         mdl.train_epoch("hogwild", "none")
-        prob.epoch_q16("serial", "none", add16=bool(atomic))
+        prob.epoch_q16("serial", "none", add16=bool(atomic) and not sr, sr=sr, t=t)
     P, Q = mdl.factors()
     Po, Qo = prob.factors()
     assert np.all(np.abs(P - Po) <= _q16_bar(Po)), np.abs(P - Po).max()
     assert np.all(np.abs(Q - Qo) <= _q16_bar(Qo)), np.abs(Q - Qo).max()
 
 
-@pytest.mark.parametrize("sync,G,Br,Bc", [("ring", 2, 4, 8), ("allreduce", 2, 4, 4)])
-def test_det_logical_shards_parity_q16(pkg, orc, sync, G, Br, Bc):
+@pytest.mark.parametrize("sync,G,Br,Bc,sr", [("ring", 2, 4, 8, False), ("allreduce", 2, 4, 4, False),
+                                             ("ring", 2, 4, 8, True), ("allreduce", 2, 4, 4, True)])
+def test_det_logical_shards_parity_q16(pkg, orc, sync, G, Br, Bc, sr):
     cfg = synth.CONFIGS["c1"]
     (u, v, r), _ = synth.make(cfg)
     k, gamma = 128, 0.02
@@ -533,11 +535,11 @@ def test_det_logical_shards_parity_q16(pkg, orc, sync, G, Br, Bc):
     prob.set_factors(P0, Q0)
     mdl = pkg.Model(cfg.m, cfg.n, k, gamma, cfg.lam)
     mdl.load(u, v, r)
-    mdl.partition(G, (Br, Bc), seed=5, storage="fp16")
+    mdl.partition(G, (Br, Bc), seed=5, storage="fp16sr" if sr else "fp16")
     mdl.set_factors(P0, Q0)
-    for _ in range(2):
+    for t in range(2):
         mdl.train_epoch("det", sync)
-        prob.epoch_q16("det", sync)
+        prob.epoch_q16("det", sync, sr=sr, t=t)
     P, Q = mdl.factors()
     Po, Qo = prob.factors()
     assert np.all(np.abs(P - Po) <= _q16_bar(Po)), np.abs(P - Po).max()

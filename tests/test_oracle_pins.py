@@ -410,3 +410,92 @@ def test_q16_storage_epoch_invariants(orc):
         c.set_factors(P0, Q0)
         c.epoch_q16(sched, sync, add16=True)
         assert 0 < np.abs(b.Q - c.Q).max() <= 8 * 2.0 ** -11 * np.abs(b.Q).max()
+
+
+def _f16_down(x):
+    """largest binary16 value <= |x| (numpy's IEEE conversion, stepped toward zero)"""
+    a = abs(float(x))
+    d = np.float16(a)
+    if float(d) > a:
+        d = np.nextafter(d, np.float16(0))
+    return float(d)
+
+
+def test_sr_rounding_definition(orc):
+    # R27: one of the two binary16 neighbours; on-grid values are kept for every R;
+    # R = 0 truncates toward zero; averaging over all 2^13 random inputs reproduces any
+    # fp32 value of the normal binary16 range exactly (13 dropped bits), i.e. unbiased
+    rng = np.random.default_rng(11)
+    xs = np.concatenate([rng.uniform(-3, 3, 40), rng.uniform(2.0 ** -14, 1e-3, 20),
+                         rng.uniform(100, 60000, 20)]).astype(np.float32)
+    R = np.arange(8192)
+    for x in xs:
+        x = float(x)
+        dn = _f16_down(x)
+        up = float(np.nextafter(np.float16(dn), np.float16(np.inf)))
+        ys = np.array([orc.round_half_sr(x, int(r)) for r in R[::64]] + [orc.round_half_sr(x, 8191)])
+        assert set(np.abs(ys)) <= {dn, up}, x
+        assert abs(orc.round_half_sr(x, 0)) == dn
+        full = np.array([orc.round_half_sr(x, int(r)) for r in R])
+        assert full.mean() == x  # exact: the fraction past dn is a multiple of 2^-13 ulp
+    for h in (np.float16(0.3), np.float16(-2.5), np.float16(6e-5), np.float16(1e-7)):
+        for r in (0, 1, 4095, 8191):
+            assert orc.round_half_sr(float(h), r) == float(h)
+
+
+def test_sr_word_is_the_stated_hash(orc):
+    # lowbias32 inverted step by step (modular inverses of the odd multipliers, xorshift
+    # inverses) must give back i*0x9E3779B1 + t*0x85EBCA77 + c*0xC2B2AE3D mod 2^32
+    M = 2 ** 32
+    inv1, inv2 = pow(0x846CA68B, -1, M), pow(0x7FEB352D, -1, M)
+    rng = np.random.default_rng(2)
+    for _ in range(300):
+        i, t, c = int(rng.integers(0, 2 ** 40)), int(rng.integers(0, 2 ** 32)), int(rng.integers(0, 2 ** 12))
+        x = orc.sr_word(i, t, c)
+        x ^= x >> 16
+        x = (x * inv1) % M
+        x ^= (x >> 15) ^ (x >> 30)
+        x = (x * inv2) % M
+        x ^= x >> 16
+        assert x == (i * 0x9E3779B1 + t * 0x85EBCA77 + c * 0xC2B2AE3D) % M
+    # the two 13-bit fields are uniform
+    w = np.array([orc.sr_word(i, 3, c) for i in range(2000) for c in range(8)], dtype=np.uint64)
+    for f in (w & 0x1FFF, (w >> 16) & 0x1FFF):
+        h = np.bincount((f >> 9).astype(np.int64), minlength=16)  # 16 bins of 512
+        exp = len(f) / 16
+        assert ((h - exp) ** 2 / exp).sum() < 50  # chi-square, 15 dof (p ~ 1e-5)
+
+
+def test_sr_epoch_single_update_and_invariants(orc):
+    # Fig. 1 rating (0, 0, 5.0), gamma = 0.005 (see test_q16_storage_single_update_hand_computed):
+    # q0 + dq0 = 2.090297041015625 lies 0.232085 ulps (2^-9) above 2.08984375, so it
+    # rounds up iff R13 >= 8192 * (1 - 0.232085) = 6290.8; q1 + dq1 = 0.6899069091796875
+    # lies 0.929350 ulps (2^-11) above 0.689453125, up iff R13 >= 8192 * 0.070650 = 578.8
+    u, v, r = np.array([0], np.int32), np.array([0], np.int32), np.array([5.0], np.float32)
+    for t in range(6):
+        w = orc.sr_word(0, t, 0)
+        prob = orc.Problem(1, 1, 2, 0.005, 0.01, u, v, r, seed=0)
+        prob.set_factors(np.array([[2.37, 0.0]]), np.array([[2.09, 0.69]]))
+        prob.epoch_q16("serial", "none", sr=True, t=t)
+        q = prob.factors()[1][0]
+        assert q[0] == (2.08984375 + 2.0 ** -9 if (w & 0x1FFF) >= 6291 else 2.08984375)
+        assert q[1] == (0.689453125 + 2.0 ** -11 if ((w >> 16) & 0x1FFF) >= 579 else 0.689453125)
+    # every stored q is binary16; the SR epoch tracks the fp64 epoch within a few ulps; a
+    # different epoch counter gives different roundings
+    import synth
+    m, n, k = 30, 20, 8
+    u, v, r = synth.tiny(m, n, 300, seed=7)
+    rng = np.random.default_rng(5)
+    P0, Q0 = rng.uniform(0, 1, (m, k)), rng.uniform(0, 1, (n, k))
+    res = []
+    for t in (0, 1):
+        a = orc.Problem(m, n, k, 0.01, 0.05, u, v, r, G=1, Br=3, Bc=3, seed=9)
+        b = orc.Problem(m, n, k, 0.01, 0.05, u, v, r, G=1, Br=3, Bc=3, seed=9)
+        a.set_factors(P0, Q0)
+        b.set_factors(P0, Q0)
+        a.epoch("det", "none")
+        b.epoch_q16("det", "none", sr=True, t=t)
+        assert all(float(np.float16(x)) == x for x in b.Q.ravel())
+        assert 0 < np.abs(a.Q - b.Q).max() <= 8 * 2.0 ** -11 * np.abs(a.Q).max()
+        res.append(b.Q.copy())
+    assert not np.array_equal(res[0], res[1])
