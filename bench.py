@@ -34,6 +34,14 @@ import synth  # noqa: E402
 
 METRIC = "rating updates/sec (whole box)"
 STORAGE = {"fp32": 0, "fp16": 1, "fp16sr": 2}
+# what ncu says actually binds the SGD kernel (profiles/r01_ncu_c3_ring.md, C3): the
+# formula roofline above counts p_u / q_v bytes that stay in registers / L2
+BINDING = {
+    "fp32": {"unit": "L1TEX->XBAR request port (q_v load + vector red through L2)", "ncu_pct_of_peak": 71.1,
+             "dram_bytes_per_update": 17.1, "source": "profiles/r01_ncu_c3_ring.md"},
+    "fp16": {"unit": "issue / L2 latency (port at 39.8 %)", "ncu_pct_of_peak": 39.8,
+             "dram_bytes_per_update": 17.0, "source": "profiles/r01_ncu_c3_ring.md"},
+}
 UNIT = "updates/s"
 FALLBACK_HBM_GBS = 6650.0
 DEVICE_GEN_NNZ = 1_000_000_000
@@ -335,7 +343,8 @@ def main():
                 "kernel": "sgd_warp_kernel (a5/a6 epoch incl. Q sync%s)"
                           % ("" if storage == "fp32" else ", binary16 round-in/write-back of Q"),
                 "bytes_per_update": b_upd, "updates_per_launch": local_nnz, "kernel_ms": kmean,
-                "kernel_share_of_step": kmean / (ms / args.steps), "peak_source": peak_src}
+                "kernel_share_of_step": kmean / (ms / args.steps), "peak_source": peak_src,
+                "binding_unit": BINDING.get(storage)}
         return nnz * args.steps / (ms / 1e3), ms, roof, clk, curve + rms
 
     value, ms, roof, clk, curve = measure(args.storage)

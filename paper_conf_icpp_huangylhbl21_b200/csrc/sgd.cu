@@ -8,8 +8,9 @@
 // B200 design:
 //  * a "rating group" of L lanes owns one rating at a time; lane l holds VEC float4
 //    slots (elements (i*L + l)*4 ..) of p_u and q_v, so every factor access is a
-//    coalesced 128-bit load/store/red.  k = 128 -> L = 16, VEC = 2 (two groups per
-//    warp, lock step); the dot product is 4 FMA chains + log2(L) shuffles.
+//    coalesced 128-bit load/store/red.  k < 128: L = k/4 lanes, 32/L groups per warp in
+//    lock step; k = 128 j: one rating per warp (WarpSgd).  The dot product is two packed
+//    FFMA2 chains + log2(L) shuffles; all float4 arithmetic runs on the fp32x2 pipe.
 //  * a persistent grid pulls tasks (record ranges [lo, hi)) from an atomic queue.
 //    Hogwild tasks are runs of whole users, so p_u stays in registers across a
 //    user's ratings; DET tasks are the blocks of one stratum (no shared rows or
@@ -71,14 +72,25 @@ struct Lanes {
   }
 };
 
+// float4 arithmetic on the sm_100 packed fp32x2 pipe (FFMA2 / FMUL2 / FADD2: two IEEE fp32
+// operations per instruction, each correctly rounded as its scalar counterpart)
+__device__ __forceinline__ float2 lo2(float4 a) { return make_float2(a.x, a.y); }
+__device__ __forceinline__ float2 hi2(float4 a) { return make_float2(a.z, a.w); }
+__device__ __forceinline__ float4 cat2(float2 l, float2 h) { return make_float4(l.x, l.y, h.x, h.y); }
 __device__ __forceinline__ float4 f4_fma(float s, float4 a, float4 b) {  // s*a + b
-  return make_float4(fmaf(s, a.x, b.x), fmaf(s, a.y, b.y), fmaf(s, a.z, b.z), fmaf(s, a.w, b.w));
+  const float2 ss = make_float2(s, s);
+  return cat2(__ffma2_rn(ss, lo2(a), lo2(b)), __ffma2_rn(ss, hi2(a), hi2(b)));
 }
 __device__ __forceinline__ float4 f4_scale(float s, float4 a) {
-  return make_float4(s * a.x, s * a.y, s * a.z, s * a.w);
+  const float2 ss = make_float2(s, s);
+  return cat2(__fmul2_rn(ss, lo2(a)), __fmul2_rn(ss, hi2(a)));
 }
 __device__ __forceinline__ float4 f4_add(float4 a, float4 b) {
-  return make_float4(a.x + b.x, a.y + b.y, a.z + b.z, a.w + b.w);
+  return cat2(__fadd2_rn(lo2(a), lo2(b)), __fadd2_rn(hi2(a), hi2(b)));
+}
+// two fp32 dot-product chains (elements x,z and y,w): acc + a .* b, packed
+__device__ __forceinline__ float2 f4_dot2(float4 a, float4 b, float2 acc) {
+  return __ffma2_rn(hi2(a), hi2(b), __ffma2_rn(lo2(a), lo2(b), acc));
 }
 // four binary16 (two half2 words) <-> float4, round to nearest even (storage = 1)
 __device__ __forceinline__ uint2 f4_to_h4(float4 a) {
@@ -231,15 +243,10 @@ struct Group {
     if (newp) lanes.load(prow(nu), pn);
 
     // ---- e = r - p.q
-    float d0 = 0.f, d1 = 0.f, d2 = 0.f, d3 = 0.f;
+    float2 dd = make_float2(0.f, 0.f);
 #pragma unroll
-    for (int i = 0; i < VEC; ++i) {
-      d0 = fmaf(p.x[i].x, qc.x[i].x, d0);
-      d1 = fmaf(p.x[i].y, qc.x[i].y, d1);
-      d2 = fmaf(p.x[i].z, qc.x[i].z, d2);
-      d3 = fmaf(p.x[i].w, qc.x[i].w, d3);
-    }
-    float d = (d0 + d1) + (d2 + d3);
+    for (int i = 0; i < VEC; ++i) dd = f4_dot2(p.x[i], qc.x[i], dd);
+    float d = dd.x + dd.y;
 #pragma unroll
     for (int o = L / 2; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
 
@@ -466,15 +473,10 @@ struct WarpSgd {
       float4 qc[VEC];
 #pragma unroll
       for (int i = 0; i < VEC; ++i) qc[i] = widen<QH>(qc_raw[i]);
-      float d0 = 0.f, d1 = 0.f, d2 = 0.f, d3 = 0.f;
+      float2 dd = make_float2(0.f, 0.f);
 #pragma unroll
-      for (int i = 0; i < VEC; ++i) {
-        d0 = fmaf(p[i].x, qc[i].x, d0);
-        d1 = fmaf(p[i].y, qc[i].y, d1);
-        d2 = fmaf(p[i].z, qc[i].z, d2);
-        d3 = fmaf(p[i].w, qc[i].w, d3);
-      }
-      float d = (d0 + d1) + (d2 + d3);
+      for (int i = 0; i < VEC; ++i) dd = f4_dot2(p[i], qc[i], dd);
+      float d = dd.x + dd.y;
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
       const float ge = g * (cr - d);
@@ -593,15 +595,10 @@ struct WarpSgd {
         if (!fwd) ld(qrow(nv), qn);
         if (newp) ld(prow(nu), pn);
       }
-      float d0 = 0.f, d1 = 0.f, d2 = 0.f, d3 = 0.f;
+      float2 dd = make_float2(0.f, 0.f);
 #pragma unroll
-      for (int i = 0; i < VEC; ++i) {
-        d0 = fmaf(p[i].x, qc[i].x, d0);
-        d1 = fmaf(p[i].y, qc[i].y, d1);
-        d2 = fmaf(p[i].z, qc[i].z, d2);
-        d3 = fmaf(p[i].w, qc[i].w, d3);
-      }
-      float d = (d0 + d1) + (d2 + d3);
+      for (int i = 0; i < VEC; ++i) dd = f4_dot2(p[i], qc[i], dd);
+      float d = dd.x + dd.y;
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
       const float ge = g * (cr - d);
@@ -714,15 +711,10 @@ struct WarpSgd {
         const bool has_next = j + 1 < left;
         const bool newp = has_next && su[cn] != su[c];
         if (newp) ld(prow(su[cn]), pn);
-        float d0 = 0.f, d1 = 0.f, d2 = 0.f, d3 = 0.f;
+        float2 dd = make_float2(0.f, 0.f);
 #pragma unroll
-        for (int i = 0; i < VEC; ++i) {
-          d0 = fmaf(p[i].x, q[c][i].x, d0);
-          d1 = fmaf(p[i].y, q[c][i].y, d1);
-          d2 = fmaf(p[i].z, q[c][i].z, d2);
-          d3 = fmaf(p[i].w, q[c][i].w, d3);
-        }
-        float d = (d0 + d1) + (d2 + d3);
+        for (int i = 0; i < VEC; ++i) dd = f4_dot2(p[i], q[c][i], dd);
+        float d = dd.x + dd.y;
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
         const float ge = g * (sr[c] - d);
