@@ -393,10 +393,15 @@ void ring_group_cols(hccmf_t h, int sched, int g, int64_t* a, int64_t* b) {
   ring_cols(h->n, h->G, h->Br, h->Bc, sched, g, a, b);
 }
 
-hccmf_status wire_reserve(hccmf_t h, size_t halves) {  // send + recv staging, binary16
+hccmf_status wire_reserve(hccmf_t h, size_t halves, bool* grown = nullptr) {  // send + recv staging, binary16
   const size_t bytes = 2 * halves * 2;
+  if (grown) *grown = false;
   if (h->wire_bytes >= bytes) return HCCMF_OK;
-  if (h->d_wire) cudaFreeAsync(h->d_wire, h->stream);
+  if (grown) *grown = true;
+  if (h->d_wire) {  // the comm stream may still read the old staging buffer
+    if (h->comm_stream) CU(h, cudaStreamSynchronize(h->comm_stream));
+    cudaFreeAsync(h->d_wire, h->stream);
+  }
   h->d_wire = nullptr;
   h->wire_bytes = 0;
   CU(h, cudaMallocAsync(&h->d_wire, bytes, h->stream));
@@ -417,9 +422,12 @@ hccmf_status ring_transfer(hccmf_t h, int64_t sa, int64_t sb, int64_t ra, int64_
   }
   // Strategy 2: pack to binary16, ship half the bytes, unpack (all on the comm stream)
   const size_t cap = (size_t)h->n * h->k;
-  hccmf_status st = wire_reserve(h, cap);
+  bool grown = false;
+  hccmf_status st = wire_reserve(h, cap, &grown);
   if (st != HCCMF_OK) return st;
-  CU(h, cudaStreamSynchronize(h->stream));  // staging allocation ordered before its use on cs
+  // a new staging buffer (stream-ordered on the handle's stream) is ready before cs uses it;
+  // afterwards transfers never wait for the compute stream (hidden synchronisation)
+  if (grown && cs != h->stream) CU(h, cudaStreamSynchronize(h->stream));
   char* sendb = static_cast<char*>(h->d_wire);
   char* recvb = sendb + cap * 2;
   CU(h, k_pack_half(h->d_Q + sa * h->k, sendb, (int64_t)ns, cs));
