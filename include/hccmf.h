@@ -164,8 +164,12 @@ typedef enum {
     HCCMF_OPT_DET_WAVE = 9,      /* 1 (default): a single-shard DET epoch on a square
                                     grid runs as one wavefront kernel (warp i waits
                                     only for warp i+1's previous stratum) when the
-                                    B warps fit on the device; 0: one launch per
-                                    stratum.  Same update order either way.       */
+                                    B warps fit on the device, each column block's
+                                    Q rows staged in shared memory while a warp
+                                    holds it (when ceil(n/B) rows fit); 2: the
+                                    wavefront without the shared-memory slab; 0: one
+                                    launch per stratum.  Same update order and
+                                    bit-identical factors in every case.          */
     HCCMF_OPT_SYNC_PHASES = 10,  /* ALLREDUCE_AVG + HOGWILD: rounds per epoch (>= 1,
                                     default 1; must divide grid_rows).  Round ph runs
                                     every shard's row blocks [ph Br/S, (ph+1) Br/S)

@@ -591,7 +591,8 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
       h->opt_phases = value;
       return HCCMF_OK;
     case HCCMF_OPT_DET_WAVE:
-      h->opt_wave = value != 0;
+      if (value < 0 || value > 2) return fail(h, HCCMF_EINVAL, "det_wave must be 0, 1 or 2");
+      h->opt_wave = (int)value;
       return HCCMF_OK;
     case HCCMF_OPT_VEC:
       if (value != 0 && value != 1 && value != 2 && value != 4) return fail(h, HCCMF_EINVAL, "vec must be 0, 1, 2 or 4");
@@ -908,8 +909,10 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     if (L != 32 || L * VEC * 4 != h->k)
       return fail(h, HCCMF_EINVAL, "binary16 Q storage needs one rating per warp (k a multiple of 128, vec = k/128)");
   }
-  if (sched == HCCMF_SCHED_DET && G == 1 && h->opt_wave && h->storage == 0 && h->Br == h->Bc && h->Br > 1 &&
-      wave_supported(h->k, (int)h->opt_vec, h->Br)) {
+  const bool wave_slab = sched == HCCMF_SCHED_DET && G == 1 && h->opt_wave == 1 && h->storage == 0 &&
+                         h->Br == h->Bc && h->Br > 1 && wave_slab_supported(h->k, (int)h->opt_vec, h->Br, h->n);
+  if (wave_slab || (sched == HCCMF_SCHED_DET && G == 1 && h->opt_wave && h->storage == 0 && h->Br == h->Bc &&
+                    h->Br > 1 && wave_supported(h->k, (int)h->opt_vec, h->Br))) {
     // DET as one wavefront kernel: same order of updates as the strata (R19)
     SgdArgs a{};
     a.ru = h->d_u;
@@ -923,7 +926,10 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     a.lambda = h->lambda;
     a.vec_pref = (int32_t)h->opt_vec;
     a.prefetch = 1;
-    CU(h, launch_wave(a, h->d_blk_off, h->Br, h->d_progress, h->stream));
+    if (wave_slab)
+      CU(h, launch_wave_slab(a, h->d_blk_off, h->Br, h->d_progress, h->n, h->stream));
+    else
+      CU(h, launch_wave(a, h->d_blk_off, h->Br, h->d_progress, h->stream));
     ++h->epoch;
     return finish(h);
   }

@@ -77,6 +77,10 @@ cudaError_t launch_sgd(const SgdArgs& a, int64_t warps, cudaStream_t st);
 bool wave_supported(int k, int vec_pref, int B);
 cudaError_t launch_wave(const SgdArgs& a, const int64_t* off /* local block offsets, B*B+1 */, int B,
                         int* progress /* B ints */, cudaStream_t st);
+// the same wavefront with each column block's Q rows staged in shared memory
+bool wave_slab_supported(int k, int vec_pref, int B, int64_t n);
+cudaError_t launch_wave_slab(const SgdArgs& a, const int64_t* off, int B, int* progress, int64_t n,
+                             cudaStream_t st);
 // lane geometry of the SGD kernel: L lanes per rating group, VEC float4 per lane
 void sgd_geometry(int k, int vec_pref, int* L, int* VEC);
 int sgd_lanes(int k, int vec_pref);

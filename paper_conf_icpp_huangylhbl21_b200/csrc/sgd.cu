@@ -30,6 +30,9 @@
 
 #include <algorithm>
 #include <type_traits>
+#include <cstdio>
+#include <cstdlib>
+#include <vector>
 
 #include "internal.cuh"
 
@@ -302,6 +305,9 @@ __global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
 // every branch is warp-uniform and a task is a plain counted loop (no lock step, no
 // per-step liveness predicates).  Same pipeline as Group: rating j+1's record and
 // q row are in flight while rating j is updated.
+// DET slab wavefront: p_u copy distance (ratings) and ring slots (> distance, power of 2)
+constexpr int kSlabD = 12, kSlabRP = 16;
+
 template <int VEC, bool ATOMIC>
 struct WarpSgd {
   static constexpr unsigned FM = 0xffffffffu;
@@ -481,7 +487,7 @@ struct WarpSgd {
       for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
       const float ge = g * (cr - d);
       QR w[VEC];  // what is written: the increment (atomic) or the new row (store), as stored
-      QR snew[VEC];  // SR: the new row as stored
+      [[maybe_unused]] QR snew[VEC];  // SR: the new row as stored
 #pragma unroll
       for (int i = 0; i < VEC; ++i) {
         if constexpr (SR) {
@@ -652,6 +658,119 @@ struct WarpSgd {
     }
   }
 
+  // DET block with the column block's Q rows resident in shared memory (slab = this
+  // warp's copy of rows [c0, c0 + w), lane's slot 0 of row v at slab[(v - c0) k4 + lane]).
+  // Nothing else touches those rows while the warp holds the block (disjoint columns
+  // within a stratum), so q_v never leaves the SM during the block: every update reads
+  // the row from shared memory after the previous update's write (the serial order,
+  // duplicates included).  Nothing else touches the block's rows either (the warp owns
+  // its row block), and a row's ratings are contiguous in a block (sorted by u'), so the
+  // p_u row of every user run is copied D ratings ahead (cp.async, one commit group per
+  // rating, wait_group D before use) into a shared-memory ring of RP row slots and
+  // written back to HBM when the run ends; a run's row was last written by this warp,
+  // before the fence of an earlier block.  Same arithmetic as run() and run_ring(): the
+  // factors are bit-identical to the per-stratum launches.
+  __device__ __forceinline__ void run_slab(int64_t lo, int left, float4* slab, int c0, float4* pring) {
+    constexpr int D = kSlabD, RP = kSlabRP;
+    static_assert(RP > D && (RP & (RP - 1)) == 0, "ring");
+    const int32_t* ru = a.ru + lo;
+    const int32_t* rv = a.rv + lo;
+    const float* rr = a.rr + lo;
+    int wu0 = 0, wv0 = 0, wu1 = 0, wv1 = 0;
+    float wr0 = 0.f, wr1 = 0.f;
+    if (lane < left) wu0 = __ldcs(ru + lane), wv0 = __ldcs(rv + lane), wr0 = __ldcs(rr + lane);
+    if (lane + 32 < left) wu1 = __ldcs(ru + 32 + lane), wv1 = __ldcs(rv + 32 + lane), wr1 = __ldcs(rr + 32 + lane);
+    if (lane + 32 < left) prefetch_p(wu1);  // window 0: the kernel's look-ahead did it
+    int wb = 0;
+    float4* const sb = slab + lane - (int64_t)c0 * k4;
+    float4* const pb = pring + lane;
+    auto copy_p = [&](int slot, int u) {  // p_u -> ring slot (this lane's VEC 16-byte pieces)
+      const float4* src = prow(u);
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) {
+        const unsigned d = (unsigned)__cvta_generic_to_shared(pb + slot * k4 + 32 * i);
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(src + 32 * i) : "memory");
+      }
+    };
+    // record of rating jn (jn - wb < 64), from the two windows
+    auto rec = [&](int jn, int& u, int& v, float& r) {
+      const int src = jn - wb;
+      const bool w1 = src >= 32;
+      u = __shfl_sync(FM, w1 ? wu1 : wu0, src & 31);
+      v = __shfl_sync(FM, w1 ? wv1 : wv0, src & 31);
+      r = __shfl_sync(FM, w1 ? wr1 : wr0, src & 31);
+    };
+    // ratings 0 .. D-1 enter the ring; ring entries carry (u, new-run flag) in registers
+    // only for the rating being updated: the record is re-read from the window at use
+    int lastu = -1;
+    for (int s = 0; s < D; ++s) {
+      if (s < left) {
+        int u, v;
+        float r;
+        rec(s, u, v, r);
+        if (u != lastu) copy_p(s & (RP - 1), u);
+        lastu = u;
+      }
+      asm volatile("cp.async.commit_group;" ::: "memory");
+    }
+    int cu = -1;  // user whose row is in p
+    float4 p[VEC], q[VEC];
+    for (int j = 0; j < left; ++j) {
+      const int jn = j + D;
+      if (j - wb == 32) {  // window 0 consumed: slide; the new window 1 is needed ~20 ratings on
+        wu0 = wu1, wv0 = wv1, wr0 = wr1;
+        wb += 32;
+        const int idx = wb + 32 + lane;
+        if (idx < left) {
+          wu1 = __ldcs(ru + idx), wv1 = __ldcs(rv + idx), wr1 = __ldcs(rr + idx);
+          prefetch_p(wu1);
+        }
+      }
+      if (jn < left) {
+        int u, v;
+        float r;
+        rec(jn, u, v, r);
+        if (u != lastu) copy_p(jn & (RP - 1), u);
+        lastu = u;
+      }
+      asm volatile("cp.async.commit_group;" ::: "memory");
+      int u, v;
+      float r;
+      rec(j, u, v, r);
+      asm volatile("cp.async.wait_group %0;" ::"n"(D) : "memory");  // rating j's copy has landed
+      if (u != cu) {  // a run starts: retire the previous user's row, take this one's
+        if (cu >= 0) st(prow(cu), p);
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) p[i] = pb[(j & (RP - 1)) * k4 + 32 * i];
+        cu = u;
+      }
+      float4* qw = sb + v * k4;
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) q[i] = qw[32 * i];  // after the previous write: serial order
+      float2 dd = make_float2(0.f, 0.f);
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) dd = f4_dot2(p[i], q[i], dd);
+      float d = dd.x + dd.y;
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
+      const float ge = g * (r - d);
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) {
+        const float4 dq = f4_fma(ge, p[i], f4_scale(ngl, q[i]));
+        p[i] = f4_fma(ge, q[i], f4_scale(c1, p[i]));
+        qw[32 * i] = f4_add(q[i], dq);
+      }
+    }
+    st(prow(cu), p);
+    asm volatile("cp.async.wait_group 0;" ::: "memory");  // nothing may still target the ring
+  }
+  // L2 prefetch of one p_u row by the calling lane, line by line (a bulk prefetch takes a
+  // uniform operand: one per lane would be a 32-way serialised loop)
+  __device__ __forceinline__ void prefetch_p(int u) const {
+    const char* pr = reinterpret_cast<const char*>(reinterpret_cast<const float4*>(a.P) + (int64_t)(u - a.row0) * k4);
+    for (int o = 0; o < k4 * 16; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(pr + o));
+  }
+
   // Deeper pipeline (D >= 2, Hogwild): the q row of rating j + D is requested while
   // rating j is updated, from a ring of D + 1 register rows (the loop is unrolled
   // D + 1 times so every slot index is static).  Every pending row whose load was
@@ -795,7 +914,6 @@ __global__ void __launch_bounds__(kThreads, (VEC == 1 ? 4 : HCCMF_WARP_MINB)) sg
 template <int VEC>
 __global__ void __launch_bounds__(kThreads) sgd_wave_kernel(SgdArgs a, const int64_t* __restrict__ off, int B,
                                                             int* progress) {
-  constexpr unsigned FM = 0xffffffffu;
   const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
   if (i >= B) return;
   WarpSgd<VEC, false> w(a);
@@ -805,9 +923,12 @@ __global__ void __launch_bounds__(kThreads) sgd_wave_kernel(SgdArgs a, const int
       if (w.lane == 0) {
         int seen;
         do {
-          asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + nb) : "memory");
+          // relaxed polling (an acquire load per poll invalidates the SM's L1 every
+          // time: CCTL.IVALL), one acquire fence once the predecessor is seen
+          asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + nb) : "memory");
           if (seen < t) __nanosleep(64);
         } while (seen < t);
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
       }
       __syncwarp();
     }
@@ -816,8 +937,121 @@ __global__ void __launch_bounds__(kThreads) sgd_wave_kernel(SgdArgs a, const int
     if (hi > lo) w.run(lo, (int)(hi - lo));
     __syncwarp();
     if (w.lane == 0) {
-      __threadfence();
-      asm volatile("st.release.gpu.global.s32 [%0], %1;" ::"l"(progress + i), "r"(t + 1) : "memory");
+      asm volatile("fence.acq_rel.gpu;" ::: "memory");  // the warp's writes (ordered by __syncwarp) first
+      asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(progress + i), "r"(t + 1) : "memory");
+    }
+  }
+}
+
+// The same wavefront with the column block's Q rows staged in shared memory
+// (WarpSgd::run_slab): per block, the w <= wmax rows of column block c are copied in
+// with cp.async (one L2 round trip for the whole slab instead of one per rating),
+// updated in place, and written back before the progress counter is released.  The
+// next block's records are bulk-prefetched into L2 while this block runs.
+// Column block c holds v' with floor(v' B / n) = c, i.e. v' in [ceil(c n / B), ceil((c+1) n / B)).
+#ifdef HCCMF_DIAG_TRACE  // diagnostic builds only: %globaltimer stamps per (warp, stratum)
+__device__ unsigned g_wave_trace[2048 * 2048 * 3];
+__device__ __forceinline__ unsigned gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return (unsigned)t;
+}
+#endif
+
+template <int VEC>
+__global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, const int64_t* __restrict__ off, int B,
+                                                                 int* progress, int64_t n, int wmax) {
+  extern __shared__ float4 wave_smem[];
+  const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+  if (i >= B) return;
+  WarpSgd<VEC, false> w(a);
+  const int k4 = a.k >> 2;
+  // per warp: the column block's slab (wmax rows), then the p_u ring (kSlabRP rows)
+  float4* slab = wave_smem + (int64_t)(threadIdx.x >> 5) * (wmax + kSlabRP) * k4;
+  float4* pring = slab + (int64_t)wmax * k4;
+  const float4* Qg = reinterpret_cast<const float4*>(a.Q);
+  float4* Qw = reinterpret_cast<float4*>(a.Q);
+  const int nb = (i + 1) % B;
+  auto prefetch_records = [&](int64_t lo, int64_t hi) {
+    if (hi <= lo || w.lane > 2) return;
+    const char* base = w.lane == 0 ? reinterpret_cast<const char*>(a.ru)
+                                   : (w.lane == 1 ? reinterpret_cast<const char*>(a.rv)
+                                                  : reinterpret_cast<const char*>(a.rr));
+    const uintptr_t b0 = reinterpret_cast<uintptr_t>(base + 4 * lo) & ~(uintptr_t)15;
+    const uintptr_t b1 = (reinterpret_cast<uintptr_t>(base + 4 * hi) + 15) & ~(uintptr_t)15;
+    const unsigned bytes = (unsigned)min((uintptr_t)(1u << 20), b1 - b0);
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(b0), "r"(bytes) : "memory");
+  };
+  const int64_t* row_off = off + (int64_t)i * B;  // block (i, c) = row_off[c] .. row_off[c + 1]
+  prefetch_records(row_off[i], row_off[i + 1]);
+  if (B > 1) prefetch_records(row_off[(i + 1) % B], row_off[(i + 1) % B + 1]);
+  for (int t = 0; t < B; ++t) {
+    const int c = (i + t) % B;
+    const int64_t lo = row_off[c], hi = row_off[c + 1];
+    // look-ahead while the predecessor finishes: block t+2's records into L2, and the p_u
+    // rows of block t+1's first 64 ratings (its records are in L2 since the last block)
+    if (t + 2 < B) {
+      const int c2 = (i + t + 2) % B;
+      prefetch_records(row_off[c2], row_off[c2 + 1]);
+    }
+    int nu0 = -1, nu1 = -1;
+    if (t + 1 < B) {
+      const int c1n = (i + t + 1) % B;
+      const int64_t nlo = row_off[c1n], nn = row_off[c1n + 1] - nlo;
+      if (w.lane < nn) nu0 = __ldcg(a.ru + nlo + w.lane);
+      if (w.lane + 32 < nn) nu1 = __ldcg(a.ru + nlo + 32 + w.lane);
+    }
+#ifdef HCCMF_DIAG_TRACE
+    if (w.lane == 0 && B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3] = gtimer();
+#endif
+#ifndef HCCMF_DIAG_NOWAIT  // diagnostic builds only: no dependency waits (wrong factors, timing bound)
+    if (t > 0 && B > 1) {
+      if (w.lane == 0) {
+        int seen;
+        do {
+          // relaxed polling (an acquire load per poll invalidates the SM's L1 every
+          // time: CCTL.IVALL), one acquire fence once the predecessor is seen
+          asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + nb) : "memory");
+          if (seen < t) __nanosleep(64);
+        } while (seen < t);
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      }
+      __syncwarp();
+    }
+#endif
+#ifdef HCCMF_DIAG_TRACE
+    if (w.lane == 0 && B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3 + 1] = gtimer();
+#endif
+    if (nu0 >= 0) w.prefetch_p(nu0);
+    if (nu1 >= 0) w.prefetch_p(nu1);
+    if (hi > lo) {
+      const int c0 = (int)(((int64_t)c * n + B - 1) / B);
+      const int c1 = (int)(((int64_t)(c + 1) * n + B - 1) / B);
+      const int rows = c1 - c0;
+      for (int r = 0; r < rows; ++r) {
+#pragma unroll
+        for (int s = 0; s < VEC; ++s) {
+          const unsigned d = (unsigned)__cvta_generic_to_shared(slab + r * k4 + w.lane + 32 * s);
+          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d),
+                       "l"(Qg + (int64_t)(c0 + r) * k4 + w.lane + 32 * s)
+                       : "memory");
+        }
+      }
+      asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+      w.run_slab(lo, (int)(hi - lo), slab, c0, pring);
+      for (int r = 0; r < rows; ++r) {
+#pragma unroll
+        for (int s = 0; s < VEC; ++s)
+          __stcg(Qw + (int64_t)(c0 + r) * k4 + w.lane + 32 * s, slab[r * k4 + w.lane + 32 * s]);
+      }
+    }
+    __syncwarp();
+    if (w.lane == 0) {
+      asm volatile("fence.acq_rel.gpu;" ::: "memory");  // the warp's writes (ordered by __syncwarp) first
+      asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(progress + i), "r"(t + 1) : "memory");
+#ifdef HCCMF_DIAG_TRACE
+      if (B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3 + 2] = gtimer();
+#endif
     }
   }
 }
@@ -926,6 +1160,85 @@ cudaError_t launch_wave(const SgdArgs& a, const int64_t* off, int B, int* progre
     case 4: sgd_wave_kernel<4><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress); break;
     default: return cudaErrorInvalidValue;
   }
+  return cudaGetLastError();
+}
+
+namespace {
+// slab wavefront geometry: warps per CTA and dynamic shared memory, or false if the
+// column blocks' rows do not fit or the B warps cannot all be co-resident
+template <int VEC>
+bool slab_geometry_t(int k, int B, int64_t n, int* wpc_out, size_t* smem_out) {
+  const int64_t wmax = (n + B - 1) / B;
+  const size_t per_warp = (size_t)(wmax + kSlabRP) * k * sizeof(float);
+  constexpr size_t kBudget = 160 * 1024;
+  int wpc = kThreads / 32;
+  while (wpc > 1 && wpc * per_warp > kBudget) wpc >>= 1;
+  if (wpc * per_warp > kBudget) return false;
+  const size_t smem = wpc * per_warp;
+  if (cudaFuncSetAttribute(sgd_wave_slab_kernel<VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+      cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  int dev = 0, sms = 0, per_sm = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sgd_wave_slab_kernel<VEC>, wpc * 32, smem) !=
+      cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  // co-residency (every warp waits on its successor) with 10 % head room
+  if ((int64_t)B * 10 > (int64_t)sms * per_sm * wpc * 9) return false;
+  *wpc_out = wpc;
+  *smem_out = smem;
+  return true;
+}
+}  // namespace
+
+bool wave_slab_supported(int k, int vec_pref, int B, int64_t n) {
+  int L, VEC, wpc;
+  size_t smem;
+  sgd_geometry(k, vec_pref, &L, &VEC);
+  if (L != 32 || L * VEC * 4 != k) return false;
+  switch (VEC) {
+    case 1: return slab_geometry_t<1>(k, B, n, &wpc, &smem);
+    case 2: return slab_geometry_t<2>(k, B, n, &wpc, &smem);
+    case 4: return slab_geometry_t<4>(k, B, n, &wpc, &smem);
+    default: return false;
+  }
+}
+
+cudaError_t launch_wave_slab(const SgdArgs& a, const int64_t* off, int B, int* progress, int64_t n, cudaStream_t st) {
+  int L, VEC, wpc = 0;
+  size_t smem = 0;
+  sgd_geometry(a.k, a.vec_pref, &L, &VEC);
+  cudaError_t e = cudaMemsetAsync(progress, 0, sizeof(int) * B, st);
+  if (e != cudaSuccess) return e;
+  const int wmax = (int)((n + B - 1) / B);
+#define SLAB_CASE(V)                                                                                        \
+  case V:                                                                                                   \
+    if (!slab_geometry_t<V>(a.k, B, n, &wpc, &smem)) return cudaErrorInvalidConfiguration;                 \
+    sgd_wave_slab_kernel<V><<<(unsigned)((B + wpc - 1) / wpc), wpc * 32, smem, st>>>(a, off, B, progress, n, wmax); \
+    break;
+  switch (VEC) {
+    SLAB_CASE(1)
+    SLAB_CASE(2)
+    SLAB_CASE(4)
+    default: return cudaErrorInvalidValue;
+  }
+#undef SLAB_CASE
+#ifdef HCCMF_DIAG_TRACE
+  if (const char* path = getenv("HCCMF_TRACE_OUT")) {
+    static std::vector<unsigned> host(2048 * 2048 * 3);
+    cudaStreamSynchronize(st);
+    cudaMemcpyFromSymbol(host.data(), g_wave_trace, sizeof(unsigned) * 3 * (size_t)B * B);
+    if (FILE* f = fopen(path, "wb")) {
+      fwrite(host.data(), sizeof(unsigned), 3 * (size_t)B * B, f);
+      fclose(f);
+    }
+  }
+#endif
   return cudaGetLastError();
 }
 

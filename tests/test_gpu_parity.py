@@ -305,18 +305,22 @@ def test_hogwild_logical_shards_band_c2(pkg, orc, sync, G, Bc):
     assert all(abs(g - want) <= 0.005 for g in got), (want, got)
 
 
-@pytest.mark.parametrize("k,B", [(128, 24), (256, 9)])
-def test_det_wavefront_equals_strata(pkg, orc, k, B):
-    # the wavefront kernel and the per-stratum launches apply the same updates in the
-    # same per-row / per-column order: bit-identical factors, and the oracle to 1e-4
+@pytest.mark.parametrize("k,B,dup", [(128, 24, False), (256, 9, False), (128, 37, True), (512, 5, True)])
+def test_det_wavefront_equals_strata(pkg, orc, k, B, dup):
+    # the wavefront kernels (Q slab in shared memory: det_wave 1; registers only: 2) and
+    # the per-stratum launches (0) apply the same updates in the same per-row /
+    # per-column order: bit-identical factors, and the oracle to 1e-4.  dup: every
+    # rating duplicated (serial read-after-write of q_v through the slab)
     cfg = synth.CONFIGS["c1"]
     (u, v, r), _ = synth.make(cfg)
+    if dup:
+        u, v, r = (np.concatenate([x[:20000], x[:20000]]) for x in (u, v, r))
     prob = orc.Problem(cfg.m, cfg.n, k, 0.02, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=6)
     prob.init(2)
     P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
     prob.set_factors(P0, Q0)
     outs = []
-    for wave in (1, 0):
+    for wave in (1, 2, 0):
         mdl = _gpu_problem(pkg, cfg.m, cfg.n, k, 0.02, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=6)
         mdl.set_option("det_wave", wave)
         mdl.set_factors(P0, Q0)
@@ -325,7 +329,8 @@ def test_det_wavefront_equals_strata(pkg, orc, k, B):
         outs.append(mdl.factors())
     for _ in range(2):
         prob.epoch("det", "none")
-    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+    for o in outs[1:]:
+        assert np.array_equal(outs[0][0], o[0]) and np.array_equal(outs[0][1], o[1])
     Po, Qo = prob.factors()
     assert max(np.abs(outs[0][0] - Po).max(), np.abs(outs[0][1] - Qo).max()) <= 1e-4
 
