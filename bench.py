@@ -42,6 +42,25 @@ BINDING = {
     "fp16": {"unit": "issue / L2 latency (port at 39.8 %)", "ncu_pct_of_peak": 39.8,
              "dram_bytes_per_update": 17.0, "source": "profiles/r01_ncu_c3_ring.md"},
 }
+PROBE = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "r01_probe_l2_roundtrip_c3.json")
+
+
+def binding_unit(storage, args, kernel_rate):
+    """The unit that bounds the SGD kernel (ncu) and, for the C3 Hogwild kernel, the
+    measured ceiling of its q_v round trip on this B200 (tools/probe_l2_roundtrip.py:
+    same record stream and warp count, no SGD arithmetic): the reductions alone for fp32
+    rows, load + reduction for binary16 rows."""
+    b = dict(BINDING.get("fp32" if storage == "fp32" else "fp16"))
+    if args.config == "c3" and args.sched == "hogwild" and os.path.exists(PROBE):
+        with open(PROBE) as f:
+            pr = json.load(f)
+        key = "red only fp32" if storage == "fp32" else "ld+red binary16 (256+256 B)"
+        ceil = pr[key]["G_upd_per_s"] * 1e9
+        b["ceiling"] = {"probe": key, "updates_per_s": ceil, "kernel_updates_per_s": kernel_rate,
+                        "frac": kernel_rate / ceil, "source": os.path.relpath(PROBE, os.path.dirname(PROBE) + "/..")}
+    return b
+
+
 UNIT = "updates/s"
 FALLBACK_HBM_GBS = 6650.0
 DEVICE_GEN_NNZ = 1_000_000_000
@@ -348,7 +367,7 @@ def main():
                           % ("" if storage == "fp32" else ", binary16 round-in/write-back of Q"),
                 "bytes_per_update": b_upd, "updates_per_launch": local_nnz, "kernel_ms": kmean,
                 "kernel_share_of_step": kmean / (ms / args.steps), "peak_source": peak_src,
-                "binding_unit": BINDING.get(storage)}
+                "binding_unit": binding_unit(storage, args, local_nnz / (kmean / 1e3))}
         return nnz * args.steps / (ms / 1e3), ms, roof, clk, curve + rms
 
     value, ms, roof, clk, curve = measure(args.storage)
