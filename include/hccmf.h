@@ -315,6 +315,12 @@ HCCMF_API hccmf_status hccmf_cost_model(int32_t p, int64_t m, int64_t n, int64_t
 /* Library version string, e.g. "hccmf 0.1 sm_100a". */
 HCCMF_API const char* hccmf_version(void);
 
+/* Process-wide count of the CUDA kernels this library has launched (every handle,
+ * every call; CUB's internal sort/scan/select launches in hccmf_partition are not
+ * counted).  Read it before and after a region to count that region's launches
+ * (bench.py's gpu_launches).  Never fails. */
+HCCMF_API int64_t hccmf_kernel_launches(void);
+
 #ifdef __cplusplus
 }
 #endif

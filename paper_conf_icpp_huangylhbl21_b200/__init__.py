@@ -92,6 +92,7 @@ def lib():
             "hccmf_get_fractions": (st, [P, P]),
             "hccmf_get_info": (st, [P, ctypes.POINTER(Info)]),
             "hccmf_version": (ctypes.c_char_p, []),
+            "hccmf_kernel_launches": (ctypes.c_int64, []),
             "hccmf_schedule": (st, [i32, i32, i32, i64, i32, i32, i32, P, P, P, P, P, P]),
             "hccmf_cost_model": (st, [i32, i64, i64, i64, i32, P, P, ctypes.c_double, i32, i32, i32,
                                       ctypes.c_double, P, P, P, P, P]),
@@ -102,6 +103,11 @@ def lib():
             fn.argtypes = args
         _lib = L
     return _lib
+
+
+def kernel_launches() -> int:
+    """Kernels the library has launched in this process (hccmf_kernel_launches)."""
+    return int(lib().hccmf_kernel_launches())
 
 
 def version() -> str:

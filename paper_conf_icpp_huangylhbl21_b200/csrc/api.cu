@@ -492,6 +492,8 @@ extern "C" {
 
 const char* hccmf_version(void) { return "hccmf 0.1 sm_100a"; }
 
+int64_t hccmf_kernel_launches(void) { return hccmf::g_kernel_launches.load(std::memory_order_relaxed); }
+
 const char* hccmf_last_error(hccmf_t h) { return h ? h->err.c_str() : g_err.c_str(); }
 
 hccmf_status hccmf_create(int64_t m, int64_t n, int32_t k, float gamma, float lambda, hccmf_t* out) {

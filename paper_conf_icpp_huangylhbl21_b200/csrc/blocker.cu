@@ -267,14 +267,14 @@ cudaError_t dalloc(T** p, size_t count, cudaStream_t st) {
 cudaError_t k_validate(const int32_t* u, const int32_t* v, const float* r, int64_t nnz, int64_t m, int64_t n,
                        unsigned int* flag, cudaStream_t st) {
   if (nnz == 0) return cudaSuccess;
-  validate_kernel<<<grid_for(nnz), kT, 0, st>>>(u, v, r, nnz, m, n, flag);
+  (note_launch(), validate_kernel<<<grid_for(nnz), kT, 0, st>>>(u, v, r, nnz, m, n, flag));
   return cudaGetLastError();
 }
 
 cudaError_t k_perm(uint64_t seed, uint64_t tag, int64_t count, int32_t* perm, cudaStream_t st) {
   if (count == 0) return cudaSuccess;
   if (seed == 0) {
-    iota_kernel<<<grid_for(count), kT, 0, st>>>(perm, count);
+    (note_launch(), iota_kernel<<<grid_for(count), kT, 0, st>>>(perm, count));
     return cudaGetLastError();
   }
   uint64_t *k0 = nullptr, *k1 = nullptr;
@@ -283,14 +283,14 @@ cudaError_t k_perm(uint64_t seed, uint64_t tag, int64_t count, int32_t* perm, cu
   CKR(dalloc(&k1, count, st));
   CKR(dalloc(&i0, count, st));
   CKR(dalloc(&i1, count, st));
-  perm_keys_kernel<<<grid_for(count), kT, 0, st>>>(seed, tag, count, k0, i0);
+  (note_launch(), perm_keys_kernel<<<grid_for(count), kT, 0, st>>>(seed, tag, count, k0, i0));
   CKR(cudaGetLastError());
   size_t tb = 0;
   void* tmp = nullptr;
   CKR(cub::DeviceRadixSort::SortPairs(nullptr, tb, k0, k1, i0, i1, count, 0, 64, st));
   CKR(cudaMallocAsync(&tmp, tb, st));
   CKR(cub::DeviceRadixSort::SortPairs(tmp, tb, k0, k1, i0, i1, count, 0, 64, st));
-  perm_scatter_kernel<<<grid_for(count), kT, 0, st>>>(i1, count, perm);
+  (note_launch(), perm_scatter_kernel<<<grid_for(count), kT, 0, st>>>(i1, count, perm));
   CKR(cudaGetLastError());
   cudaFreeAsync(tmp, st);
   cudaFreeAsync(k0, st);
@@ -306,7 +306,7 @@ cudaError_t k_row_prefix(const int32_t* u, int64_t nnz, const int32_t* perm_row,
   CKR(dalloc(&cnt, m + 1, st));
   CKR(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * (m + 1), st));
   if (nnz) {
-    row_count_kernel<<<grid_for(nnz), kT, 0, st>>>(u, nnz, perm_row, cnt);
+    (note_launch(), row_count_kernel<<<grid_for(nnz), kT, 0, st>>>(u, nnz, perm_row, cnt));
     CKR(cudaGetLastError());
   }
   size_t tb = 0;
@@ -322,7 +322,7 @@ cudaError_t k_row_prefix(const int32_t* u, int64_t nnz, const int32_t* perm_row,
 cudaError_t k_bound_search(const unsigned long long* S, int64_t m, const int64_t* targets, int32_t nt, int64_t* out,
                            cudaStream_t st) {
   if (nt <= 0) return cudaSuccess;
-  bound_search_kernel<<<(nt + 127) / 128, 128, 0, st>>>(S, m, targets, nt, out);
+  (note_launch(), bound_search_kernel<<<(nt + 127) / 128, 128, 0, st>>>(S, m, targets, nt, out));
   return cudaGetLastError();
 }
 
@@ -347,7 +347,7 @@ cudaError_t k_block_sort(const BlockGeom& g, const int32_t* bounds, const int32_
   CKR(dalloc(&k1, nnz, st));
   bs_mark(st, "bs: alloc keys");
   if (nnz) {
-    block_key_kernel<<<grid_for(nnz), kT, 0, st>>>(g, bounds, perm_row, perm_col, u, v, nnz, k0);
+    (note_launch(), block_key_kernel<<<grid_for(nnz), kT, 0, st>>>(g, bounds, perm_row, perm_col, u, v, nnz, k0));
     CKR(cudaGetLastError());
   }
   bs_mark(st, "bs: key kernel");
@@ -366,11 +366,11 @@ cudaError_t k_block_sort(const BlockGeom& g, const int32_t* bounds, const int32_
   }
   bs_mark(st, "bs: radix sort");
   if (nnz) {
-    block_decode_kernel<<<grid_for(nnz), kT, 0, st>>>(g, bounds, ks, nnz, ou, ov);
+    (note_launch(), block_decode_kernel<<<grid_for(nnz), kT, 0, st>>>(g, bounds, ks, nnz, ou, ov));
     CKR(cudaGetLastError());
   }
   bs_mark(st, "bs: decode");
-  block_off_kernel<<<grid_for(nblk + 1), kT, 0, st>>>(ks, nnz, g.bu + g.bv, nblk, block_off);
+  (note_launch(), block_off_kernel<<<grid_for(nblk + 1), kT, 0, st>>>(ks, nnz, g.bu + g.bv, nblk, block_off));
   CKR(cudaGetLastError());
   cudaFreeAsync(k0, st);
   cudaFreeAsync(k1, st);
@@ -393,8 +393,8 @@ cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, i
   CKR(dalloc(&flag, nrec, st));
   CKR(dalloc(&runs, nrec, st));
   CKR(dalloc(&nsel, 1, st));
-  run_flag_kernel<<<grid_for(nrec), kT, 0, st>>>(ru, nrec, flag);
-  block_start_flag_kernel<<<grid_for(nb), kT, 0, st>>>(off, nb, nrec, flag);
+  (note_launch(), run_flag_kernel<<<grid_for(nrec), kT, 0, st>>>(ru, nrec, flag));
+  (note_launch(), block_start_flag_kernel<<<grid_for(nb), kT, 0, st>>>(off, nb, nrec, flag));
   CKR(cudaGetLastError());
   size_t tb = 0;
   void* tmp = nullptr;
@@ -412,7 +412,7 @@ cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, i
   CKR(dalloc(&ccnt, nb + 1, st));
   CKR(dalloc(&coff, nb + 1, st));
   CKR(cudaMemsetAsync(ccnt, 0, sizeof(int64_t) * (nb + 1), st));
-  cand_count_kernel<<<grid_for(nb), kT, 0, st>>>(off, nb, target, ccnt);
+  (note_launch(), cand_count_kernel<<<grid_for(nb), kT, 0, st>>>(off, nb, target, ccnt));
   CKR(cudaGetLastError());
   tb = 0;
   CKR(cub::DeviceScan::ExclusiveSum(nullptr, tb, ccnt, coff, nb + 1, st));
@@ -429,7 +429,7 @@ cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, i
   CKR(dalloc(&cpos, ncand, st));
   CKR(dalloc(&keep, ncand, st));
   CKR(dalloc(&lo, ncand, st));
-  cand_map_kernel<<<grid_for(ncand), kT, 0, st>>>(coff, nb, ncand, off, target, runs, nruns, cpos, keep);
+  (note_launch(), cand_map_kernel<<<grid_for(ncand), kT, 0, st>>>(coff, nb, ncand, off, target, runs, nruns, cpos, keep));
   CKR(cudaGetLastError());
   tb = 0;
   CKR(cub::DeviceSelect::Flagged(nullptr, tb, cpos, keep, lo, nsel, ncand, st));
@@ -448,7 +448,7 @@ cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, i
   CKR(dalloc(&sk1, nt, st));
   CKR(dalloc(&ix0, nt, st));
   CKR(dalloc(&ix1, nt, st));
-  task_hi_kernel<<<grid_for(nt), kT, 0, st>>>(lo, nt, off, nb, heavy, hi, sk0, ix0);
+  (note_launch(), task_hi_kernel<<<grid_for(nt), kT, 0, st>>>(lo, nt, off, nb, heavy, hi, sk0, ix0));
   CKR(cudaGetLastError());
   tb = 0;
   CKR(cub::DeviceRadixSort::SortPairs(nullptr, tb, sk0, sk1, ix0, ix1, nt, 0, 64, st));
@@ -457,7 +457,7 @@ cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, i
   cudaFreeAsync(tmp, st);
   CKR(cudaMallocAsync((void**)task_lo, sizeof(int64_t) * (nt ? nt : 1), st));
   CKR(cudaMallocAsync((void**)task_hi, sizeof(int64_t) * (nt ? nt : 1), st));
-  permute_tasks_kernel<<<grid_for(nt), kT, 0, st>>>(ix1, nt, lo, hi, *task_lo, *task_hi);
+  (note_launch(), permute_tasks_kernel<<<grid_for(nt), kT, 0, st>>>(ix1, nt, lo, hi, *task_lo, *task_hi));
   CKR(cudaGetLastError());
   for (void* p : {(void*)flag, (void*)runs, (void*)nsel, (void*)ccnt, (void*)coff, (void*)cpos, (void*)keep,
                   (void*)lo, (void*)hi, (void*)sk0, (void*)sk1, (void*)ix0, (void*)ix1})

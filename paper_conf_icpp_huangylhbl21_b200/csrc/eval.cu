@@ -161,44 +161,44 @@ __global__ void average_half_kernel(const float* reps, int32_t G, int64_t count,
 
 cudaError_t k_round_half(float* x, int64_t count, cudaStream_t st) {
   if (count <= 0) return cudaSuccess;
-  round_half_kernel<<<grid_for(count), kT, 0, st>>>(x, count);
+  (note_launch(), round_half_kernel<<<grid_for(count), kT, 0, st>>>(x, count));
   return cudaGetLastError();
 }
 cudaError_t k_pack_half(const float* x, void* y, int64_t count, cudaStream_t st) {
   if (count <= 0) return cudaSuccess;
-  pack_half_kernel<<<grid_for(count), kT, 0, st>>>(x, reinterpret_cast<__half*>(y), count);
+  (note_launch(), pack_half_kernel<<<grid_for(count), kT, 0, st>>>(x, reinterpret_cast<__half*>(y), count));
   return cudaGetLastError();
 }
 cudaError_t k_unpack_half(const void* y, float* x, int64_t count, cudaStream_t st) {
   if (count <= 0) return cudaSuccess;
-  unpack_half_kernel<<<grid_for(count), kT, 0, st>>>(reinterpret_cast<const __half*>(y), x, count);
+  (note_launch(), unpack_half_kernel<<<grid_for(count), kT, 0, st>>>(reinterpret_cast<const __half*>(y), x, count));
   return cudaGetLastError();
 }
 cudaError_t k_average_half(const float* reps, int32_t G, int64_t count, float* out, cudaStream_t st) {
-  average_half_kernel<<<grid_for(count), kT, 0, st>>>(reps, G, count, out);
+  (note_launch(), average_half_kernel<<<grid_for(count), kT, 0, st>>>(reps, G, count, out));
   return cudaGetLastError();
 }
 
 cudaError_t k_init_factors(uint64_t seed, uint64_t tag, int64_t rows_total, int32_t k, const int32_t* perm,
                            int64_t row0, int64_t rows, float* X, cudaStream_t st) {
   if (rows_total == 0) return cudaSuccess;
-  init_kernel<<<grid_for(rows_total * k), kT, 0, st>>>(seed, tag, rows_total, k, perm, row0, rows, X);
+  (note_launch(), init_kernel<<<grid_for(rows_total * k), kT, 0, st>>>(seed, tag, rows_total, k, perm, row0, rows, X));
   return cudaGetLastError();
 }
 
 cudaError_t k_scatter_rows(const float* src, int64_t rows_total, int32_t k, const int32_t* perm, int64_t row0,
                            int64_t rows, float* dst, cudaStream_t st) {
   const int32_t k4 = k / 4;
-  scatter_kernel<<<grid_for(rows_total * k4), kT, 0, st>>>(reinterpret_cast<const float4*>(src), rows_total, k4,
-                                                           perm, row0, rows, reinterpret_cast<float4*>(dst));
+  (note_launch(), scatter_kernel<<<grid_for(rows_total * k4), kT, 0, st>>>(reinterpret_cast<const float4*>(src), rows_total, k4,
+                                                           perm, row0, rows, reinterpret_cast<float4*>(dst)));
   return cudaGetLastError();
 }
 
 cudaError_t k_gather_rows(const float* src, int64_t rows_total, int32_t k, const int32_t* perm, int64_t row0,
                           float* dst, cudaStream_t st) {
   const int32_t k4 = k / 4;
-  gather_kernel<<<grid_for(rows_total * k4), kT, 0, st>>>(reinterpret_cast<const float4*>(src), rows_total, k4, perm,
-                                                          row0, reinterpret_cast<float4*>(dst));
+  (note_launch(), gather_kernel<<<grid_for(rows_total * k4), kT, 0, st>>>(reinterpret_cast<const float4*>(src), rows_total, k4, perm,
+                                                          row0, reinterpret_cast<float4*>(dst)));
   return cudaGetLastError();
 }
 
@@ -209,18 +209,18 @@ cudaError_t k_rmse(const int32_t* tu, const int32_t* tv, const float* tr, int64_
   switch (L) {
 #define RM(LL)                                                                                                    \
   case LL:                                                                                                        \
-    rmse_kernel<LL><<<RMSE_BLOCKS, kT, 0, st>>>(tu, tv, tr, nt, perm_row, perm_col, P, row0, rows, Q, k, partials); \
+    (note_launch(), rmse_kernel<LL><<<RMSE_BLOCKS, kT, 0, st>>>(tu, tv, tr, nt, perm_row, perm_col, P, row0, rows, Q, k, partials)); \
     break;
     RM(1) RM(2) RM(4) RM(8) RM(16) RM(32)
 #undef RM
     default: return cudaErrorInvalidValue;
   }
-  rmse_final_kernel<<<1, 32, 0, st>>>(partials, RMSE_BLOCKS, out2);
+  (note_launch(), rmse_final_kernel<<<1, 32, 0, st>>>(partials, RMSE_BLOCKS, out2));
   return cudaGetLastError();
 }
 
 cudaError_t k_average(const float* reps, int32_t G, int64_t count, float* out, cudaStream_t st) {
-  average_kernel<<<grid_for(count), kT, 0, st>>>(reps, G, count, out);
+  (note_launch(), average_kernel<<<grid_for(count), kT, 0, st>>>(reps, G, count, out));
   return cudaGetLastError();
 }
 

@@ -5,12 +5,18 @@
 #include <nccl.h>
 #include <stdint.h>
 
+#include <atomic>
 #include <string>
 #include <vector>
 
 #include "hccmf.h"
 
 namespace hccmf {
+
+// every <<<...>>> launch site of the library is written (note_launch(), kernel<<<...>>>(...))
+// so hccmf_kernel_launches() reports what actually ran (bench.py's gpu_launches)
+inline std::atomic<long long> g_kernel_launches{0};
+inline void note_launch() { g_kernel_launches.fetch_add(1, std::memory_order_relaxed); }
 
 // ------------------------------------------------------------------ hashing
 // DESIGN.md R8: SplitMix64 finaliser (Steele, Lea, Flood 2014) and the

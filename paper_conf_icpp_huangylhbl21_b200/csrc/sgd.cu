@@ -1070,9 +1070,9 @@ cudaError_t launch_t(const SgdArgs& a, int64_t warps, cudaStream_t st) {
 #define WARP_CASE(DD, QQ)                                                     \
   if (depth == DD && a.qhalf == QQ) {                                         \
     if (a.atomic_q)                                                           \
-      sgd_warp_kernel<VEC, true, DD, QQ><<<(unsigned)blocks, threads, 0, st>>>(a);  \
+      (note_launch(), sgd_warp_kernel<VEC, true, DD, QQ><<<(unsigned)blocks, threads, 0, st>>>(a));  \
     else                                                                      \
-      sgd_warp_kernel<VEC, false, DD, QQ><<<(unsigned)blocks, threads, 0, st>>>(a); \
+      (note_launch(), sgd_warp_kernel<VEC, false, DD, QQ><<<(unsigned)blocks, threads, 0, st>>>(a)); \
     return cudaGetLastError();                                                \
   }
     WARP_CASE(1, 0) WARP_CASE(2, 0) WARP_CASE(3, 0) WARP_CASE(4, 0) WARP_CASE(1, 1) WARP_CASE(1, 2)
@@ -1081,9 +1081,9 @@ cudaError_t launch_t(const SgdArgs& a, int64_t warps, cudaStream_t st) {
   }
   if (a.qhalf) return cudaErrorInvalidValue;  // binary16 Q: warp-per-rating geometry only
   if (a.atomic_q)
-    sgd_kernel<L, VEC, FULL, true><<<(unsigned)blocks, threads, 0, st>>>(a);
+    (note_launch(), sgd_kernel<L, VEC, FULL, true><<<(unsigned)blocks, threads, 0, st>>>(a));
   else
-    sgd_kernel<L, VEC, FULL, false><<<(unsigned)blocks, threads, 0, st>>>(a);
+    (note_launch(), sgd_kernel<L, VEC, FULL, false><<<(unsigned)blocks, threads, 0, st>>>(a));
   return cudaGetLastError();
 }
 
@@ -1155,9 +1155,9 @@ cudaError_t launch_wave(const SgdArgs& a, const int64_t* off, int B, int* progre
   if (e != cudaSuccess) return e;
   const int64_t blocks = ((int64_t)B * 32 + kThreads - 1) / kThreads;
   switch (VEC) {
-    case 1: sgd_wave_kernel<1><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress); break;
-    case 2: sgd_wave_kernel<2><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress); break;
-    case 4: sgd_wave_kernel<4><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress); break;
+    case 1: (note_launch(), sgd_wave_kernel<1><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress)); break;
+    case 2: (note_launch(), sgd_wave_kernel<2><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress)); break;
+    case 4: (note_launch(), sgd_wave_kernel<4><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress)); break;
     default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();
@@ -1219,7 +1219,7 @@ cudaError_t launch_wave_slab(const SgdArgs& a, const int64_t* off, int B, int* p
 #define SLAB_CASE(V)                                                                                        \
   case V:                                                                                                   \
     if (!slab_geometry_t<V>(a.k, B, n, &wpc, &smem)) return cudaErrorInvalidConfiguration;                 \
-    sgd_wave_slab_kernel<V><<<(unsigned)((B + wpc - 1) / wpc), wpc * 32, smem, st>>>(a, off, B, progress, n, wmax); \
+    (note_launch(), sgd_wave_slab_kernel<V><<<(unsigned)((B + wpc - 1) / wpc), wpc * 32, smem, st>>>(a, off, B, progress, n, wmax)); \
     break;
   switch (VEC) {
     SLAB_CASE(1)
