@@ -119,3 +119,26 @@ def test_c5_full_size_properties(pkg):
     mdl.train_epoch("hogwild", "none")
     r1 = mdl.rmse(tu, tv, tr)
     assert np.isfinite(r1) and r1 < r0
+
+
+def test_c3_det_epoch_full_size(pkg, c3):
+    # bench.py --sched det --grid 2048,2048: one DET epoch on the full C3 problem runs as
+    # ONE wavefront kernel (shared-memory Q slabs) and matches the serial fp64 oracle on
+    # sampled rows (the heaviest users and items included) to 1e-4 (SURVEY 8(c) bar)
+    path = os.path.join(GOLDEN, "oracle_det_c3_B2048.npz")
+    if not os.path.exists(path):
+        pytest.skip("tools/oracle_curves.py det:c3:2048 not run")
+    ref = np.load(path)
+    cfg = synth.CONFIGS["c3"]
+    (u, v, r), _ = c3
+    mdl = pkg.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam)
+    mdl.load(u, v, r)
+    mdl.partition(1, (2048, 2048), seed=cfg.seed)
+    mdl.init(1)
+    l0 = pkg.kernel_launches()
+    mdl.train_epoch("det", "none")
+    assert pkg.kernel_launches() - l0 == 1
+    P, Q = mdl.factors()
+    mdl.close()
+    assert np.abs(P[ref["users"]] - ref["P"]).max() <= 1e-4
+    assert np.abs(Q[ref["items"]] - ref["Q"]).max() <= 1e-4

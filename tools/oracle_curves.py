@@ -7,6 +7,8 @@ first epoch whose GPU test RMSE <= oracle RMSE@E + 0.005).  Settings mirror benc
 one shard, grid (1, 1), shuffle seed = config seed, init seed 1, serial order.
 
     python tools/oracle_curves.py c1 c2 c3      # C3: ~4 min on one core
+    python tools/oracle_curves.py c3:2048        # digest of the 2048 x 2048 DET partition
+    python tools/oracle_curves.py det:c3:2048    # sampled P, Q rows after one DET epoch
 """
 import hashlib
 import json
@@ -45,8 +47,41 @@ def det_digest(name, B):
     print(name, B, out[f"partition_sha256_grid_{B}x{B}"], flush=True)
 
 
+def det_epoch_sample(name, B, rows=128):
+    """One DET epoch (B x B grid, the bench's DET configuration: shuffle seed = config
+    seed, init seed 1) by the oracle; stores `rows` sampled rows of P and of Q (the
+    heaviest users / items first, then uniform draws) as float32 in
+    tests/golden/oracle_det_<name>_B<B>.npz, for the full-size DET parity test."""
+    import numpy as np
+    cfg = synth.CONFIGS[name]
+    (u, v, r), _ = synth.make(cfg)
+    t0 = time.time()
+    prob = oracle.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=cfg.seed)
+    prob.init(1)
+    prob.epoch("det", "none")
+    P, Q = prob.factors()
+    rng = np.random.default_rng(7)
+    cu, cv = np.bincount(u, minlength=cfg.m), np.bincount(v, minlength=cfg.n)
+
+    def pick(cnt, n):
+        top = np.argsort(-cnt, kind="stable")[: rows // 4]
+        rest = rng.choice(np.setdiff1d(np.arange(n), top), rows - len(top), replace=False)
+        return np.sort(np.concatenate([top, rest])).astype(np.int64)
+
+    iu, iv = pick(cu, cfg.m), pick(cv, cfg.n)
+    path = os.path.join(ROOT, "tests", "golden", f"oracle_det_{name}_B{B}.npz")
+    np.savez_compressed(path, users=iu, items=iv, P=P[iu].astype(np.float32), Q=Q[iv].astype(np.float32),
+                        note=np.array("oracle DET epoch 1 from init(1), shuffle seed = config seed, "
+                                      f"grid {B}x{B}; rows of P (users) and Q (items) in original ids"))
+    print(name, B, "det sample", path, f"{time.time() - t0:.0f}s", flush=True)
+
+
 def main(names):
     for name in names:
+        if name.startswith("det:"):  # e.g. det:c3:2048 -> sampled rows after one DET epoch
+            _, n_, B = name.split(":")
+            det_epoch_sample(n_, int(B))
+            continue
         if ":" in name:  # e.g. c3:2048 -> digest of the B x B DET partition only
             n_, B = name.split(":")
             det_digest(n_, int(B))
