@@ -78,6 +78,7 @@ def parse():
     ap.add_argument("--warps", type=int, default=0)
     ap.add_argument("--task", type=int, default=0)
     ap.add_argument("--vec", type=int, default=0, help="float4 slots per lane (0 = library auto)")
+    ap.add_argument("--depth", type=int, default=0, help="Hogwild q_v prefetch distance (0 = library auto)")
     ap.add_argument("--det-wave", type=int, default=1, choices=[0, 1, 2],
                     help="DET: 1 wavefront with Q slabs in shared memory, 2 wavefront, 0 per-stratum launches")
     ap.add_argument("--impl", default="hccmf", choices=["hccmf", "reference"])
@@ -297,6 +298,8 @@ def main():
         mdl.set_option("task_ratings", args.task)
     if args.vec:
         mdl.set_option("vec", args.vec)
+    if args.depth:
+        mdl.set_option("prefetch_depth", args.depth)
     if args.det_wave != 1:
         mdl.set_option("det_wave", args.det_wave)
     if not on_device:

@@ -185,9 +185,11 @@ typedef enum {
     HCCMF_OPT_L2_PERSIST = 12,   /* 1: during a Hogwild epoch Q is an L2 persisting
                                     access-policy window on the launch stream
                                     (removed afterwards).  Default 0.             */
-    HCCMF_OPT_PREFETCH_DEPTH = 13,/* Hogwild, one rating per warp (k = 128 j): the
-                                    q_v row of rating j + D is requested while
-                                    rating j is updated (1..4; default 1).  Loads
+    HCCMF_OPT_PREFETCH_DEPTH = 13,/* Hogwild, one rating per warp (k = 32, 64 and
+                                    k = 128 j): the q_v row of rating j + D is
+                                    requested while rating j is updated (1..4;
+                                    0 = auto, the default: 1 for k = 128 j, 4 for
+                                    k = 32 / 64).  Loads
                                     issued before a warp's own update of the same
                                     item are corrected in registers, so a single
                                     warp stays serial; across warps D widens the

@@ -381,7 +381,7 @@ int64_t auto_warps(hccmf_t h, int64_t items_in_play) {
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
   int64_t w = (int64_t)sms * 32;
   if (h->opt_conflict > 0) {
-    const int64_t groups_per_warp = 32 / sgd_lanes(h->k, (int)h->opt_vec);
+    const int64_t groups_per_warp = hogwild_groups_per_warp(h->k, (int)h->opt_vec);
     const int64_t cap = std::max<int64_t>(1, (items_in_play / h->opt_conflict) / groups_per_warp);
     w = std::min(w, cap);
   }
@@ -585,7 +585,7 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
       h->storage = (int32_t)value;
       return HCCMF_OK;
     case HCCMF_OPT_PREFETCH_DEPTH:
-      if (value < 1 || value > 4) return fail(h, HCCMF_EINVAL, "prefetch depth must be in [1, 4]");
+      if (value < 0 || value > 4) return fail(h, HCCMF_EINVAL, "prefetch depth must be in [0, 4] (0 = auto)");
       h->opt_depth = value;
       return HCCMF_OK;
     case HCCMF_OPT_SYNC_PHASES:

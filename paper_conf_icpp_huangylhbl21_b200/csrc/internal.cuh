@@ -90,6 +90,8 @@ cudaError_t launch_wave_slab(const SgdArgs& a, const int64_t* off, int B, int* p
 // lane geometry of the SGD kernel: L lanes per rating group, VEC float4 per lane
 void sgd_geometry(int k, int vec_pref, int* L, int* VEC);
 int sgd_lanes(int k, int vec_pref);
+// Hogwild rating groups per warp (1 for the warp-per-rating kernels)
+int hogwild_groups_per_warp(int k, int vec_pref);
 // lanes per rating of the RMSE kernel (one float4 per lane)
 int lanes_per_rating(int k);
 
@@ -152,7 +154,7 @@ struct hccmf_ctx {
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 3, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1, opt_wire16 = 0, opt_l2persist = 0, opt_depth = 1;
+  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 3, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1, opt_wire16 = 0, opt_l2persist = 0, opt_depth = 0;
   bool sync_stream = true;
   size_t device_bytes = 0;
 

@@ -876,6 +876,166 @@ struct WarpSgd {
   }
 };
 
+// ---- Hogwild for k = 32 / 64 (C2): one rating per warp, lane l holds E = k/32
+// consecutive floats of p_u and q_v (one coalesced 4- or 8-byte access per lane; a row is
+// 128 / 256 B).  Why not the lane-group kernel (k/4 lanes per rating, 32/L ratings in
+// lock step): it waits on every q_v load one rating ahead, so a heavy user's run -- one
+// task, serial through p_u -- advanced at ~one L2 round trip per rating and formed the
+// epoch's tail (C2's heaviest user has 5,919 ratings).  Here q_v is requested D ratings
+// ahead from a register ring (the run_deep scheme: rows loaded before this warp's own
+// update of the same item get the increment in registers, so one warp alone is serial),
+// and a run advances at the latency of its dot-product chain.
+template <int E, bool ATOMIC>
+struct NarrowSgd {
+  static constexpr unsigned FM = 0xffffffffu;
+  const SgdArgs& a;
+  int lane, k;
+  float g, c1, ngl;
+  const float* Pb;
+  const float* Qb;
+  __device__ NarrowSgd(const SgdArgs& args) : a(args) {
+    lane = threadIdx.x & 31;
+    k = a.k;
+    g = a.gamma;
+    c1 = 1.f - a.gamma * a.lambda;
+    ngl = -a.gamma * a.lambda;
+    Pb = a.P + lane * E - (int64_t)a.row0 * k;
+    Qb = a.Q + lane * E;
+  }
+  __device__ __forceinline__ const float* prow(int u) const { return Pb + (int64_t)u * k; }
+  __device__ __forceinline__ const float* qrow(int v) const { return Qb + (int64_t)v * k; }
+  static __device__ __forceinline__ void ld(const float* r, float (&x)[E]) {
+    if constexpr (E == 1) {
+      x[0] = __ldcg(r);
+    } else {
+      const float2 t = __ldcg(reinterpret_cast<const float2*>(r));
+      x[0] = t.x, x[1] = t.y;
+    }
+  }
+  static __device__ __forceinline__ void st(const float* r, const float (&x)[E]) {
+    if constexpr (E == 1)
+      __stcg(const_cast<float*>(r), x[0]);
+    else
+      __stcg(reinterpret_cast<float2*>(const_cast<float*>(r)), make_float2(x[0], x[1]));
+  }
+  static __device__ __forceinline__ void red(const float* r, const float (&x)[E]) {
+    if constexpr (E == 1)
+      asm volatile("red.relaxed.gpu.global.add.f32 [%0], %1;" ::"l"(r), "f"(x[0]) : "memory");
+    else
+      asm volatile("red.relaxed.gpu.global.add.v2.f32 [%0], {%1, %2};" ::"l"(r), "f"(x[0]), "f"(x[1]) : "memory");
+  }
+
+  template <int D>
+  __device__ __forceinline__ void run(int64_t lo, int left) {
+    constexpr int R = D + 1;
+    const int32_t* ru = a.ru + lo;
+    const int32_t* rv = a.rv + lo;
+    const float* rr = a.rr + lo;
+    int wu0 = 0, wv0 = 0, wu1 = 0, wv1 = 0;
+    float wr0 = 0.f, wr1 = 0.f;
+    if (lane < left) wu0 = __ldcs(ru + lane), wv0 = __ldcs(rv + lane), wr0 = __ldcs(rr + lane);
+    if (lane + 32 < left) wu1 = __ldcs(ru + 32 + lane), wv1 = __ldcs(rv + 32 + lane), wr1 = __ldcs(rr + 32 + lane);
+    int wb = 0;
+    int su[R], sv[R];
+    float sr[R];
+    float q[R][E], p[E], pn[E];
+#pragma unroll
+    for (int s = 0; s < R; ++s) {
+      su[s] = sv[s] = 0;
+      sr[s] = 0.f;
+    }
+#pragma unroll
+    for (int s = 0; s < D; ++s) {
+      if (s < left) {
+        su[s] = __shfl_sync(FM, wu0, s);
+        sv[s] = __shfl_sync(FM, wv0, s);
+        sr[s] = __shfl_sync(FM, wr0, s);
+        ld(qrow(sv[s]), q[s]);
+      }
+    }
+    ld(prow(su[0]), p);
+    for (int j0 = 0; j0 < left; j0 += R) {
+#pragma unroll
+      for (int c = 0; c < R; ++c) {
+        const int j = j0 + c;
+        if (j >= left) break;
+        const int ns = (c + D) % R;  // slot of rating j + D
+        const int jn = j + D;
+        if (jn < left) {
+          if (jn - wb == 32) {  // slide the record window
+            wu0 = wu1, wv0 = wv1, wr0 = wr1;
+            wb += 32;
+            const int idx = wb + 32 + lane;
+            if (idx < left) wu1 = __ldcs(ru + idx), wv1 = __ldcs(rv + idx), wr1 = __ldcs(rr + idx);
+          }
+          const int src = jn - wb;
+          su[ns] = __shfl_sync(FM, wu0, src);
+          sv[ns] = __shfl_sync(FM, wv0, src);
+          sr[ns] = __shfl_sync(FM, wr0, src);
+          ld(qrow(sv[ns]), q[ns]);
+        }
+        const int cn = (c + 1) % R;
+        const bool has_next = j + 1 < left;
+        const bool newp = has_next && su[cn] != su[c];
+        if (newp) ld(prow(su[cn]), pn);
+        float d = p[0] * q[c][0];
+#pragma unroll
+        for (int e = 1; e < E; ++e) d = fmaf(p[e], q[c][e], d);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
+        const float ge = g * (sr[c] - d);
+        float dq[E];
+#pragma unroll
+        for (int e = 0; e < E; ++e) {
+          dq[e] = fmaf(ge, p[e], ngl * q[c][e]);
+          p[e] = fmaf(ge, q[c][e], c1 * p[e]);
+        }
+        const float* qw = qrow(sv[c]);
+        if (ATOMIC) {
+          red(qw, dq);
+        } else {
+#pragma unroll
+          for (int e = 0; e < E; ++e) dq[e] = q[c][e] + dq[e];
+          st(qw, dq);
+        }
+        // pending rows j+1 .. j+D were all requested before this update
+#pragma unroll
+        for (int t = 1; t <= D; ++t) {
+          const int s2 = (c + t) % R;
+          if (j + t < left && sv[s2] == sv[c]) {
+#pragma unroll
+            for (int e = 0; e < E; ++e) q[s2][e] = ATOMIC ? q[s2][e] + dq[e] : dq[e];
+          }
+        }
+        if (!has_next || newp) {
+          st(prow(su[c]), p);
+          if (newp) {
+#pragma unroll
+            for (int e = 0; e < E; ++e) p[e] = pn[e];
+          }
+        }
+      }
+    }
+  }
+};
+
+template <int E, bool ATOMIC, int D>
+__global__ void __launch_bounds__(kThreads) sgd_narrow_kernel(SgdArgs a) {
+  constexpr unsigned FM = 0xffffffffu;
+  NarrowSgd<E, ATOMIC> w(a);
+  unsigned long long tn = 0;
+  if (w.lane == 0) tn = atomicAdd(a.counter, 1ull);
+  tn = __shfl_sync(FM, tn, 0);
+  while (tn < (unsigned long long)a.n_tasks) {
+    const int64_t lo = a.task_lo[tn];
+    const int left = (int)(a.task_hi[tn] - lo);
+    unsigned long long tn2 = 0;
+    if (w.lane == 0) tn2 = atomicAdd(a.counter, 1ull);  // next task id, fetched one task ahead
+    w.template run<D>(lo, left);
+    tn = __shfl_sync(FM, tn2, 0);
+  }
+}
+
 #ifndef HCCMF_WARP_MINB
 #define HCCMF_WARP_MINB 1
 #endif
@@ -1066,7 +1226,7 @@ cudaError_t launch_t(const SgdArgs& a, int64_t warps, cudaStream_t st) {
   const int threads = w < kThreads / 32 ? (int)w * 32 : kThreads;
   const int64_t blocks = (w * 32 + threads - 1) / threads;
   if (L == 32 && FULL) {  // warp-per-rating specialisation
-    const int depth = a.depth < 1 ? 1 : a.depth;
+    const int depth = a.depth < 1 ? 1 : a.depth;  // auto: one rating ahead
 #define WARP_CASE(DD, QQ)                                                     \
   if (depth == DD && a.qhalf == QQ) {                                         \
     if (a.atomic_q)                                                           \
@@ -1242,8 +1402,36 @@ cudaError_t launch_wave_slab(const SgdArgs& a, const int64_t* off, int B, int* p
   return cudaGetLastError();
 }
 
+// Hogwild with k = 32 or 64 (auto geometry, fp32 Q) runs one rating per warp (NarrowSgd)
+static bool narrow_hogwild(int k, int vec_pref) { return vec_pref == 0 && (k == 32 || k == 64); }
+
+int hogwild_groups_per_warp(int k, int vec_pref) {
+  return narrow_hogwild(k, vec_pref) ? 1 : 32 / sgd_lanes(k, vec_pref);
+}
+
+static cudaError_t launch_narrow(const SgdArgs& a, int64_t warps, cudaStream_t st) {
+  int64_t w = std::min<int64_t>(warps, a.n_tasks);
+  if (w < 1) return cudaSuccess;
+  const int threads = w < kThreads / 32 ? (int)w * 32 : kThreads;
+  const unsigned blocks = (unsigned)((w * 32 + threads - 1) / threads);
+  const int depth = a.depth < 1 ? 4 : a.depth;  // auto: 4 ratings ahead
+#define NARROW_CASE(EE, DD)                                                                       \
+  if (a.k == 32 * EE && depth == DD) {                                                            \
+    if (a.atomic_q)                                                                               \
+      (note_launch(), sgd_narrow_kernel<EE, true, DD><<<blocks, threads, 0, st>>>(a));           \
+    else                                                                                          \
+      (note_launch(), sgd_narrow_kernel<EE, false, DD><<<blocks, threads, 0, st>>>(a));          \
+    return cudaGetLastError();                                                                    \
+  }
+  NARROW_CASE(1, 1) NARROW_CASE(1, 2) NARROW_CASE(1, 3) NARROW_CASE(1, 4)
+  NARROW_CASE(2, 1) NARROW_CASE(2, 2) NARROW_CASE(2, 3) NARROW_CASE(2, 4)
+#undef NARROW_CASE
+  return cudaErrorInvalidValue;
+}
+
 cudaError_t launch_sgd(const SgdArgs& a, int64_t warps, cudaStream_t st) {
   if (a.n_tasks <= 0) return cudaSuccess;
+  if (!a.prefetch && !a.qhalf && narrow_hogwild(a.k, a.vec_pref)) return launch_narrow(a, warps, st);
   int L, VEC;
   sgd_geometry(a.k, a.vec_pref, &L, &VEC);
   const bool full = (L * VEC * 4 == a.k);

@@ -232,9 +232,12 @@ def test_det_logical_shards_parity(pkg, orc, sync, G, Br, Bc):
 @pytest.mark.parametrize("k,task,depth,dup", [(128, 64, 1, False), (256, 64, 1, False), (128, 1000, 1, False),
                                               (128, 1000, 2, False), (128, 100, 3, False), (128, 1000, 4, False),
                                               (128, 300, 1, True), (256, 300, 1, True), (128, 300, 2, True),
-                                              (128, 300, 4, True)])
+                                              (128, 300, 4, True),
+                                              # k = 32 / 64: the one-rating-per-warp narrow kernel
+                                              (32, 64, 0, False), (32, 1000, 1, False), (64, 1000, 3, False),
+                                              (32, 300, 2, True), (64, 300, 0, True), (32, 300, 4, True)])
 def test_hogwild_single_group_is_the_serial_oracle(pkg, orc, atomic, k, task, depth, dup):
-    # One warp = one rating group (k >= 128) walks the tasks in record order: the
+    # One warp = one rating group (k = 32, 64 and k >= 128) walks the tasks in record order: the
     # Hogwild kernel then IS the oracle's serial epoch (task builder, user runs,
     # p_u carry, q forwarding and same-thread red->load ordering all pinned).
     # dup: every rating twice (adjacent after the sort): q forwarding on every other step.
