@@ -25,7 +25,8 @@ SRC = r'''
 #include <cstdint>
 #include <cuda_fp16.h>
 // MODE 0: ld + dependent red (fp32 rows), 1: same with binary16 rows,
-// 2: ld only (fp32), 3: red only (fp32), 4: records only
+// 2: ld only (fp32), 3: red only (fp32), 4: records only, 5: TMA bulk reduce only,
+// 6: ld + dependent TMA bulk reduce
 template <int MODE>
 __device__ void body(const int* __restrict__ rv, const float* __restrict__ rr, long long nrec, char* Q, int rowb,
                      long long per_warp, float* sink) {
@@ -35,6 +36,8 @@ __device__ void body(const int* __restrict__ rv, const float* __restrict__ rr, l
   if (hi > nrec) hi = nrec;
   if (lo >= hi) return;
   const int lb = (MODE == 1) ? 8 : 16;
+  __shared__ float4 stage_all[8][64];
+  float4* stage = stage_all[(threadIdx.x >> 5) & 7];
   float acc = 0.f;
   int wv = 0; float wr = 0.f;
   long long wb = lo;
@@ -44,7 +47,7 @@ __device__ void body(const int* __restrict__ rv, const float* __restrict__ rr, l
   float4 qc = make_float4(0, 0, 0, 0), qn;
   uint2 hc = make_uint2(0, 0), hn;
   const char* qp = Q + (long long)cv * rowb + lane * lb;
-  if (MODE == 0 || MODE == 2) qc = __ldcg(reinterpret_cast<const float4*>(qp));
+  if (MODE == 0 || MODE == 2 || MODE == 6) qc = __ldcg(reinterpret_cast<const float4*>(qp));
   if (MODE == 1) hc = __ldcg(reinterpret_cast<const uint2*>(qp));
   for (long long j = lo; j < hi; ++j) {
     const long long jn = j + 1;
@@ -59,7 +62,7 @@ __device__ void body(const int* __restrict__ rv, const float* __restrict__ rr, l
     }
     const char* np = Q + (long long)nv * rowb + lane * lb;
     if (jn < hi) {
-      if (MODE == 0 || MODE == 2) qn = __ldcg(reinterpret_cast<const float4*>(np));
+      if (MODE == 0 || MODE == 2 || MODE == 6) qn = __ldcg(reinterpret_cast<const float4*>(np));
       if (MODE == 1) hn = __ldcg(reinterpret_cast<const uint2*>(np));
     }
     const float s = cr * 1e-30f;  // the reduced value depends on the record and the load
@@ -76,22 +79,41 @@ __device__ void body(const int* __restrict__ rv, const float* __restrict__ rr, l
     } else if (MODE == 3) {
       asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(qp), "f"(s), "f"(s),
                    "f"(s), "f"(s) : "memory");
+    } else if (MODE == 5 || MODE == 6) {
+      // TMA bulk reduction of the whole 512 B row from shared memory (async proxy), the
+      // warp's staging slot double-buffered; MODE 6 reduces the loaded row (dependent)
+      float4* st = stage + ((j & 1) << 5) + lane;
+      asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+      __syncwarp();
+      *st = MODE == 6 ? make_float4(qc.x * s, qc.y * s, qc.z * s, qc.w * s) : make_float4(s, s, s, s);
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) {
+        const unsigned sa = (unsigned)__cvta_generic_to_shared(stage + ((j & 1) << 5));
+        asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f32 [%0], [%1], 512;"
+                     :: "l"(Q + (long long)cv * rowb), "r"(sa) : "memory");
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      }
     } else {
       acc += s + (float)cv;
     }
     qc = qn; hc = hn; qp = np; cv = nv; cr = nr;
   }
+  if (MODE == 5 || MODE == 6) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   if (acc == 1.2345f) sink[0] = acc;
 }
 extern "C" __global__ void __launch_bounds__(256) probe0(const int* rv, const float* rr, long long n, char* Q, int rowb, long long pw, float* s) { body<0>(rv, rr, n, Q, rowb, pw, s); }
 extern "C" __global__ void __launch_bounds__(256) probe1(const int* rv, const float* rr, long long n, char* Q, int rowb, long long pw, float* s) { body<1>(rv, rr, n, Q, rowb, pw, s); }
 extern "C" __global__ void __launch_bounds__(256) probe2(const int* rv, const float* rr, long long n, char* Q, int rowb, long long pw, float* s) { body<2>(rv, rr, n, Q, rowb, pw, s); }
 extern "C" __global__ void __launch_bounds__(256) probe3(const int* rv, const float* rr, long long n, char* Q, int rowb, long long pw, float* s) { body<3>(rv, rr, n, Q, rowb, pw, s); }
+extern "C" __global__ void __launch_bounds__(256) probe5(const int* rv, const float* rr, long long n, char* Q, int rowb, long long pw, float* s) { body<5>(rv, rr, n, Q, rowb, pw, s); }
+extern "C" __global__ void __launch_bounds__(256) probe6(const int* rv, const float* rr, long long n, char* Q, int rowb, long long pw, float* s) { body<6>(rv, rr, n, Q, rowb, pw, s); }
 extern "C" __global__ void __launch_bounds__(256) probe4(const int* rv, const float* rr, long long n, char* Q, int rowb, long long pw, float* s) { body<4>(rv, rr, n, Q, rowb, pw, s); }
 '''
 
 MODES = {0: "ld+red fp32 (512+512 B)", 1: "ld+red binary16 (256+256 B)", 2: "ld only fp32",
-         3: "red only fp32", 4: "records only"}
+         3: "red only fp32", 4: "records only", 5: "bulk reduce only fp32 (TMA, 512 B)",
+         6: "ld + dependent bulk reduce fp32 (TMA)"}
 
 
 def main():
@@ -130,7 +152,7 @@ def main():
     per_warp = (nrec + args.warps - 1) // args.warps
     Q = torch.zeros(cfg.n * k, dtype=torch.float32, device="cuda")
     sink = torch.zeros(1, device="cuda")
-    for mode in range(5):
+    for mode in range(7):
         _, fn = drv.cuModuleGetFunction(mod, f"probe{mode}".encode())
         rowb = k * (2 if mode == 1 else 4)
         vals = [ctypes.c_void_p(rv.data_ptr()), ctypes.c_void_p(rr.data_ptr()), ctypes.c_longlong(nrec),
