@@ -79,6 +79,8 @@ def parse():
     ap.add_argument("--task", type=int, default=0)
     ap.add_argument("--vec", type=int, default=0, help="float4 slots per lane (0 = library auto)")
     ap.add_argument("--depth", type=int, default=0, help="Hogwild q_v prefetch distance (0 = library auto)")
+    ap.add_argument("--no-det-leg", dest="det_leg", action="store_false",
+                    help="skip the DET-schedule leg (C3 only) reported beside the Hogwild headline")
     ap.add_argument("--det-wave", type=int, default=1, choices=[0, 1, 2],
                     help="DET: 1 wavefront with Q slabs in shared memory, 2 wavefront, 0 per-stratum launches")
     ap.add_argument("--impl", default="hccmf", choices=["hccmf", "reference"])
@@ -321,22 +323,24 @@ def main():
     peak, peak_src = hbm_peak()
     local_nnz = info["local_nnz"]
 
-    def measure(storage):
+    def measure(storage, sched=None, steps=None):
         """W warm-up + K timed steps (epoch + Q sync + test RMSE) from a fresh init(1)."""
+        sched = sched or args.sched
+        steps = steps or args.steps
         rm0 = mdl.rmse(dtu, dtv, dtr)
         mdl.set_option("sync_stream", 0)
 
         def step(ev=None):
             if ev is not None:
                 ev[0].record(stream)
-            mdl.train_epoch(args.sched, sync)
+            mdl.train_epoch(sched, sync)
             if ev is not None:
                 ev[1].record(stream)
             return mdl.rmse(dtu, dtv, dtr)
 
         curve = [rm0] + [step() for _ in range(args.warmup)]
         kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-               for _ in range(args.steps)]
+               for _ in range(steps)]
         t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         clocks = Clocks(local)
         clocks.start()
@@ -346,7 +350,7 @@ def main():
         torch.cuda.synchronize()
         l0 = hc.kernel_launches()
         t_start.record(stream)
-        rms = [step(kev[i]) for i in range(args.steps)]
+        rms = [step(kev[i]) for i in range(steps)]
         t_end.record(stream)
         launches = hc.kernel_launches() - l0  # counted by the library at its launch sites
         torch.cuda.synchronize()
@@ -367,14 +371,15 @@ def main():
         b_upd = 12 + (16 if storage == "fp32" else 12) * cfg.k
         achieved = local_nnz * b_upd / (kmean / 1e3) / 1e9
         roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": ncu_traffic(args.config + ("" if storage == "fp32" else "-" + storage), args.sched),
+                "traffic": ncu_traffic(args.config + ("" if storage == "fp32" else "-" + storage), sched),
                 "kernel": "sgd_warp_kernel (a5/a6 epoch incl. Q sync%s)"
                           % ("" if storage == "fp32" else ", binary16 round-in/write-back of Q"),
                 "bytes_per_update": b_upd, "updates_per_launch": local_nnz, "kernel_ms": kmean,
-                "kernel_share_of_step": kmean / (ms / args.steps), "peak_source": peak_src,
-                "binding_unit": binding_unit(storage, args, local_nnz / (kmean / 1e3))}
+                "kernel_share_of_step": kmean / (ms / steps), "peak_source": peak_src,
+                "binding_unit": binding_unit(storage, args, local_nnz / (kmean / 1e3)) if sched == "hogwild"
+                else None}
         roof["kernel_launches_timed"] = launches
-        return nnz * args.steps / (ms / 1e3), ms, roof, clk, curve + rms
+        return nnz * steps / (ms / 1e3), ms, roof, clk, curve + rms
 
     value, ms, roof, clk, curve = measure(args.storage)
 
@@ -409,6 +414,26 @@ def main():
                                        "same band vs the fp64 oracle"
                                        % (", stochastic rounding of every q write" if args.fp16_leg == "fp16sr"
                                           else "")}
+
+    # secondary leg: the deterministic schedule (a5) on the same data, the bench's DET
+    # configuration (one shard, 2048 x 2048 grid, the shared-memory-slab wavefront: one
+    # launch per epoch), fp32; parity with the oracle is the full-size GPU test's
+    if (args.det_leg and args.sched == "hogwild" and world == 1 and args.config == "c3" and not on_device):
+        mdl.close()  # the handle released its input COO after partition: a fresh one for DET
+        mdl = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, device=local)
+        mdl.set_stream(stream)
+        mdl.load(u, v, r)
+        mdl.partition(1, (2048, 2048), "DP0", seed=cfg.seed)
+        mdl.init(1)
+        kd = min(args.steps, 3)
+        vd, msd, roofd, clkd, curved = measure("fp32", sched="det", steps=kd)
+        roofd["kernel"] = "sgd_wave_slab_kernel (a5 DET epoch, one launch)"
+        out["det"] = {"sched": "det", "grid": [2048, 2048], "value": vd, "unit": UNIT, "steps": kd,
+                      "warmup": args.warmup, "ms_per_step": msd / kd,
+                      "gpu_launches": roofd.pop("kernel_launches_timed"), "roofline": roofd, "clocks": clkd,
+                      "test_rmse": curved[-1],
+                      "note": "serial-equivalent FPSGD strata (R19); bound by the hottest column block's "
+                              "serial chain (profiles/r01_det_wavefront.md)"}
 
     mdl.close()  # free HBM before the e2e jobs build their own handles
     # ---- e2e: the whole job through the public API from pinned host buffers
