@@ -605,3 +605,31 @@ def test_kernel_launch_counter(pkg):
     mdl.train_epoch("hogwild", "none")
     assert pkg.kernel_launches() - l0 == 4
     mdl.close()
+
+
+@pytest.mark.parametrize("m,n,nnz,B,k", [(50, 20, 3000, 37, 128), (40, 300, 4000, 2, 128), (300, 7, 2500, 5, 256),
+                                         (64, 64, 0, 8, 128), (1, 90, 400, 3, 128)])
+def test_det_wavefront_degenerate_grids(pkg, orc, m, n, nnz, B, k):
+    # the slab wavefront on degenerate geometries: more column blocks than items (empty,
+    # zero-width slabs), more row blocks than rows, one row, an empty problem, duplicated
+    # cells (synth.tiny): one launch, bit-identical to the per-stratum launches, oracle to 1e-4
+    u, v, r = synth.tiny(m, n, nnz, seed=m + n + B)
+    prob = orc.Problem(m, n, k, 0.02, 0.01, u, v, r, G=1, Br=B, Bc=B, seed=9)
+    prob.init(5)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    outs = []
+    for wave in (1, 0):
+        mdl = _gpu_problem(pkg, m, n, k, 0.02, 0.01, u, v, r, G=1, Br=B, Bc=B, seed=9)
+        mdl.set_option("det_wave", wave)
+        mdl.set_factors(P0, Q0)
+        l0 = pkg.kernel_launches()
+        mdl.train_epoch("det", "none")
+        if wave == 1:
+            assert pkg.kernel_launches() - l0 == 1
+        outs.append(mdl.factors())
+        mdl.close()
+    prob.epoch("det", "none")
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+    Po, Qo = prob.factors()
+    assert max(np.abs(outs[0][0] - Po).max(), np.abs(outs[0][1] - Qo).max()) <= 1e-4
