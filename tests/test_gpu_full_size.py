@@ -76,15 +76,16 @@ def test_hogwild_band_full_size(pkg, c3, name, data, storage):
     mdl = pkg.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam)
     mdl.load(u, v, r)
     mdl.partition(1, (1, 1), seed=cfg.seed, storage=storage)
-    mdl.init(1)
-    curve = [mdl.rmse(tu, tv, tr)]
     E = ref["epochs"]
-    for _ in range(E):
-        mdl.train_epoch("hogwild", "none")
-        curve.append(mdl.rmse(tu, tv, tr))
-    if storage == "fp32":
-        assert curve[0] == pytest.approx(ref["test_rmse"][0], rel=1e-6)  # same init, same data
-    assert abs(curve[E] - ref["test_rmse"][E]) <= 0.005, (curve, ref["test_rmse"])
+    for _ in range(3):  # Hogwild is nondeterministic: every one of 3 runs in the band
+        mdl.init(1)
+        curve = [mdl.rmse(tu, tv, tr)]
+        for _ in range(E):
+            mdl.train_epoch("hogwild", "none")
+            curve.append(mdl.rmse(tu, tv, tr))
+        if storage == "fp32":
+            assert curve[0] == pytest.approx(ref["test_rmse"][0], rel=1e-6)  # same init, same data
+        assert abs(curve[E] - ref["test_rmse"][E]) <= 0.005, (curve, ref["test_rmse"])
 
 
 def test_c5_full_size_properties(pkg):

@@ -297,7 +297,7 @@ def test_hogwild_band_c1(pkg, orc):
 
 def test_hogwild_band_c2_full(pkg, orc):
     # BASELINE.json config 2 at full size; band read at E = 20 epochs (R15)
-    want, got = _band(pkg, orc, "c2", 1.0, 32, 20)
+    want, got = _band(pkg, orc, "c2", 1.0, 32, 20, repeats=3)  # Hogwild bands run 3 times
     assert all(abs(g - want) <= 0.005 for g in got), (want, got)
 
 
