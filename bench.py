@@ -202,15 +202,24 @@ def oracle_sample(cfg, u, v, r, seconds):
     prob = oracle.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u[:S], v[:S], r[:S], G=1, Br=1, Bc=1,
                           seed=cfg.seed)
     prob.init(1)
-    t0 = time.perf_counter()
-    epochs = 0
-    while True:
-        prob.epoch("serial", "none")
-        epochs += 1
-        if time.perf_counter() - t0 >= seconds:
-            break
-    dt = time.perf_counter() - t0
-    return S * epochs / dt, S, epochs, dt
+    # one host core: pin this thread while the serial oracle runs
+    saved = os.sched_getaffinity(0) if hasattr(os, "sched_getaffinity") else None
+    core = max(saved) if saved else -1
+    if saved:
+        os.sched_setaffinity(0, {core})
+    try:
+        t0 = time.perf_counter()
+        epochs = 0
+        while True:
+            prob.epoch("serial", "none")
+            epochs += 1
+            if time.perf_counter() - t0 >= seconds:
+                break
+        dt = time.perf_counter() - t0
+    finally:
+        if saved:
+            os.sched_setaffinity(0, saved)
+    return S * epochs / dt, S, epochs, dt, core
 
 
 # ------------------------------------------------------------ reference arm
@@ -490,11 +499,12 @@ def main():
                               "host pinned buffers", "s_per_step": e2e_s}
 
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        val, S, ep, dt = oracle_sample(cfg, *sample, args.cpu_seconds)
+        val, S, ep, dt, core = oracle_sample(cfg, *sample, args.cpu_seconds)
         model, ncpu = host_cpu()
         out["cpu_baseline"] = {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",
                                "sample": f"{ep} serial fp64 oracle epoch(s) over the first {S} ratings of the "
-                                         f"same stream, {dt:.1f} s on 1 of {ncpu} cores ({model})"}
+                                         f"same stream, {dt:.1f} s on 1 of {ncpu} cores (core {core} pinned; "
+                                         f"{model})"}
     if rank == 0:
         print(json.dumps(out), flush=True)
     if world > 1:
