@@ -715,6 +715,7 @@ struct WarpSgd {
     }
     int cu = -1;  // user whose row is in p
     float4 p[VEC], q[VEC];
+#pragma unroll 2
     for (int j = 0; j < left; ++j) {
       const int jn = j + D;
       if (j - wb == 32) {  // window 0 consumed: slide; the new window 1 is needed ~20 ratings on
