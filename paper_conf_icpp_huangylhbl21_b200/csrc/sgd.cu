@@ -538,6 +538,7 @@ struct WarpSgd {
     using T = std::true_type;
     using F = std::false_type;
     int j = 0;
+#pragma unroll 2
     for (; left - j >= 3; j += 2) {  // j even: only the odd step can enter a new window
       step(j, qa, qb, T{}, F{});
       step(j + 1, qb, qa, T{}, T{});
