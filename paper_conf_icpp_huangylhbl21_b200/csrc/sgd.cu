@@ -40,6 +40,13 @@ namespace hccmf {
 namespace {
 
 constexpr int kThreads = 256;
+#ifndef HCCMF_WARP_UNROLL  // 2-rating steps per record-ring loop iteration (Hogwild, k = 128 j)
+#define HCCMF_WARP_UNROLL 8
+#endif
+#ifndef HCCMF_NARROW_UNROLL  // R-rating rounds per loop iteration (Hogwild, k = 32 / 64)
+#define HCCMF_NARROW_UNROLL 1
+#endif
+constexpr int kWarpUnroll = HCCMF_WARP_UNROLL, kNarrowUnroll = HCCMF_NARROW_UNROLL;
 
 template <int VEC>
 struct Row {
@@ -538,7 +545,7 @@ struct WarpSgd {
     using T = std::true_type;
     using F = std::false_type;
     int j = 0;
-#pragma unroll 2
+#pragma unroll kWarpUnroll
     for (; left - j >= 3; j += 2) {  // j even: only the odd step can enter a new window
       step(j, qa, qb, T{}, F{});
       step(j + 1, qb, qa, T{}, T{});
@@ -956,6 +963,7 @@ struct NarrowSgd {
       }
     }
     ld(prow(su[0]), p);
+#pragma unroll kNarrowUnroll
     for (int j0 = 0; j0 < left; j0 += R) {
 #pragma unroll
       for (int c = 0; c < R; ++c) {
