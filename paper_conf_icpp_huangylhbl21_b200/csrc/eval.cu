@@ -54,7 +54,11 @@ __global__ void gather_kernel(const float4* src, int64_t rows_total, int32_t k4,
 // a8: one rating group of L lanes per test rating (same lane mapping as the SGD
 // kernel), fp32 dot product, squared error accumulated in fp64 per group in a
 // fixed order, then a fixed-order tree per CTA -> partials[blockIdx].
-template <int L>
+// Each group walks a contiguous chunk of the test set in windows of L ratings: lane sl
+// resolves rating w+sl's permuted ids (tu -> perm_row, tv -> perm_col: two dependent
+// loads, once per window for L ratings at a time), and the p_u / q_v rows of rating
+// j+1 are requested before rating j is reduced.
+template <int L, int S>  // S: float4 slots per lane, ceil(k / 4L) rounded up to 1, 2, 4
 __global__ void __launch_bounds__(kT) rmse_kernel(const int32_t* __restrict__ tu, const int32_t* __restrict__ tv,
                                                   const float* __restrict__ tr, int64_t nt,
                                                   const int32_t* __restrict__ perm_row,
@@ -66,36 +70,73 @@ __global__ void __launch_bounds__(kT) rmse_kernel(const int32_t* __restrict__ tu
   const int sl = lane & (L - 1);
   const int64_t group = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) / L;
   const int64_t ngroups = (int64_t)gridDim.x * blockDim.x / L;
+  const int64_t chunk = (nt + ngroups - 1) / ngroups;
+  const int64_t lo = group * chunk < nt ? group * chunk : nt;
+  const int64_t hi = lo + chunk < nt ? lo + chunk : nt;
   double acc = 0.0, cnt = 0.0;
-  const int64_t iters = (nt + ngroups - 1) / ngroups;
-  for (int64_t it = 0; it < iters; ++it) {
-    const int64_t i = it * ngroups + group;
-    const bool in = i < nt;
-    int64_t up = -1, vp = 0;
-    float rv = 0.f;
-    if (in) {
-      up = (int64_t)perm_row[tu[i]] - row0;
-      vp = perm_col[tv[i]];
-      rv = tr[i];
-    }
-    const bool act = in && up >= 0 && up < rows;
-    float d = 0.f;
-    if (act) {
-      for (int c = sl * 4; c < k; c += 4 * L) {
-        const float4 p = *reinterpret_cast<const float4*>(P + up * k + c);
-        const float4 q = *reinterpret_cast<const float4*>(Q + vp * k + c);
-        d = fmaf(p.x, q.x, d);
-        d = fmaf(p.y, q.y, d);
-        d = fmaf(p.z, q.z, d);
-        d = fmaf(p.w, q.w, d);
+  auto load = [&](int64_t up, int64_t vp, bool act, float4 (&p)[S], float4 (&q)[S]) {
+#pragma unroll
+    for (int s = 0; s < S; ++s) {
+      const int c = (s * L + sl) * 4;
+      if (act && c < k) {
+        p[s] = __ldcs(reinterpret_cast<const float4*>(P + up * k + c));
+        q[s] = __ldg(reinterpret_cast<const float4*>(Q + vp * k + c));
+      } else {
+        p[s] = q[s] = make_float4(0.f, 0.f, 0.f, 0.f);
       }
     }
+  };
+  // every group of a warp runs the same number of windows and steps (the shuffles are
+  // warp-wide): ceil(chunk / L) windows of L steps, masked past the group's own end
+  const int64_t nwin = (chunk + L - 1) / L;
+  for (int64_t wi = 0; wi < nwin; ++wi) {
+    const int64_t w = lo + wi * L;
+    const int64_t idx = w + sl;
+    int64_t ul = -1, vl = 0;
+    float rl = 0.f;
+    if (idx < hi) {
+      ul = (int64_t)perm_row[tu[idx]] - row0;
+      vl = perm_col[tv[idx]];
+      rl = tr[idx];
+    }
+    const int nw = (int)(hi - w <= 0 ? 0 : (hi - w < L ? hi - w : L));
+    float4 pa[S], qa[S], pb[S], qb[S];
+    const int64_t up = __shfl_sync(FM, ul, 0, L), vp = __shfl_sync(FM, vl, 0, L);
+    float r = __shfl_sync(FM, rl, 0, L);
+    bool act = nw > 0 && up >= 0 && up < rows;
+    load(up, vp, act, pa, qa);
+    auto step = [&](int j, float4 (&pc)[S], float4 (&qc)[S], float4 (&pn)[S], float4 (&qn)[S]) {
+      // rating j+1's rows in flight while rating j is reduced
+      const int64_t un = __shfl_sync(FM, ul, (j + 1) & (L - 1), L), vn = __shfl_sync(FM, vl, (j + 1) & (L - 1), L);
+      const float rn = __shfl_sync(FM, rl, (j + 1) & (L - 1), L);
+      const bool actn = j + 1 < nw && un >= 0 && un < rows;
+      load(un, vn, actn, pn, qn);
+      float d = 0.f;
 #pragma unroll
-    for (int o = L / 2; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
-    if (act && sl == 0) {
-      const double e = (double)rv - (double)d;
-      acc += e * e;
-      cnt += 1.0;
+      for (int s = 0; s < S; ++s) {
+        d = fmaf(pc[s].x, qc[s].x, d);
+        d = fmaf(pc[s].y, qc[s].y, d);
+        d = fmaf(pc[s].z, qc[s].z, d);
+        d = fmaf(pc[s].w, qc[s].w, d);
+      }
+#pragma unroll
+      for (int o = L / 2; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o, L);
+      if (act && sl == 0) {
+        const double e = (double)r - (double)d;
+        acc += e * e;
+        cnt += 1.0;
+      }
+      act = actn;
+      r = rn;
+    };
+    if (L == 1) {
+      step(0, pa, qa, pb, qb);
+    } else {
+#pragma unroll 1
+      for (int j = 0; j < L; j += 2) {
+        step(j, pa, qa, pb, qb);
+        step(j + 1, pb, qb, pa, qa);
+      }
     }
   }
   __shared__ double sa[kT], sc[kT];
@@ -206,15 +247,16 @@ cudaError_t k_rmse(const int32_t* tu, const int32_t* tv, const float* tr, int64_
                    const int32_t* perm_col, const float* P, int64_t row0, int64_t rows, const float* Q, int32_t k,
                    double* partials, double* out2, cudaStream_t st) {
   const int L = lanes_per_rating(k);
-  switch (L) {
-#define RM(LL)                                                                                                    \
-  case LL:                                                                                                        \
-    (note_launch(), rmse_kernel<LL><<<RMSE_BLOCKS, kT, 0, st>>>(tu, tv, tr, nt, perm_row, perm_col, P, row0, rows, Q, k, partials)); \
-    break;
-    RM(1) RM(2) RM(4) RM(8) RM(16) RM(32)
+  int S = (k / 4 + L - 1) / L;
+  if (S == 3) S = 4;
+#define RM(LL, SS)                                                                                              \
+  if (L == LL && S == SS) {                                                                                     \
+    (note_launch(), rmse_kernel<LL, SS><<<RMSE_BLOCKS, kT, 0, st>>>(tu, tv, tr, nt, perm_row, perm_col, P, row0, \
+                                                                   rows, Q, k, partials));                      \
+  } else
+  RM(1, 1) RM(2, 1) RM(4, 1) RM(8, 1) RM(16, 1) RM(32, 1) RM(32, 2) RM(32, 4)
 #undef RM
-    default: return cudaErrorInvalidValue;
-  }
+  return cudaErrorInvalidValue;
   (note_launch(), rmse_final_kernel<<<1, 32, 0, st>>>(partials, RMSE_BLOCKS, out2));
   return cudaGetLastError();
 }
