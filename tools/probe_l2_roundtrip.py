@@ -139,12 +139,58 @@ extern "C" __global__ void __launch_bounds__(256) probe7(const int* __restrict__
   }
   if (sink[0] == 1.2345f) sink[1] = 0.f;
 }
+// MODE 8 / 9: fp32 rows in a 64-byte-chunk interleaved layout (chunk j of item v at
+// ((j * n + v) * 64): a row's 8 chunks sit in 8 different lines / L2 slices instead of 4),
+// MODE 8: red only, MODE 9: load + dependent red
+template <int MODE>
+__device__ void body_il(const int* __restrict__ rv, const float* __restrict__ rr, long long nrec, char* Q, int n,
+                        long long per_warp, float* sink) {
+  const int lane = threadIdx.x & 31;
+  const long long w = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+  long long lo = w * per_warp, hi = lo + per_warp;
+  if (hi > nrec) hi = nrec;
+  if (lo >= hi) return;
+  const long long off_l = (long long)(lane >> 2) * n * 64 + (lane & 3) * 16;
+  int wv = 0; float wr = 0.f;
+  long long wb = lo;
+  if (wb + lane < hi) { wv = __ldcs(rv + wb + lane); wr = __ldcs(rr + wb + lane); }
+  int cv = __shfl_sync(~0u, wv, 0);
+  float cr = __shfl_sync(~0u, wr, 0);
+  const char* qp = Q + off_l + (long long)cv * 64;
+  float4 qc = MODE == 9 ? __ldcg(reinterpret_cast<const float4*>(qp)) : make_float4(0, 0, 0, 0), qn = qc;
+  for (long long j = lo; j < hi; ++j) {
+    const long long jn = j + 1;
+    int nv = cv; float nr = cr;
+    if (jn < hi) {
+      if (jn - wb == 32) {
+        wb += 32;
+        if (wb + lane < hi) { wv = __ldcs(rv + wb + lane); wr = __ldcs(rr + wb + lane); }
+      }
+      nv = __shfl_sync(~0u, wv, (int)(jn - wb));
+      nr = __shfl_sync(~0u, wr, (int)(jn - wb));
+    }
+    const char* np = Q + off_l + (long long)nv * 64;
+    if (MODE == 9 && jn < hi) qn = __ldcg(reinterpret_cast<const float4*>(np));
+    const float sc = cr * 1e-30f;
+    if (MODE == 9)
+      asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(qp), "f"(qc.x * sc),
+                   "f"(qc.y * sc), "f"(qc.z * sc), "f"(qc.w * sc) : "memory");
+    else
+      asm volatile("red.relaxed.gpu.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(qp), "f"(sc), "f"(sc),
+                   "f"(sc), "f"(sc) : "memory");
+    qc = qn; qp = np; cv = nv; cr = nr;
+  }
+  if (sink[0] == 1.2345f) sink[1] = 0.f;
+}
+extern "C" __global__ void __launch_bounds__(256) probe8(const int* rv, const float* rr, long long n, char* Q, int rowb, long long pw, float* s) { body_il<8>(rv, rr, n, Q, rowb, pw, s); }
+extern "C" __global__ void __launch_bounds__(256) probe9(const int* rv, const float* rr, long long n, char* Q, int rowb, long long pw, float* s) { body_il<9>(rv, rr, n, Q, rowb, pw, s); }
 extern "C" __global__ void __launch_bounds__(256) probe4(const int* rv, const float* rr, long long n, char* Q, int rowb, long long pw, float* s) { body<4>(rv, rr, n, Q, rowb, pw, s); }
 '''
 
 MODES = {0: "ld+red fp32 (512+512 B)", 1: "ld+red binary16 (256+256 B)", 2: "ld only fp32",
          3: "red only fp32", 4: "records only", 5: "bulk reduce only fp32 (TMA, 512 B)",
-         6: "ld + dependent bulk reduce fp32 (TMA)", 7: "ld+red binary16, 16 lanes x 16 B, 2 ratings per warp"}
+         6: "ld + dependent bulk reduce fp32 (TMA)", 7: "ld+red binary16, 16 lanes x 16 B, 2 ratings per warp",
+         8: "red only fp32, 64 B-chunk interleaved rows", 9: "ld+red fp32, 64 B-chunk interleaved rows"}
 
 
 def main():
@@ -183,9 +229,9 @@ def main():
     per_warp = (nrec + args.warps - 1) // args.warps
     Q = torch.zeros(cfg.n * k, dtype=torch.float32, device="cuda")
     sink = torch.zeros(1, device="cuda")
-    for mode in range(8):
+    for mode in range(10):
         _, fn = drv.cuModuleGetFunction(mod, f"probe{mode}".encode())
-        rowb = k * (2 if mode in (1, 7) else 4)
+        rowb = cfg.n if mode in (8, 9) else k * (2 if mode in (1, 7) else 4)  # 8, 9: the item count
         pw = (nrec + 2 * args.warps - 1) // (2 * args.warps) if mode == 7 else per_warp
         vals = [ctypes.c_void_p(rv.data_ptr()), ctypes.c_void_p(rr.data_ptr()), ctypes.c_longlong(nrec),
                 ctypes.c_void_p(Q.data_ptr()), ctypes.c_int(rowb), ctypes.c_longlong(pw),
