@@ -308,7 +308,8 @@ def test_hogwild_logical_shards_band_c2(pkg, orc, sync, G, Bc):
     assert all(abs(g - want) <= 0.005 for g in got), (want, got)
 
 
-@pytest.mark.parametrize("k,B,dup", [(128, 24, False), (256, 9, False), (128, 37, True), (512, 5, True)])
+@pytest.mark.parametrize("k,B,dup", [(128, 24, False), (256, 9, False), (128, 37, True), (512, 12, True),
+                                     (512, 5, True)])  # k=512, B=5: slab too big -> register wavefront
 def test_det_wavefront_equals_strata(pkg, orc, k, B, dup):
     # the wavefront kernels (Q slab in shared memory: det_wave 1; registers only: 2) and
     # the per-stratum launches (0) apply the same updates in the same per-row /
