@@ -911,8 +911,15 @@ struct NarrowSgd {
     Pb = a.P + lane * E - (int64_t)a.row0 * k;
     Qb = a.Q + lane * E;
   }
-  __device__ __forceinline__ const float* prow(int u) const { return Pb + (int64_t)u * k; }
-  __device__ __forceinline__ const float* qrow(int v) const { return Qb + (int64_t)v * k; }
+  // row addresses with one 32x32->64 multiply-add (ids are non-negative and < 2^31)
+  __device__ __forceinline__ const float* prow(int u) const {
+    return reinterpret_cast<const float*>(reinterpret_cast<const char*>(Pb) +
+                                          (unsigned long long)(unsigned)u * (unsigned)(k * 4));
+  }
+  __device__ __forceinline__ const float* qrow(int v) const {
+    return reinterpret_cast<const float*>(reinterpret_cast<const char*>(Qb) +
+                                          (unsigned long long)(unsigned)v * (unsigned)(k * 4));
+  }
   static __device__ __forceinline__ void ld(const float* r, float (&x)[E]) {
     if constexpr (E == 1) {
       x[0] = __ldcg(r);
