@@ -173,8 +173,15 @@ struct Group {
     for (int t = 0; t < RPL; ++t) wu0[t] = wv0[t] = wu1[t] = wv1[t] = 0, wr0[t] = wr1[t] = 0.f;
   }
 
-  __device__ __forceinline__ const float4* prow(int u) const { return Pb + (int64_t)u * k4; }
-  __device__ __forceinline__ const float4* qrow(int v) const { return Qb + (int64_t)v * k4; }
+  // row addresses with one 32x32->64 multiply-add (ids are non-negative and < 2^31)
+  __device__ __forceinline__ const float4* prow(int u) const {
+    return reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Pb) +
+                                           (unsigned long long)(unsigned)u * (unsigned)(k4 * 16));
+  }
+  __device__ __forceinline__ const float4* qrow(int v) const {
+    return reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Qb) +
+                                           (unsigned long long)(unsigned)v * (unsigned)(k4 * 16));
+  }
 
   __device__ __forceinline__ void load_window(int (&wu)[RPL], int (&wv)[RPL], float (&wr)[RPL], int64_t base,
                                               int avail) {
@@ -336,8 +343,14 @@ struct WarpSgd {
     Qhb = reinterpret_cast<const char*>(a.Q) + lane * 8;
   }
   // 32-bit row offsets: m_local * k/4 and n * k/4 < 2^31
-  __device__ __forceinline__ const float4* prow(int u) const { return Pb + (int64_t)(u * k4); }
-  __device__ __forceinline__ const float4* qrow(int v) const { return Qb + (int64_t)(v * k4); }
+  __device__ __forceinline__ const float4* prow(int u) const {
+    return reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Pb) +
+                                           (unsigned long long)(unsigned)u * (unsigned)(k4 * 16));
+  }
+  __device__ __forceinline__ const float4* qrow(int v) const {
+    return reinterpret_cast<const float4*>(reinterpret_cast<const char*>(Qb) +
+                                           (unsigned long long)(unsigned)v * (unsigned)(k4 * 16));
+  }
   __device__ __forceinline__ void ld(const float4* r, float4 (&x)[VEC]) const {
 #pragma unroll
     for (int i = 0; i < VEC; ++i) x[i] = __ldcg(r + 32 * i);
