@@ -330,11 +330,13 @@ double orc_round_half_sr(double x, uint32_t r13)
 }
 
 /* The random word of element pair c (elements 2c, 2c+1) for the q write of record i in
- * epoch t (R27): lowbias32(i*0x9E3779B1 + t*0x85EBCA77 + c*0xC2B2AE3D mod 2^32), with
- * lowbias32 the 32-bit finaliser of C. Wellons (xorshift-multiply, 2 rounds).  Element 2c
- * takes bits 12:0, element 2c+1 bits 28:16. */
+ * epoch t (R27): for even c, lowbias32(i*0x9E3779B1 + t*0x85EBCA77 + c*0xC2B2AE3D mod 2^32),
+ * with lowbias32 the 32-bit finaliser of C. Wellons (xorshift-multiply, 2 rounds); for odd
+ * c, the word of pair c-1 times 0x9E3779B1 mod 2^32.  Element 2c takes bits 12:0, element
+ * 2c+1 bits 28:16. */
 uint32_t orc_sr_word(int64_t i, uint32_t t, uint32_t c)
 {
+    if (c & 1u) return orc_sr_word(i, t, c - 1u) * 0x9E3779B1u;
     uint32_t x = (uint32_t)i * 0x9E3779B1u + t * 0x85EBCA77u + c * 0xC2B2AE3Du;
     x ^= x >> 16;
     x *= 0x7FEB352Du;

@@ -109,8 +109,10 @@ __device__ __forceinline__ uint2 f4_to_h4(float4 a) {
 }
 // Stochastic rounding (storage = 2, R27).  The random word of element pair c
 // (elements 2c, 2c+1) of the q_v write by the update of record i (global index in the
-// sorted order) in epoch t is r = lowbias32(i*0x9E3779B1 + t*0x85EBCA77 + c*0xC2B2AE3D)
-// (mod 2^32; lowbias32 = C. Wellons' 32-bit finaliser); element 2c is rounded with
+// sorted order) in epoch t is, for even c, r = lowbias32(i*0x9E3779B1 + t*0x85EBCA77 +
+// c*0xC2B2AE3D) (mod 2^32; lowbias32 = C. Wellons' 32-bit finaliser) and, for odd c, the
+// even neighbour's word times 0x9E3779B1 (one multiply instead of a second finaliser: a
+// bijection of the even word, so each 13-bit field stays uniform); element 2c is rounded with
 // r[12:0], element 2c+1 with r[28:16] by cvt.rs.f16x2.f32 (sm_100a F2FP.RS):
 // y = sign(x) floor((|x| + R13 ulp / 2^13) / ulp) ulp, ulp = the binary16 spacing at |x|.
 __device__ __forceinline__ unsigned lowbias32(unsigned x) {
@@ -517,8 +519,9 @@ struct WarpSgd {
           const float4 qq = f4_fma(ge, p[i], f4_scale(c1, qc[i]));
           const unsigned r = rb0 + (unsigned)j * 0x9E3779B1u + (unsigned)(64 * i) * 0xC2B2AE3Du;
           uint2 hs;
-          hs.x = cvt_rs_h2(qq.y, qq.x, lowbias32(r));
-          hs.y = cvt_rs_h2(qq.w, qq.z, lowbias32(r + 0xC2B2AE3Du));
+          const unsigned w0 = lowbias32(r);  // pair c = 64 i + 2 lane (even); pair c + 1: w0 * 0x9E3779B1
+          hs.x = cvt_rs_h2(qq.y, qq.x, w0);
+          hs.y = cvt_rs_h2(qq.w, qq.z, w0 * 0x9E3779B1u);
           snew[i] = hs;
           w[i] = ATOMIC ? make_uint2(hsub2_bits(hs.x, qc_raw[i].x), hsub2_bits(hs.y, qc_raw[i].y)) : hs;
         } else {

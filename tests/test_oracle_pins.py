@@ -445,13 +445,17 @@ def test_sr_rounding_definition(orc):
 
 def test_sr_word_is_the_stated_hash(orc):
     # lowbias32 inverted step by step (modular inverses of the odd multipliers, xorshift
-    # inverses) must give back i*0x9E3779B1 + t*0x85EBCA77 + c*0xC2B2AE3D mod 2^32
+    # inverses) must give back i*0x9E3779B1 + t*0x85EBCA77 + c*0xC2B2AE3D mod 2^32 for even c;
+    # an odd pair's word is its even neighbour's times 0x9E3779B1 (R27): undo that first
     M = 2 ** 32
-    inv1, inv2 = pow(0x846CA68B, -1, M), pow(0x7FEB352D, -1, M)
+    inv1, inv2, inv_phi = pow(0x846CA68B, -1, M), pow(0x7FEB352D, -1, M), pow(0x9E3779B1, -1, M)
     rng = np.random.default_rng(2)
     for _ in range(300):
         i, t, c = int(rng.integers(0, 2 ** 40)), int(rng.integers(0, 2 ** 32)), int(rng.integers(0, 2 ** 12))
         x = orc.sr_word(i, t, c)
+        if c % 2:
+            x = (x * inv_phi) % M
+            c -= 1
         x ^= x >> 16
         x = (x * inv1) % M
         x ^= (x >> 15) ^ (x >> 30)
