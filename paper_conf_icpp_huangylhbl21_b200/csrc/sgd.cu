@@ -1155,7 +1155,11 @@ template <int VEC>
 __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, const int64_t* __restrict__ off, int B,
                                                                  int* progress, int64_t n, int wmax) {
   extern __shared__ float4 wave_smem[];
-  const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+  // row block i -> warp i / CTAs of CTA i mod CTAs: successive row blocks, which hand the
+  // column blocks on to each other, run on different SMs rather than sharing one SM's
+  // schedulers (C3, B = 2048: 71.5 -> 69.5 ms per step).  Waits go through progress[],
+  // so the mapping does not change the order of updates.
+  const int i = (int)((threadIdx.x >> 5) * gridDim.x + blockIdx.x);
   if (i >= B) return;
   WarpSgd<VEC, false> w(a);
   const int k4 = a.k >> 2;
