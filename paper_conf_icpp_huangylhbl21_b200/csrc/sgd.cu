@@ -1107,7 +1107,8 @@ __global__ void __launch_bounds__(kThreads, (VEC == 1 ? 4 : HCCMF_WARP_MINB)) sg
 template <int VEC>
 __global__ void __launch_bounds__(kThreads) sgd_wave_kernel(SgdArgs a, const int64_t* __restrict__ off, int B,
                                                             int* progress) {
-  const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+  // row block i on CTA i mod CTAs, as in sgd_wave_slab_kernel
+  const int i = (int)((threadIdx.x >> 5) * gridDim.x + blockIdx.x);
   if (i >= B) return;
   WarpSgd<VEC, false> w(a);
   const int nb = (i + 1) % B;
