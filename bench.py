@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """bench.py -- rating updates/s of the HCC-MF hot path on B200 (BASELINE.json metric).
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--sched hogwild]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c5] [--sched hogwild]
     torchrun --nproc-per-node N bench.py --gpus N ...         (one rank per GPU, NCCL)
     python bench.py --impl reference ...                       (the oracle arm, host cores)
 
@@ -14,6 +14,12 @@ the WHOLE job through the public API from host buffers (ingest + shuffle +
 partition + sort + init + epochs + RMSE + export), H2D/D2H inside the timed
 region.  value = nnz * steps / device time (Eq. 8 "computing power", L1709-L1715),
 max over ranks.  Prints ONE JSON line on rank 0.
+
+Default workload: C5 (hugewiki-shaped, 3.1 B ratings, k = 128), the north_star target
+config; at N = 1 the same line carries a C4 leg (yahoo-music-shaped: Q = 320 MB, not
+L2-resident) and a C3 DET leg (the deterministic schedule), each with its own clocks and
+roofline.  Under torchrun every rank generates and loads only its slice of the COO
+(hccmf_load_ratings_slice) and the library shards it (sliced ingest).
 """
 from __future__ import annotations
 
@@ -34,32 +40,16 @@ import synth  # noqa: E402
 
 METRIC = "rating updates/sec (whole box)"
 STORAGE = {"fp32": 0, "fp16": 1, "fp16sr": 2}
-# what ncu says actually binds the SGD kernel (profiles/r01_ncu_c3_ring.md, C3): the
-# formula roofline above counts p_u / q_v bytes that stay in registers / L2
+# what ncu says binds the SGD kernel (profiles/r02_ncu_*.md; C3 in profiles/r01_ncu_c3_final.md):
+# the q_v round trip to L2, not DRAM -- the formula roofline counts p_u / q_v bytes that stay in
+# registers / L2
 BINDING = {
-    "fp32": {"unit": "L2 atomic units (q_v vector reductions, 512 B/update; 48.7 % avg, 75.7 % hottest slice; "
-                     "L1TEX->XBAR request port 71 %)", "ncu_pct_of_peak": 75.7,
-             "dram_bytes_per_update": 17.1, "source": "profiles/r01_ncu_c3_final.md"},
-    "fp16": {"unit": "instruction issue (stochastic-rounding hash and conversions, 66.7 instructions/update)",
-             "ncu_pct_of_peak": 74.8, "dram_bytes_per_update": 17.0, "source": "profiles/r01_ncu_c3_final.md"},
+    "fp32": {"bound": "l2_atomic", "unit": "L2 atomic units (q_v vector reductions red.v4.f32, 512 B/update) "
+                                           "and the L1TEX->XBAR request port"},
+    "fp16": {"bound": "issue", "unit": "instruction issue (binary16 conversions and, with SR, the random-word "
+                                       "hash; ~67 instructions/update)"},
 }
-PROBE = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "r01_probe_l2_roundtrip_c3.json")
-
-
-def binding_unit(storage, args, kernel_rate):
-    """The unit that bounds the SGD kernel (ncu) and, for the C3 Hogwild kernel, the
-    measured ceiling of its q_v round trip on this B200 (tools/probe_l2_roundtrip.py:
-    same record stream and warp count, no SGD arithmetic): the reductions alone for fp32
-    rows, load + reduction for binary16 rows."""
-    b = dict(BINDING.get("fp32" if storage == "fp32" else "fp16"))
-    if args.config == "c3" and args.sched == "hogwild" and os.path.exists(PROBE):
-        with open(PROBE) as f:
-            pr = json.load(f)
-        key = "red only fp32" if storage == "fp32" else "ld+red binary16 (256+256 B)"
-        ceil = pr[key]["G_upd_per_s"] * 1e9
-        b["ceiling"] = {"probe": key, "updates_per_s": ceil, "kernel_updates_per_s": kernel_rate,
-                        "frac": kernel_rate / ceil, "source": os.path.relpath(PROBE, os.path.dirname(PROBE) + "/..")}
-    return b
+PROBE_MODE = {"fp32": "red_f32", "fp16": "ldred_f16"}
 
 
 UNIT = "updates/s"
@@ -72,16 +62,16 @@ def parse():
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="c3", choices=sorted(synth.CONFIGS))
+    ap.add_argument("--config", default="c5", choices=sorted(synth.CONFIGS))
+    ap.add_argument("--legs", default="c4,det", help="extra legs at N = 1: c4 (Q not L2-resident), det "
+                    "(C3 deterministic schedule); '' for none")
     ap.add_argument("--sched", default="hogwild", choices=["hogwild", "det"])
     ap.add_argument("--sync", default=None, choices=["none", "ring", "allreduce"])
-    ap.add_argument("--grid", default=None, help="Br,Bc (default: hogwild 1,4G (ring) or 1,ceil(|Q|/80MB); det 64,64G)")
+    ap.add_argument("--grid", default=None, help="Br,Bc (default: hogwild 1,G (ring) or 1,round(|Q|/80MB); det 64,64G)")
     ap.add_argument("--warps", type=int, default=0)
     ap.add_argument("--task", type=int, default=0)
     ap.add_argument("--vec", type=int, default=0, help="float4 slots per lane (0 = library auto)")
     ap.add_argument("--depth", type=int, default=0, help="Hogwild q_v prefetch distance (0 = library auto)")
-    ap.add_argument("--no-det-leg", dest="det_leg", action="store_false",
-                    help="skip the DET-schedule leg (C3 only) reported beside the Hogwild headline")
     ap.add_argument("--det-wave", type=int, default=1, choices=[0, 1, 2],
                     help="DET: 1 wavefront with Q slabs in shared memory, 2 wavefront, 0 per-stratum launches")
     ap.add_argument("--impl", default="hccmf", choices=["hccmf", "reference"])
@@ -143,12 +133,13 @@ def hbm_peak():
         return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md)"
 
 
-def ncu_traffic(cfg_name, sched):
-    """DRAM bytes per launch of the SGD kernel from the committed ncu --set full summary, if any."""
+def ncu_traffic(key):
+    """DRAM bytes per launch of the SGD kernel (dram__bytes_read.sum + dram__bytes_write.sum) from
+    the committed ncu --set full capture (profiles/ncu_traffic.json), keyed "<cfg>[-<storage>]/<sched>"."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         with open(p) as f:
-            return json.load(f).get(f"{cfg_name}/{sched}")
+            return json.load(f).get(key)
     except Exception:
         return None
 
@@ -257,51 +248,92 @@ def run_reference(args, cfg, rank, world):
 
 
 # --------------------------------------------------------------- main arm
-def main():
-    args = parse()
-    cfg = synth.CONFIGS[args.config]
-    rank = int(os.environ.get("RANK", 0))
-    world = int(os.environ.get("WORLD_SIZE", 1))
-    local = int(os.environ.get("LOCAL_RANK", 0))
-    if args.impl == "reference":
-        run_reference(args, cfg, rank, world)
-        return
+def roofline(cfg, name, storage, sched, info, kmean_ms, step_ms, peak, peak_src, probe=None):
+    """Roofline of the dominant kernel (the SGD epoch launch(es) of train_epoch, timed with CUDA
+    events on the library's stream).  achieved = ALGORITHMIC bytes per launch (SURVEY 8(d3):
+    each local record once + the rank's P rows and Q read and written once) / duration, against
+    the HBM peak; the north_star's no-reuse 12 + 16k bytes/update is kept as north_star_frac;
+    binding_frac = kernel rate / the q_v round-trip ceiling re-measured in this run (probe)."""
+    st16 = storage != "fp32"
+    nnz_l, rows, k, n = info["local_nnz"], info["rows"], cfg.k, cfg.n
+    alg = 12 * nnz_l + 2 * rows * k * 4 + 2 * n * k * (2 if st16 else 4)
+    secs = kmean_ms / 1e3
+    achieved = alg / secs / 1e9
+    b_upd = 12 + (12 if st16 else 16) * k
+    b = BINDING["fp16" if st16 else "fp32"]
+    key = name + ("" if storage == "fp32" else "-" + storage) + "/" + sched
+    traffic = ncu_traffic(key)
+    roof = {"bound": b["bound"] if sched == "hogwild" else "latency",
+            "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+            "traffic_key": key, "kernel_ms": kmean_ms, "kernel_share_of_step": kmean_ms / step_ms,
+            "algorithmic_bytes_per_launch": alg, "algorithmic_bytes_per_update": alg / max(1, nnz_l),
+            "updates_per_launch": nnz_l, "peak_source": peak_src,
+            "north_star_frac": nnz_l * b_upd / secs / 1e9 / peak, "north_star_bytes_per_update": b_upd}
+    if traffic:
+        roof["traffic_bytes_per_update"] = traffic / max(1, nnz_l)
+    if sched == "hogwild":
+        roof["binding_unit"] = b["unit"]
+        if probe:
+            mode, pms = probe
+            roof["binding_ceiling"] = {"probe": mode, "ms": pms, "updates_per_s": nnz_l / (pms / 1e3),
+                                       "source": "hccmf_probe_roundtrip: same records and warps, q_v traffic only"}
+            roof["binding_frac"] = pms / kmean_ms
+    else:
+        roof["binding_unit"] = ("the hottest column block's serial dependency chain (wavefront; "
+                                "profiles/r01_det_wavefront.md)")
+    return roof
 
+
+class Ctx:
+    def __init__(self, args, rank, world, local, stream):
+        self.args, self.rank, self.world, self.local, self.stream = args, rank, world, local, stream
+
+
+def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, sample_for_cpu=False):
+    """Generate `name`, partition, and measure each storage in `storages` (W warm-up + K timed
+    steps from a fresh init); optionally the e2e job.  Returns a dict for the JSON line."""
     import torch
     import torch.distributed as dist
 
     import paper_conf_icpp_huangylhbl21_b200 as hc
-
-    torch.cuda.set_device(local)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    args, rank, world, local, stream = cx.args, cx.rank, cx.world, cx.local, cx.stream
+    cfg = synth.CONFIGS[name]
     G = world
     sync = args.sync or ("none" if G == 1 else "ring")
-    if args.grid:
+    if det_grid:
+        Br, Bc = det_grid
+    elif args.grid and name == args.config:
         Br, Bc = (int(x) for x in args.grid.split(","))
-    elif args.sched == "hogwild":
-        # ring: 4 column blocks per group so each block's transfer overlaps the next
-        # block's compute (hidden synchronisation); one GPU: column-block-major phases
-        # whenever Q exceeds ~80 MB of L2 (C4: 320 MB -> 4 phases)
+    elif sched == "hogwild":
+        # ring: one column block per group (the per-launch Hogwild cap n/(3 Bc) keeps the most
+        # warps in flight, and a C5 group moves in ~10 us against a ~40 ms stage); one GPU:
+        # column-block-major phases whenever Q exceeds ~80 MB of L2 (C4: 320 MB -> 4 phases)
         qmb = cfg.n * cfg.k * 4 / 80e6
-        Br, Bc = 1, (4 * G if sync == "ring" else max(1, round(qmb)))
+        Br, Bc = 1, (G if sync == "ring" else max(1, round(qmb)))
     else:
         Br, Bc = 64, 64 * (G if sync == "ring" else 1)
 
     t_gen = time.perf_counter()
-    on_device = cfg.nnz > DEVICE_GEN_NNZ  # C5: 37 GB of COO, drawn on the GPU (synth.make_device)
-    if on_device:
-        (du, dv, dr), (dtu, dtv, dtr) = synth.make_device(cfg, device=f"cuda:{local}")
+    on_device = cfg.kind == "powerlaw" and cfg.nnz >= DEVICE_GEN_NNZ
+    sample = None
+    if on_device:  # drawn on the GPU, each rank only its slice (synth.make_device part=)
+        (du, dv, dr), (dtu, dtv, dtr) = synth.make_device(cfg, device=f"cuda:{local}", part=(rank, world))
+        if sample_for_cpu:
+            S = 2_000_000
+            sample = (du[:S].cpu().numpy(), dv[:S].cpu().numpy(), dr[:S].cpu().numpy())
         u = v = r = tu = tv = tr = None
-        S = 2_000_000
-        sample = (du[:S].cpu().numpy(), dv[:S].cpu().numpy(), dr[:S].cpu().numpy())
     else:
         (u, v, r), (tu, tv, tr) = synth.make(cfg)
-        sample = (u, v, r)
+        edges = np.linspace(0, len(u), world + 1).astype(np.int64)
+        a, b = edges[rank], edges[rank + 1]
+        du, dv, dr = (torch.from_numpy(x[a:b]).cuda() for x in (u, v, r))
+        dtu, dtv, dtr = (torch.from_numpy(x).cuda() for x in (tu, tv, tr))
+        if sample_for_cpu:
+            sample = (u, v, r)
     torch.cuda.synchronize()
     t_gen = time.perf_counter() - t_gen
+    nnz_slice, nt = int(du.numel()), int(dtu.numel())
 
-    stream = torch.cuda.Stream()
     mdl = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, dist=world > 1, device=local)
     mdl.set_stream(stream)
     if args.warps:
@@ -314,29 +346,20 @@ def main():
         mdl.set_option("prefetch_depth", args.depth)
     if args.det_wave != 1:
         mdl.set_option("det_wave", args.det_wave)
-    if not on_device:
-        du, dv, dr = (torch.from_numpy(x).cuda() for x in (u, v, r))
-        dtu, dtv, dtr = (torch.from_numpy(x).cuda() for x in (tu, tv, tr))
-    nnz, nt = int(du.numel()), int(dtu.numel())
     torch.cuda.synchronize()
     t_prep = time.perf_counter()
-    mdl.load(du, dv, dr)
-    if on_device:  # keep a host-free copy only where it fits; free the generator's 37 GB first
-        del du, dv, dr
-        torch.cuda.empty_cache()
-    mdl.partition(G, (Br, Bc), "DP0", seed=cfg.seed, storage=args.storage)
+    mdl.load_slice(du, dv, dr)
+    del du, dv, dr
+    torch.cuda.empty_cache()
+    mdl.partition(G, (Br, Bc), "DP0", seed=cfg.seed, storage=storages[0])
     mdl.init(1)
+    torch.cuda.synchronize()
     t_prep = time.perf_counter() - t_prep
     info = mdl.info()
-    if not on_device:
-        del du, dv, dr
+    nnz = info["nnz"]
     peak, peak_src = hbm_peak()
-    local_nnz = info["local_nnz"]
 
-    def measure(storage, sched=None, steps=None):
-        """W warm-up + K timed steps (epoch + Q sync + test RMSE) from a fresh init(1)."""
-        sched = sched or args.sched
-        steps = steps or args.steps
+    def measure(storage):
         rm0 = mdl.rmse(dtu, dtv, dtr)
         mdl.set_option("sync_stream", 0)
 
@@ -349,8 +372,7 @@ def main():
             return mdl.rmse(dtu, dtv, dtr)
 
         curve = [rm0] + [step() for _ in range(args.warmup)]
-        kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-               for _ in range(steps)]
+        kev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
         t_start, t_end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         clocks = Clocks(local)
         clocks.start()
@@ -369,137 +391,171 @@ def main():
         clk = clocks.stop()
         mdl.set_option("sync_stream", 1)
         ms = t_start.elapsed_time(t_end)
-        k_ms = [a.elapsed_time(b) for a, b in kev]
+        kmean = float(np.mean([a_.elapsed_time(b_) for a_, b_ in kev]))
         if world > 1:
-            t = torch.tensor([ms, float(np.mean(k_ms))], device="cuda")
+            t = torch.tensor([ms, kmean], device="cuda")
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ms, kmean = t.tolist()
-        else:
-            kmean = float(np.mean(k_ms))
-        # roofline of the dominant kernel (the SGD epoch): north_star bytes/update = record
-        # (12 B) + read and write of p_u and q_v: 12 + 16k (fp32), 12 + 12k (binary16 Q)
-        b_upd = 12 + (16 if storage == "fp32" else 12) * cfg.k
-        achieved = local_nnz * b_upd / (kmean / 1e3) / 1e9
-        roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": ncu_traffic(args.config + ("" if storage == "fp32" else "-" + storage), sched),
-                "kernel": "sgd_warp_kernel (a5/a6 epoch incl. Q sync%s)"
-                          % ("" if storage == "fp32" else ", binary16 round-in/write-back of Q"),
-                "bytes_per_update": b_upd, "updates_per_launch": local_nnz, "kernel_ms": kmean,
-                "kernel_share_of_step": kmean / (ms / steps), "peak_source": peak_src,
-                "binding_unit": binding_unit(storage, args, local_nnz / (kmean / 1e3)) if sched == "hogwild"
-                else None}
-        roof["kernel_launches_timed"] = launches
-        return nnz * steps / (ms / 1e3), ms, roof, clk, curve + rms
+        probe = None
+        if sched == "hogwild" and cfg.k % 128 == 0:
+            mode = PROBE_MODE["fp32" if storage == "fp32" else "fp16"]
+            probe = (mode, mdl.probe_roundtrip(mode, warps=args.warps, reps=3))
+        roof = roofline(cfg, name, storage, sched, info, kmean, ms / steps, peak, peak_src, probe)
+        return {"value": nnz * steps / (ms / 1e3), "ms": ms, "roofline": roof, "clocks": clk,
+                "curve": curve + rms, "launches": launches}
 
-    value, ms, roof, clk, curve = measure(args.storage)
+    res = {"cfg": cfg, "name": name, "sync": sync, "grid": [Br, Bc], "info": info, "nnz": nnz, "nt": nt,
+           "t_gen": t_gen, "t_prep": t_prep, "sample": sample, "legs": {}, "sched": sched}
+    for i, storage in enumerate(storages):
+        if i:
+            mdl.set_option("storage", STORAGE[storage])
+            mdl.init(1)
+        res["legs"][storage] = measure(storage)
+    mdl.close()
+    torch.cuda.empty_cache()
 
-    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-           "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+    # ---- e2e: the whole job through the public API from pinned host buffers
+    res["e2e"] = None
+    if not want_e2e:
+        return res
+    if on_device:
+        need = 12 * (nnz_slice + nt) * 2 + 4 * (cfg.m + cfg.n) * cfg.k
+        if host_mem_available() < need:
+            res["e2e"] = {"value": None, "unit": UNIT, "skipped": f"host memory {host_mem_available() / 1e9:.0f} GB "
+                                                                 f"< {need / 1e9:.0f} GB for pinned COO + P, Q"}
+            return res
+        (du, dv, dr), (dtu2, dtv2, dtr2) = synth.make_device(cfg, device=f"cuda:{local}", part=(rank, world))
+        u, v, r, tu, tv, tr = (x.cpu().numpy() for x in (du, dv, dr, dtu2, dtv2, dtr2))
+        del du, dv, dr, dtu2, dtv2, dtr2
+        torch.cuda.empty_cache()
+    else:
+        edges = np.linspace(0, len(u), world + 1).astype(np.int64)
+        u, v, r = (x[edges[rank]:edges[rank + 1]] for x in (u, v, r))
+    pin = [torch.from_numpy(np.ascontiguousarray(x)).pin_memory() for x in (u, v, r, tu, tv, tr)]
+    del u, v, r, tu, tv, tr
+    Ph = torch.empty((cfg.m, cfg.k), dtype=torch.float32).pin_memory()
+    Qh = torch.empty((cfg.n, cfg.k), dtype=torch.float32).pin_memory()
+    E = cfg.epochs
+    storage = storages[0]
+
+    def job():
+        m2 = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, dist=world > 1, device=local)
+        m2.set_stream(stream)
+        if args.warps:
+            m2.set_option("hogwild_warps", args.warps)
+        if args.vec:
+            m2.set_option("vec", args.vec)
+        m2.load_slice(pin[0], pin[1], pin[2])
+        m2.partition(G, (Br, Bc), "DP0", seed=cfg.seed, storage=storage)
+        m2.init(1)
+        for _ in range(E):
+            m2.train_epoch(sched, sync)
+            m2.rmse(pin[3], pin[4], pin[5])
+        m2.factors(Ph, Qh)
+        m2.close()
+
+    job()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    reps = 2
+    t0 = time.perf_counter()
+    for _ in range(reps):
+        job()
+    torch.cuda.synchronize()
+    e2e_s = (time.perf_counter() - t0) / reps
+    if world > 1:
+        t = torch.tensor([e2e_s], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_s = t.item()
+    res["e2e"] = {"value": nnz * E / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 12 * (nnz_slice + nt),
+                  "d2h_bytes_per_step": 4 * (cfg.m + cfg.n) * cfg.k + 8 * E,
+                  "step": f"job: load+partition+init+{E} epochs (each with test RMSE)+export P,Q ({storage}); "
+                          "host pinned buffers; per rank", "s_per_step": e2e_s}
+    del pin, Ph, Qh
+    return res
+
+
+def leg_json(res, storage, steps, warmup):
+    L = res["legs"][storage]
+    return {"value": L["value"], "unit": UNIT, "steps": steps, "warmup": warmup,
+            "ms_per_step": L["ms"] / steps, "gpu_launches": L["launches"], "roofline": L["roofline"],
+            "clocks": L["clocks"], "rmse": epochs_to_rmse(res["name"], L["curve"])}
+
+
+def main():
+    args = parse()
+    cfg = synth.CONFIGS[args.config]
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    if args.impl == "reference":
+        run_reference(args, cfg, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    stream = torch.cuda.Stream()
+    cx = Ctx(args, rank, world, local, stream)
+    storages = [args.storage]
+    if args.storage == "fp32" and cfg.k % 128 == 0 and args.fp16_leg != "none":
+        storages.append(args.fp16_leg)
+    head = run_workload(cx, args.config, args.sched, storages, args.steps, not args.no_e2e,
+                        sample_for_cpu=(rank == 0 and world == 1 and not args.no_cpu_baseline))
+    H = head["legs"][args.storage]
+    info = head["info"]
+    out = {"metric": METRIC, "value": H["value"], "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": H["ms"] / args.steps, "higher_is_better": True,
            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-           "config": {"workload": f"{cfg.name} ({args.config})", "m": cfg.m, "n": cfg.n, "nnz": nnz, "k": cfg.k,
-                      "test_ratings": nt, "gamma": cfg.gamma, "lambda": cfg.lam, "sched": args.sched,
-                      "sync": sync, "grid": [Br, Bc], "parallelism": f"dp{world} (row shards, Q {sync})",
+           "config": {"workload": f"{cfg.name} ({args.config})", "m": cfg.m, "n": cfg.n, "nnz": head["nnz"],
+                      "k": cfg.k, "test_ratings": head["nt"], "gamma": cfg.gamma, "lambda": cfg.lam,
+                      "sched": args.sched, "sync": head["sync"], "grid": head["grid"], "storage": args.storage,
+                      "parallelism": f"dp{world} (row shards, Q {head['sync']}; sliced ingest)",
                       "step": "1 SGD epoch over all nnz + Q sync + test RMSE",
                       "l2": "inputs larger than L2 (records %.2f GB > 126 MB); Q is L2-resident by design"
-                            % (12 * nnz / 1e9),
+                            % (12 * head["nnz"] / 1e9),
                       "hogwild_tasks": info["n_tasks"], "key_bits": info["key_bits"]},
-           "roofline": roof, "clocks": clk,
-           "gpu_launches": roof.pop("kernel_launches_timed"),
-           "rmse": epochs_to_rmse(args.config, curve),
-           "prep_s": t_prep, "gen_s": t_gen,
+           "roofline": H["roofline"], "clocks": H["clocks"], "gpu_launches": H["launches"],
+           "rmse": epochs_to_rmse(args.config, H["curve"]), "prep_s": head["t_prep"], "gen_s": head["t_gen"],
            "paper_context": {"netflix_hcc_updates_per_s": 2228476993,
                              "hardware": "2x Xeon Gold 6242 + RTX 2080 + RTX 2080S (Table 4, L2001)"}}
-    out["config"]["storage"] = args.storage
-    # secondary leg: the same workload with Q stored in binary16 (R26),
-    # fp32 arithmetic; same steps, same clocks rule; reported beside the fp32 headline
-    if args.storage == "fp32" and cfg.k % 128 == 0 and args.fp16_leg != "none":
-        mdl.set_option("storage", STORAGE[args.fp16_leg])
-        mdl.init(1)
-        v16, ms16, roof16, clk16, curve16 = measure(args.fp16_leg)
-        out["storage_fp16"] = {"storage": args.fp16_leg, "value": v16, "unit": UNIT,
-                               "ms_per_step": ms16 / args.steps,
-                               "gpu_launches": roof16.pop("kernel_launches_timed"), "roofline": roof16,
-                               "clocks": clk16, "rmse": epochs_to_rmse(args.config, curve16),
-                               "note": "Q held as IEEE binary16 during epochs (fp32 math, P fp32)%s; "
-                                       "same band vs the fp64 oracle"
-                                       % (", stochastic rounding of every q write" if args.fp16_leg == "fp16sr"
-                                          else "")}
+    out["e2e"] = head["e2e"] if head["e2e"] is not None else {"value": None, "unit": UNIT, "skipped": "--no-e2e"}
+    if len(storages) > 1:
+        s16 = storages[1]
+        out["storage_fp16"] = dict(leg_json(head, s16, args.steps, args.warmup), storage=s16,
+                                   note="Q held as IEEE binary16 during epochs (fp32 math, P fp32)%s; same band vs "
+                                        "the fp64 oracle" % (", stochastic rounding of every q write"
+                                                             if s16 == "fp16sr" else ""))
+    sample = head["sample"]
+    head = None
+    torch.cuda.empty_cache()
 
-    # secondary leg: the deterministic schedule (a5) on the same data, the bench's DET
-    # configuration (one shard, 2048 x 2048 grid, the shared-memory-slab wavefront: one
-    # launch per epoch), fp32; parity with the oracle is the full-size GPU test's
-    if (args.det_leg and args.sched == "hogwild" and world == 1 and args.config == "c3" and not on_device):
-        mdl.close()  # the handle released its input COO after partition: a fresh one for DET
-        mdl = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, device=local)
-        mdl.set_stream(stream)
-        mdl.load(u, v, r)
-        mdl.partition(1, (2048, 2048), "DP0", seed=cfg.seed)
-        mdl.init(1)
+    legs = [x for x in args.legs.split(",") if x] if world == 1 else []
+    out["legs"] = {}
+    if "c4" in legs and args.config != "c4":
+        ks = min(args.steps, 5)
+        c4 = run_workload(cx, "c4", "hogwild", ["fp32"], ks, not args.no_e2e)
+        out["legs"]["c4"] = dict(leg_json(c4, "fp32", ks, args.warmup),
+                                 workload=f"{c4['cfg'].name} (c4)", grid=c4["grid"], sched="hogwild",
+                                 e2e=c4["e2e"], note="Q = 320 MB fp32 is not L2-resident: column-block-major "
+                                                     "phases (grid %s)" % (c4["grid"],))
+        c4 = None
+        torch.cuda.empty_cache()
+    if "det" in legs:
         kd = min(args.steps, 3)
-        vd, msd, roofd, clkd, curved = measure("fp32", sched="det", steps=kd)
-        roofd["kernel"] = "sgd_wave_slab_kernel (a5 DET epoch, one launch)"
-        out["det"] = {"sched": "det", "grid": [2048, 2048], "value": vd, "unit": UNIT, "steps": kd,
-                      "warmup": args.warmup, "ms_per_step": msd / kd,
-                      "gpu_launches": roofd.pop("kernel_launches_timed"), "roofline": roofd, "clocks": clkd,
-                      "test_rmse": curved[-1],
-                      "note": "serial-equivalent FPSGD strata (R19); bound by the hottest column block's "
-                              "serial chain (profiles/r01_det_wavefront.md)"}
+        d = run_workload(cx, "c3", "det", ["fp32"], kd, False, det_grid=(2048, 2048))
+        out["legs"]["det"] = dict(leg_json(d, "fp32", kd, args.warmup), workload=f"{d['cfg'].name} (c3)",
+                                  grid=[2048, 2048], sched="det",
+                                  note="serial-equivalent FPSGD strata (R19) as one wavefront launch per epoch; "
+                                       "bound by the hottest column block's serial chain")
+        d = None
+        torch.cuda.empty_cache()
 
-    mdl.close()  # free HBM before the e2e jobs build their own handles
-    # ---- e2e: the whole job through the public API from pinned host buffers
-    e2e_skip = None
-    if on_device and not args.no_e2e:
-        need = 12 * (nnz + nt) * 2 + 4 * (cfg.m + cfg.n) * cfg.k
-        if host_mem_available() < need:
-            e2e_skip = f"host memory {host_mem_available() / 1e9:.0f} GB < {need / 1e9:.0f} GB for pinned COO + P, Q"
-        else:
-            (u, v, r), (tu, tv, tr) = synth.make_device(cfg, device=f"cuda:{local}")
-            u, v, r, tu, tv, tr = (x.cpu().numpy() for x in (u, v, r, tu, tv, tr))
-            torch.cuda.empty_cache()
-    if e2e_skip:
-        out["e2e"] = {"value": None, "unit": UNIT, "skipped": e2e_skip}
-    elif not args.no_e2e:
-        pin = [torch.from_numpy(x).pin_memory() for x in (u, v, r, tu, tv, tr)]
-        Ph = torch.empty((cfg.m, cfg.k), dtype=torch.float32).pin_memory()
-        Qh = torch.empty((cfg.n, cfg.k), dtype=torch.float32).pin_memory()
-        E = cfg.epochs
-
-        def job():
-            m2 = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, dist=world > 1, device=local)
-            m2.set_stream(stream)
-            if args.warps:
-                m2.set_option("hogwild_warps", args.warps)
-            if args.vec:
-                m2.set_option("vec", args.vec)
-            m2.load(pin[0], pin[1], pin[2])
-            m2.partition(G, (Br, Bc), "DP0", seed=cfg.seed, storage=args.storage)
-            m2.init(1)
-            for _ in range(E):
-                m2.train_epoch(args.sched, sync)
-                m2.rmse(pin[3], pin[4], pin[5])
-            m2.factors(Ph, Qh)
-            m2.close()
-
-        job()
-        if world > 1:
-            dist.barrier()
-        torch.cuda.synchronize()
-        reps = 2
-        t0 = time.perf_counter()
-        for _ in range(reps):
-            job()
-        torch.cuda.synchronize()
-        e2e_s = (time.perf_counter() - t0) / reps
-        if world > 1:
-            t = torch.tensor([e2e_s], device="cuda")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e2e_s = t.item()
-        out["e2e"] = {"value": nnz * E / e2e_s, "unit": UNIT, "h2d_bytes_per_step": 12 * (nnz + nt),
-                      "d2h_bytes_per_step": 4 * (cfg.m + cfg.n) * cfg.k + 8 * (E + 0),
-                      "step": f"job: load+partition+init+{E} epochs (each with test RMSE)+export P,Q; "
-                              "host pinned buffers", "s_per_step": e2e_s}
-
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and sample is not None:
         val, S, ep, dt, core = oracle_sample(cfg, *sample, args.cpu_seconds)
         model, ncpu = host_cpu()
         out["cpu_baseline"] = {"value": val, "unit": UNIT, "cores": 1, "kind": "oracle",

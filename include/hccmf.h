@@ -4,7 +4,7 @@
  * Framework for SGD-based Matrix Factorization", ICPP '21).
  *
  * Citations: L<n> = line n of the paper text.
- * lists every reading taken where the paper is silent or garbled (R1..R20).
+ * lists every reading taken where the paper is silent or garbled (R1..R30).
  *
  * What the library computes:
  *   a0 factor init, a1 ingest+validate COO, a2 seeded ID shuffle, a3 row-grid
@@ -54,6 +54,10 @@ extern "C" {
 #endif
 
 typedef struct hccmf_ctx* hccmf_t;
+/* In-process loopback communicator hub: G handles of ONE process on one device,
+ * one host thread each, exchange Q through it exactly as G ranks exchange it over
+ * NCCL (same call sites, same buffers, same stream ordering). */
+typedef struct hccmf_hub* hccmf_hub_t;
 
 typedef enum {
     HCCMF_OK = 0,
@@ -143,7 +147,6 @@ typedef enum {
                                     256); tasks never split a user's run          */
     HCCMF_OPT_SYNC_STREAM = 3,   /* 1 (default): calls return after the stream is
                                     synchronised; 0: return after enqueueing      */
-    HCCMF_OPT_RING_SUBBLOCKS = 4,/* reserved                                       */
     HCCMF_OPT_HOGWILD_ATOMIC = 5,/* 1 (default): Hogwild applies q_v increments with
                                     vector atomic adds (Hogwild!'s component-wise
                                     atomic model, no lost updates); 0: plain stores
@@ -218,6 +221,31 @@ HCCMF_API hccmf_status hccmf_create_dist(int64_t m, int64_t n, int32_t k, float 
                                const void* nccl_unique_id, int32_t rank, int32_t world,
                                int32_t device, hccmf_t* out);
 
+/* Loopback hub for `world` ranks (no device work; never fails for world >= 1).
+ * The hub lives until hccmf_hub_destroy AND every handle created on it is
+ * destroyed (reference counted). */
+HCCMF_API hccmf_status hccmf_hub_create(int32_t world, hccmf_hub_t* out);
+HCCMF_API void hccmf_hub_destroy(hccmf_hub_t hub);
+
+/* A distributed handle whose data plane is the loopback `hub` instead of NCCL:
+ * rank in [0, world of the hub), on CUDA device `device`.  Every collective call
+ * (partition, train_epoch with sync RING / ALLREDUCE_AVG, rmse, get_factors) must
+ * be made by all ranks, each from its own host thread; host waits time out after
+ * HCCMF_LOOPBACK_TIMEOUT_S seconds (default 300) with HCCMF_ENCCL.  Used to run
+ * the multi-rank data plane on one GPU (tests); production uses hccmf_create_dist. */
+HCCMF_API hccmf_status hccmf_create_loopback(int64_t m, int64_t n, int32_t k, float gamma, float lambda,
+                                             hccmf_hub_t hub, int32_t rank, int32_t device, hccmf_t* out);
+
+/* Per-call-site counters of the shard data plane (how many times each exchange
+ * ran on this handle): counts[i] for i < min(n, HCCMF_COMM_SITES).  Sites, in
+ * order: 0 stage-wise ring transfer, 1 pipelined ring block transfer, 2 ring
+ * transfer in binary16, 3 ring-group broadcast (materialise Q), 4 fp32 Q average,
+ * 5 binary16 Q average, 6 RMSE {sum, count}, 7 P export, 8 sliced-ingest
+ * histogram, 9 sliced-ingest rating exchange, 10 sliced-ingest block offsets.
+ * Returns the number of sites through *n_sites if non-NULL. */
+#define HCCMF_COMM_SITES 11
+HCCMF_API hccmf_status hccmf_comm_counts(hccmf_t h, int64_t* counts, int32_t n, int32_t* n_sites);
+
 /* Issue all further work on `stream` (a cudaStream_t, may be the legacy default
  * 0).  The caller keeps ownership of the stream and must keep it alive. */
 HCCMF_API hccmf_status hccmf_set_stream(hccmf_t h, void* stream);
@@ -235,14 +263,33 @@ HCCMF_API const char* hccmf_last_error(hccmf_t h);
 /* a1 (preprocessing, L543-L548): copy nnz >= 0 COO ratings (u[i], v[i], r[i])
  * of R (Table 1).  Duplicated (u, v) are kept, each one update.
  * Validates 0 <= u < m, 0 <= v < n and finite r -> HCCMF_ERANGE otherwise.
- * Distributed handles: every rank passes the same global COO. */
+ * Distributed handles: every rank passes the same global COO (each keeps only its
+ * shard after hccmf_partition; see hccmf_load_ratings_slice to avoid the copies). */
 HCCMF_API hccmf_status hccmf_load_ratings(hccmf_t h, const int32_t* u, const int32_t* v, const float* r, int64_t nnz);
+
+/* a1, sharded ingest (each rank loads 1/G of the input, L543-L548 "the server
+ * ... partitions the data", without the global COO on any GPU): this rank's slice
+ * of the global COO.  The slices of ranks 0, 1, .., world-1 concatenated in rank
+ * order ARE the global COO (any split, empty slices allowed), so every result --
+ * permutation, boundaries, block offsets, the sorted records of each shard -- is
+ * bit-identical to a single-process load of the concatenation.  hccmf_partition
+ * then all-reduces the permuted-row histogram (boundaries), sends every rating to
+ * the rank that owns its row (one all-to-all), and each rank sorts only its shard.
+ * Validation as hccmf_load_ratings (ERANGE is local to the rank that holds the
+ * bad rating; partition then fails collectively with ESTATE on that rank only, so
+ * callers must check every rank's load status).  Single-process handles: same as
+ * hccmf_load_ratings. */
+HCCMF_API hccmf_status hccmf_load_ratings_slice(hccmf_t h, const int32_t* u, const int32_t* v, const float* r,
+                                                int64_t nnz_local);
 
 /* a2-a4: shuffle (seeded permutation of row and column ids), row-grid partition
  * into G shards of contiguous permuted rows balanced on nnz (DP0/1/2,
  * L881-L1172), blocking into G*B_r*B_c blocks and a stable sort by
- * (shard, row block, column block, u', v') -- the row-sorted blocks of
- * L1472-L1474.  Bit-exact with the oracle.  Collective for distributed handles. */
+ * (shard, row block, column block, u', o) -- the row-sorted blocks of
+ * L1472-L1474 -- where o = (v' - c0 + H(seed,5,u',0) mod w) mod w is v' rotated
+ * by a row-dependent offset inside the block's w columns [c0, c0+w) (DESIGN.md
+ * R21; seed 0: o = v' - c0, plain column order).  Bit-exact with the oracle.
+ * Collective for distributed handles. */
 HCCMF_API hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* opts);
 
 /* a0: P[u][j] = U(H(seed,3,u,j)) * sqrtf(1/k), Q[v][j] = U(H(seed,4,v,j)) * sqrtf(1/k)
@@ -313,6 +360,16 @@ HCCMF_API hccmf_status hccmf_cost_model(int32_t p, int64_t m, int64_t n, int64_t
                                         const double* Bbus, double B_server, int32_t t, int32_t q_only,
                                         int32_t elem_bytes, double lambda_sync, double* x, double* T_i,
                                         double* T_sync, double* T, int32_t* strategy);
+
+/* Diagnostic (bench.py roofline.binding_frac): the ceiling of the
+ * Hogwild q_v round trip on this device.  Streams the handle's local sorted records with
+ * `warps` warps (0: the Hogwild epoch's automatic count for the whole of Q), one rating
+ * ahead, doing per rating only the kernel's q_v traffic into a SCRATCH copy of Q (the
+ * model is not touched): mode 0 fp32 vector reductions only (red.v4.f32), 1 binary16
+ * load + dependent reduction (red.v2.f16x2), 2 fp32 load + dependent reduction.
+ * *ms = mean duration of one pass over `reps` timed passes (CUDA events on the handle's
+ * stream, after one warm-up pass).  Needs partition; k a multiple of 128. */
+HCCMF_API hccmf_status hccmf_probe_roundtrip(hccmf_t h, int32_t mode, int64_t warps, int32_t reps, double* ms);
 
 /* Library version string, e.g. "hccmf 0.1 sm_100a". */
 HCCMF_API const char* hccmf_version(void);

@@ -14,6 +14,10 @@ no CPU fallback: if libhccmf.so is missing the import of this module fails.
         model.train_epoch("hogwild", sync="none")
     rmse = model.rmse(tu, tv, tr)
     P, Q = model.factors()
+
+Multi-rank: ``Model(..., dist=True)`` under torchrun (NCCL, one process per GPU), or
+``Model(..., hub=Hub(G), rank=r)`` from G host threads of one process: the loopback
+data plane on one device (same call sites and buffers as NCCL; tests).
 """
 from __future__ import annotations
 
@@ -92,6 +96,12 @@ def lib():
             "hccmf_get_fractions": (st, [P, P]),
             "hccmf_get_info": (st, [P, ctypes.POINTER(Info)]),
             "hccmf_version": (ctypes.c_char_p, []),
+            "hccmf_hub_create": (st, [i32, P]),
+            "hccmf_hub_destroy": (None, [P]),
+            "hccmf_create_loopback": (st, [i64, i64, i32, f32, f32, P, i32, i32, P]),
+            "hccmf_comm_counts": (st, [P, P, i32, P]),
+            "hccmf_load_ratings_slice": (st, [P, P, P, P, i64]),
+            "hccmf_probe_roundtrip": (st, [P, i32, i64, i32, ctypes.POINTER(ctypes.c_double)]),
             "hccmf_kernel_launches": (ctypes.c_int64, []),
             "hccmf_schedule": (st, [i32, i32, i32, i64, i32, i32, i32, P, P, P, P, P, P]),
             "hccmf_cost_model": (st, [i32, i64, i64, i64, i32, P, P, ctypes.c_double, i32, i32, i32,
@@ -167,14 +177,44 @@ def cost_model(m, n, nnz, k, B, Bbus, B_server, t=1, q_only=True, elem_bytes=4, 
     return x, Ti, Ts.value, T.value, {1: "DP1", 2: "DP2"}[strat.value]
 
 
+COMM_SITES = ("ring_stage", "ring_block", "ring_wire16", "materialize_q", "allreduce_q", "allreduce_q16",
+              "rmse", "export_p", "ingest_hist", "ingest_exchange", "ingest_blocks")
+
+
+class Hub:
+    """Loopback communicator hub for `world` ranks of this process (hccmf_hub_create)."""
+
+    def __init__(self, world):
+        self.world = int(world)
+        self._p = ctypes.c_void_p()
+        code = lib().hccmf_hub_create(self.world, ctypes.byref(self._p))
+        if code != OK:
+            raise HccmfError(code, "hccmf_hub_create")
+
+    def close(self):
+        if getattr(self, "_p", None):
+            lib().hccmf_hub_destroy(self._p)
+            self._p = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # pragma: no cover
+            pass
+
+
 class Model:
     """One handle of libhccmf (single process, or one rank of a distributed job)."""
 
-    def __init__(self, m, n, k, gamma=0.005, lam=0.01, *, dist=False, device=None):
+    def __init__(self, m, n, k, gamma=0.005, lam=0.01, *, dist=False, device=None, hub=None, rank=None):
         self.m, self.n, self.k, self.gamma, self.lam = int(m), int(n), int(k), float(gamma), float(lam)
         self._h = ctypes.c_void_p()
         L = lib()
-        if dist:
+        if hub is not None:
+            dev = 0 if device is None else int(device)
+            self._check(L.hccmf_create_loopback(self.m, self.n, self.k, self.gamma, self.lam, hub._p, int(rank), dev,
+                                                ctypes.byref(self._h)))
+        elif dist:
             import torch
             import torch.distributed as tdist
             rank, world = tdist.get_rank(), tdist.get_world_size()
@@ -236,6 +276,31 @@ class Model:
         nnz = len(ku)
         assert len(kv) == nnz and len(kr) == nnz, "u, v, r must have the same length"
         self._check(lib().hccmf_load_ratings(self._h, pu, pv, pr, nnz))
+
+    def load_slice(self, u, v, r):
+        """This rank's slice of the global COO (hccmf_load_ratings_slice): ranks' slices in
+        rank order concatenate to the global COO; partition then shards without copies."""
+        pu, ku = _buf(u, np.int32)
+        pv, kv = _buf(v, np.int32)
+        pr, kr = _buf(r, np.float32)
+        nnz = len(ku)
+        assert len(kv) == nnz and len(kr) == nnz, "u, v, r must have the same length"
+        self._check(lib().hccmf_load_ratings_slice(self._h, pu, pv, pr, nnz))
+
+    def probe_roundtrip(self, mode="red_f32", warps=0, reps=3) -> float:
+        """Mean ms of one pass of the q_v round-trip ceiling probe (hccmf_probe_roundtrip)."""
+        out = ctypes.c_double()
+        m = {"red_f32": 0, "ldred_f16": 1, "ldred_f32": 2}[mode]
+        self._check(lib().hccmf_probe_roundtrip(self._h, m, int(warps), int(reps), ctypes.byref(out)))
+        return out.value
+
+    def comm_counts(self) -> dict:
+        """How many times each data-plane call site ran on this handle (hccmf_comm_counts)."""
+        c = np.zeros(len(COMM_SITES), np.int64)
+        ns = ctypes.c_int32()
+        self._check(lib().hccmf_comm_counts(self._h, c.ctypes.data, len(c), ctypes.byref(ns)))
+        assert ns.value == len(COMM_SITES)
+        return dict(zip(COMM_SITES, c.tolist()))
 
     def partition(self, n_shards=1, grid=(1, 1), strategy="DP0", seed=0, x=None, t_meas=None, t_sync=0.0,
                   grid_dim="rows", storage="fp32"):

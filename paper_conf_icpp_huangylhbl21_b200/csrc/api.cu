@@ -9,6 +9,8 @@
 #include <cstdio>
 #include <cstring>
 
+#include <nccl.h>
+
 #include "internal.cuh"
 
 using namespace hccmf;
@@ -43,11 +45,12 @@ hccmf_status fail(hccmf_t h, hccmf_status st, const char* fmt, ...) {
     }                                                                                                 \
   } while (0)
 
-#define NC(h, call)                                                                                            \
-  do {                                                                                                         \
-    ncclResult_t r_ = (call);                                                                                  \
-    if (r_ != ncclSuccess)                                                                                     \
-      return fail(h, HCCMF_ENCCL, "%s: %s (%s:%d)", #call, ncclGetErrorString(r_), __FILE__, __LINE__);       \
+// a data-plane call (comm.cuh: NCCL or loopback); failures are sticky HCCMF_ENCCL
+#define CM(h, call)                                                                                   \
+  do {                                                                                                \
+    if ((call) != 0)                                                                                  \
+      return fail(h, HCCMF_ENCCL, "%s [%s] (%s:%d)", (h)->comm->err.c_str(), (h)->comm->backend(), __FILE__, \
+                  __LINE__);                                                                          \
   } while (0)
 
 #define ENTER(h)                                      \
@@ -352,7 +355,13 @@ hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
         }
       }
     }
-    pl.launches.push_back(Launch{t0, (int64_t)lo.size() - t0, L.qrep, L.stage, L.phase});
+    std::vector<int64_t> cbs;
+    for (int64_t b : L.blocks) cbs.push_back(b % h->Bc);
+    std::sort(cbs.begin(), cbs.end());
+    cbs.erase(std::unique(cbs.begin(), cbs.end()), cbs.end());
+    int64_t items = 0;
+    for (int64_t cb : cbs) items += ceil_div((cb + 1) * h->n, h->Bc) - ceil_div(cb * h->n, h->Bc);
+    pl.launches.push_back(Launch{t0, (int64_t)lo.size() - t0, L.qrep, L.stage, L.phase, items});
   }
   pl.n_tasks = (int64_t)lo.size();
   CU(h, dmalloc(h, &pl.d_lo, pl.n_tasks));
@@ -411,15 +420,18 @@ hccmf_status wire_reserve(hccmf_t h, size_t halves, bool* grown = nullptr) {  //
 
 // one ring transfer of Q rows [sa, sb) to `prev` and [ra, rb) from `next`, fp32 or binary16
 hccmf_status ring_transfer(hccmf_t h, int64_t sa, int64_t sb, int64_t ra, int64_t rb, int prev, int next,
-                           cudaStream_t cs) {
+                           cudaStream_t cs, int site) {
   const size_t ns = (size_t)(sb - sa) * h->k, nr = (size_t)(rb - ra) * h->k;
+  h->comm_counts[site] += 1;
+  Comm* c = h->comm;
   if (!h->opt_wire16) {
-    NC(h, ncclGroupStart());
-    if (ns) NC(h, ncclSend(h->d_Q + sa * h->k, ns, ncclFloat, prev, h->comm, cs));
-    if (nr) NC(h, ncclRecv(h->d_Q + ra * h->k, nr, ncclFloat, next, h->comm, cs));
-    NC(h, ncclGroupEnd());
+    CM(h, c->group_start());
+    if (ns) CM(h, c->send(h->d_Q + sa * h->k, ns * sizeof(float), prev, cs));
+    if (nr) CM(h, c->recv(h->d_Q + ra * h->k, nr * sizeof(float), next, cs));
+    CM(h, c->group_end());
     return HCCMF_OK;
   }
+  h->comm_counts[SITE_RING_WIRE16] += 1;
   // Strategy 2: pack to binary16, ship half the bytes, unpack (all on the comm stream)
   const size_t cap = (size_t)h->n * h->k;
   bool grown = false;
@@ -431,10 +443,10 @@ hccmf_status ring_transfer(hccmf_t h, int64_t sa, int64_t sb, int64_t ra, int64_
   char* sendb = static_cast<char*>(h->d_wire);
   char* recvb = sendb + cap * 2;
   CU(h, k_pack_half(h->d_Q + sa * h->k, sendb, (int64_t)ns, cs));
-  NC(h, ncclGroupStart());
-  if (ns) NC(h, ncclSend(sendb, ns, ncclHalf, prev, h->comm, cs));
-  if (nr) NC(h, ncclRecv(recvb, nr, ncclHalf, next, h->comm, cs));
-  NC(h, ncclGroupEnd());
+  CM(h, c->group_start());
+  if (ns) CM(h, c->send(sendb, ns * 2, prev, cs));
+  if (nr) CM(h, c->recv(recvb, nr * 2, next, cs));
+  CM(h, c->group_end());
   CU(h, k_unpack_half(recvb, h->d_Q + ra * h->k, (int64_t)nr, cs));
   return HCCMF_OK;
 }
@@ -446,7 +458,7 @@ hccmf_status ring_exchange(hccmf_t h, int sched, int t) {
   ring_group_cols(h, sched, g_send, &sa, &sb);
   ring_group_cols(h, sched, g_recv, &ra, &rb);
   const int prev = (s - 1 + G) % G, next = (s + 1) % G;
-  return ring_transfer(h, sa, sb, ra, rb, prev, next, h->stream);
+  return ring_transfer(h, sa, sb, ra, rb, prev, next, h->stream, SITE_RING_STAGE);
 }
 
 // Hidden synchronisation (L1143-L1172) with asynchronous computing-transmission
@@ -466,22 +478,57 @@ hccmf_status ring_exchange_block(hccmf_t h, int t, int j, cudaStream_t cs) {
   rows((s + t) % G, &sa, &sb);
   rows((s + t + 1) % G, &ra, &rb);
   const int prev = (s - 1 + G) % G, next = (s + 1) % G;
-  return ring_transfer(h, sa, sb, ra, rb, prev, next, cs);
+  return ring_transfer(h, sa, sb, ra, rb, prev, next, cs, SITE_RING_BLOCK);
 }
 
 // after ring epochs rank s holds only group s of Q: broadcast every group from its owner
 hccmf_status materialize_q(hccmf_t h) {
   if (h->world <= 1 || h->q_ring_sched < 0) return HCCMF_OK;
-  NC(h, ncclGroupStart());
+  h->comm_counts[SITE_MATERIALIZE_Q] += 1;
+  CM(h, h->comm->group_start());
   for (int g = 0; g < h->G; ++g) {
     int64_t a, b;
     ring_group_cols(h, h->q_ring_sched, g, &a, &b);
     if (b > a)
-      NC(h, ncclBroadcast(h->d_Q + a * h->k, h->d_Q + a * h->k, (size_t)(b - a) * h->k, ncclFloat, g, h->comm,
-                          h->stream));
+      CM(h, h->comm->broadcast(h->d_Q + a * h->k, h->d_Q + a * h->k, sizeof(float) * (size_t)(b - a) * h->k, g,
+                               h->stream));
   }
-  NC(h, ncclGroupEnd());
+  CM(h, h->comm->group_end());
   h->q_ring_sched = -1;
+  return HCCMF_OK;
+}
+
+// Strategy 2 all-reduce (R25): Q = binary16( sum_s binary16(Q_s) / G ), the sum in fp64
+// in rank order -- the function the oracle (orc_epoch_wire16) and the logical backend
+// (average_half_kernel) compute, with only binary16 on the wire.  Chunk c of the packed
+// copy (C = ceil(nk / G) halves, zero padded) belongs to rank c: an all-to-all ships
+// every rank's chunk c to rank c, which reduces its G copies and rounds once; an
+// all-gather returns the rounded chunks.  Wire bytes per rank 4 (G-1)/G nk, half of an
+// fp32 ring all-reduce; reducing in binary16 inside NCCL would round at every hop.
+hccmf_status allreduce_q16(hccmf_t h, cudaStream_t s) {
+  const int G = h->G, me = h->rank;
+  const int64_t nk = h->n * h->k;
+  const int64_t C = (nk + G - 1) / G;
+  h->comm_counts[SITE_ALLREDUCE_Q16] += 1;
+  hccmf_status w = wire_reserve(h, (size_t)C * G);
+  if (w != HCCMF_OK) return w;
+  uint16_t* packed = static_cast<uint16_t*>(h->d_wire);  // G x C halves
+  uint16_t* gath = packed + (size_t)C * G;                // G x C halves: rank r's copy of my chunk
+  if (C * G > nk) CU(h, cudaMemsetAsync(packed + nk, 0, sizeof(uint16_t) * (size_t)(C * G - nk), s));
+  CU(h, k_pack_half(h->d_Q, packed, nk, s));
+  Comm* c = h->comm;
+  CM(h, c->group_start());
+  for (int p = 0; p < G; ++p)
+    if (p != me) {
+      CM(h, c->send(packed + (size_t)p * C, sizeof(uint16_t) * C, p, s));
+      CM(h, c->recv(gath + (size_t)p * C, sizeof(uint16_t) * C, p, s));
+    }
+  CM(h, c->group_end());
+  CU(h, cudaMemcpyAsync(gath + (size_t)me * C, packed + (size_t)me * C, sizeof(uint16_t) * C,
+                        cudaMemcpyDeviceToDevice, s));
+  CU(h, k_mean_gathered_half(gath, G, C, C, packed + (size_t)me * C, s));
+  CM(h, c->allgather(packed + (size_t)me * C, packed, sizeof(uint16_t) * C, s));
+  CU(h, k_unpack_half(packed, h->d_Q, nk, s));
   return HCCMF_OK;
 }
 
@@ -532,15 +579,41 @@ hccmf_status hccmf_create_dist(int64_t m, int64_t n, int32_t k, float gamma, flo
   hccmf_t h = *out;
   h->rank = rank;
   h->world = world;
-  ncclUniqueId id;
-  memcpy(&id, nccl_unique_id, sizeof(id));
-  ncclResult_t r = ncclCommInitRank(&h->comm, world, id, rank);
-  if (r != ncclSuccess) {
-    st = fail(nullptr, HCCMF_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+  std::string why;
+  h->comm = make_nccl_comm(nccl_unique_id, rank, world, device, &why);
+  if (!h->comm) {
+    st = fail(nullptr, HCCMF_ENCCL, "%s", why.c_str());
     hccmf_destroy(h);
     *out = nullptr;
     return st;
   }
+  return HCCMF_OK;
+}
+
+hccmf_status hccmf_create_loopback(int64_t m, int64_t n, int32_t k, float gamma, float lambda, hccmf_hub_t hub,
+                                   int32_t rank, int32_t device, hccmf_t* out) {
+  if (!out || !hub) return fail(nullptr, HCCMF_EINVAL, "NULL argument");
+  *out = nullptr;
+  hccmf_status st = check_problem(m, n, k, gamma, lambda);
+  if (st != HCCMF_OK) return st;
+  std::string why;
+  Comm* c = make_loopback_comm(hub, rank, device, &why);
+  if (!c) return fail(nullptr, HCCMF_EINVAL, "loopback: %s", why.c_str());
+  st = make_ctx(m, n, k, gamma, lambda, device, out);
+  if (st != HCCMF_OK) {
+    delete c;
+    return st;
+  }
+  (*out)->rank = rank;
+  (*out)->world = c->world;
+  (*out)->comm = c;
+  return HCCMF_OK;
+}
+
+hccmf_status hccmf_comm_counts(hccmf_t h, int64_t* counts, int32_t n, int32_t* n_sites) {
+  if (!h) return fail(nullptr, HCCMF_EINVAL, "NULL handle");
+  if (n_sites) *n_sites = N_COMM_SITES;
+  for (int i = 0; i < n && i < N_COMM_SITES; ++i) counts[i] = h->comm_counts[i];
   return HCCMF_OK;
 }
 
@@ -568,8 +641,6 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
       return HCCMF_OK;
     case HCCMF_OPT_SYNC_STREAM:
       h->sync_stream = value != 0;
-      return HCCMF_OK;
-    case HCCMF_OPT_RING_SUBBLOCKS:
       return HCCMF_OK;
     case HCCMF_OPT_HOGWILD_ATOMIC:
       h->opt_atomic = value != 0;
@@ -617,9 +688,9 @@ void hccmf_destroy(hccmf_t h) {
   cudaSetDevice(h->device);
   if (h->stream) cudaStreamSynchronize(h->stream);
   free_partition(h);
-  dfree(h, h->d_in_u, h->nnz);
-  dfree(h, h->d_in_v, h->nnz);
-  dfree(h, h->d_in_r, h->nnz);
+  dfree(h, h->d_in_u, h->nnz_in);
+  dfree(h, h->d_in_v, h->nnz_in);
+  dfree(h, h->d_in_r, h->nnz_in);
   dfree(h, h->d_partials, 2 * RMSE_BLOCKS);
   dfree(h, h->d_scalar, 2);
   if (h->d_wire) cudaFreeAsync(h->d_wire, h->stream);
@@ -629,27 +700,29 @@ void hccmf_destroy(hccmf_t h) {
     cudaStreamSynchronize(h->comm_stream);
     cudaStreamDestroy(h->comm_stream);
   }
-  if (h->comm) ncclCommDestroy(h->comm);
+  delete h->comm;
   if (getenv("HCCMF_TRIM")) trim_pool(h);
   if (h->stream) cudaStreamSynchronize(h->stream);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   delete h;
 }
 
-hccmf_status hccmf_load_ratings(hccmf_t h, const int32_t* u, const int32_t* v, const float* r, int64_t nnz) {
-  ENTER(h);
+namespace {
+hccmf_status load_impl(hccmf_t h, const int32_t* u, const int32_t* v, const float* r, int64_t nnz, bool sliced) {
   if (nnz < 0) return fail(h, HCCMF_EINVAL, "nnz must be >= 0");
   if (nnz > 0 && (!u || !v || !r)) return fail(h, HCCMF_EINVAL, "NULL rating array");
   free_partition(h);
-  dfree(h, h->d_in_u, h->nnz);
-  dfree(h, h->d_in_v, h->nnz);
-  dfree(h, h->d_in_r, h->nnz);
+  dfree(h, h->d_in_u, h->nnz_in);
+  dfree(h, h->d_in_v, h->nnz_in);
+  dfree(h, h->d_in_r, h->nnz_in);
   if (h->transposed) {  // back to the caller's orientation
     std::swap(h->m, h->n);
     h->transposed = false;
   }
   h->state = 0;
   h->nnz = nnz;
+  h->nnz_in = nnz;
+  h->sliced = sliced && h->world > 1;
   CU(h, dmalloc(h, &h->d_in_u, nnz));
   CU(h, dmalloc(h, &h->d_in_v, nnz));
   CU(h, dmalloc(h, &h->d_in_r, nnz));
@@ -666,12 +739,25 @@ hccmf_status hccmf_load_ratings(hccmf_t h, const int32_t* u, const int32_t* v, c
     CU(h, cudaStreamSynchronize(h->stream));
     if (bad) {
       h->nnz = 0;
+      h->nnz_in = 0;
       return fail(h, HCCMF_ERANGE, "invalid ratings:%s%s%s", (bad & 1) ? " u out of [0,m)" : "",
                   (bad & 2) ? " v out of [0,n)" : "", (bad & 4) ? " non-finite r" : "");
     }
   }
   h->state = 1;
   return finish(h);
+}
+}  // namespace
+
+hccmf_status hccmf_load_ratings(hccmf_t h, const int32_t* u, const int32_t* v, const float* r, int64_t nnz) {
+  ENTER(h);
+  return load_impl(h, u, v, r, nnz, false);
+}
+
+hccmf_status hccmf_load_ratings_slice(hccmf_t h, const int32_t* u, const int32_t* v, const float* r,
+                                      int64_t nnz_local) {
+  ENTER(h);
+  return load_impl(h, u, v, r, nnz_local, true);
 }
 
 hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
@@ -715,7 +801,8 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   h->Bc = o->grid_cols;
   h->seed = o->seed;
   h->storage = o->storage;
-  const int64_t m = h->m, n = h->n, nnz = h->nnz;
+  const int64_t m = h->m, n = h->n;
+  int64_t nnz = h->nnz_in;  // ratings held now (the global COO, or this rank's slice)
   cudaStream_t st = h->stream;
 
   PhaseTimer timer(h->stream);
@@ -730,11 +817,20 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   unsigned long long* dS = nullptr;
   CU(h, cudaMallocAsync((void**)&dS, sizeof(unsigned long long) * (m + 1), st));
   CU(h, k_row_prefix(h->d_in_u, nnz, h->d_perm_row, m, dS, st));
+  if (h->sliced) {  // the global prefix is the sum of the ranks' prefixes
+    h->comm_counts[SITE_INGEST_HIST] += 1;
+    CM(h, h->comm->allreduce(dS, dS, (size_t)m + 1, DType::u64, ROp::sum, st));
+    unsigned long long tot = 0;
+    CU(h, cudaMemcpyAsync(&tot, dS + m, sizeof(tot), cudaMemcpyDeviceToHost, st));
+    CU(h, cudaStreamSynchronize(st));
+    h->nnz = (int64_t)tot;
+  }
+  const int64_t nnz_glob = h->sliced ? h->nnz : nnz;
   std::vector<int64_t> targets(G > 1 ? G - 1 : 1, 0), rstar(G > 1 ? G - 1 : 1, 0);
   double cum = 0.0;
   for (int s = 1; s < G; ++s) {
     cum += x[s - 1];
-    targets[s - 1] = llround((double)nnz * cum);
+    targets[s - 1] = llround((double)nnz_glob * cum);
   }
   h->bounds.assign(G + 1, 0);
   h->bounds[G] = (int32_t)m;
@@ -756,6 +852,67 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   CU(h, cudaMemcpyAsync(dB, h->bounds.data(), sizeof(int32_t) * (G + 1), cudaMemcpyHostToDevice, st));
 
   timer.mark("a3 histogram+bounds");
+  if (h->sliced) {
+    // ---- sliced ingest: every rating to the rank that owns its (permuted) row.  Each
+    // source's ratings stay in input order and arrive in rank order, so the received
+    // sequence is the global COO restricted to this shard, in global order.
+    h->comm_counts[SITE_INGEST_EXCHANGE] += 1;
+    const int me = h->rank;
+    int32_t *xu = nullptr, *xv = nullptr;
+    float* xr = nullptr;
+    CU(h, dmalloc(h, &xu, nnz));
+    CU(h, dmalloc(h, &xv, nnz));
+    CU(h, dmalloc(h, &xr, nnz));
+    std::vector<int64_t> mine(G), all((size_t)G * G);
+    CU(h, k_shard_split(h->d_in_u, h->d_in_v, h->d_in_r, nnz, h->d_perm_row, dB, G, xu, xv, xr, mine.data(), st));
+    dfree(h, h->d_in_u, nnz);
+    dfree(h, h->d_in_v, nnz);
+    dfree(h, h->d_in_r, nnz);
+    int64_t* dcnt = nullptr;
+    CU(h, cudaMallocAsync((void**)&dcnt, sizeof(int64_t) * G * G, st));
+    CU(h, cudaMemcpyAsync(dcnt + (size_t)me * G, mine.data(), sizeof(int64_t) * G, cudaMemcpyHostToDevice, st));
+    CM(h, h->comm->allgather(dcnt + (size_t)me * G, dcnt, sizeof(int64_t) * G, st));
+    CU(h, cudaMemcpyAsync(all.data(), dcnt, sizeof(int64_t) * G * G, cudaMemcpyDeviceToHost, st));
+    CU(h, cudaStreamSynchronize(st));
+    cudaFreeAsync(dcnt, st);
+    std::vector<int64_t> soff(G + 1, 0), roff(G + 1, 0);  // send offsets (by dest), recv offsets (by source)
+    for (int p = 0; p < G; ++p) {
+      soff[p + 1] = soff[p] + all[(size_t)me * G + p];
+      roff[p + 1] = roff[p] + all[(size_t)p * G + me];
+    }
+    const int64_t got = roff[G];
+    CU(h, dmalloc(h, &h->d_in_u, got));
+    CU(h, dmalloc(h, &h->d_in_v, got));
+    CU(h, dmalloc(h, &h->d_in_r, got));
+    Comm* c = h->comm;
+    CM(h, c->group_start());
+    for (int p = 0; p < G; ++p) {
+      if (p == me) continue;
+      const int64_t ns = soff[p + 1] - soff[p], nr = roff[p + 1] - roff[p];
+      if (ns) {
+        CM(h, c->send(xu + soff[p], 4 * ns, p, st));
+        CM(h, c->send(xv + soff[p], 4 * ns, p, st));
+        CM(h, c->send(xr + soff[p], 4 * ns, p, st));
+      }
+      if (nr) {
+        CM(h, c->recv(h->d_in_u + roff[p], 4 * nr, p, st));
+        CM(h, c->recv(h->d_in_v + roff[p], 4 * nr, p, st));
+        CM(h, c->recv(h->d_in_r + roff[p], 4 * nr, p, st));
+      }
+    }
+    CM(h, c->group_end());
+    if (const int64_t nm = soff[me + 1] - soff[me]) {
+      CU(h, cudaMemcpyAsync(h->d_in_u + roff[me], xu + soff[me], 4 * nm, cudaMemcpyDeviceToDevice, st));
+      CU(h, cudaMemcpyAsync(h->d_in_v + roff[me], xv + soff[me], 4 * nm, cudaMemcpyDeviceToDevice, st));
+      CU(h, cudaMemcpyAsync(h->d_in_r + roff[me], xr + soff[me], 4 * nm, cudaMemcpyDeviceToDevice, st));
+    }
+    dfree(h, xu, nnz);
+    dfree(h, xv, nnz);
+    dfree(h, xr, nnz);
+    nnz = got;
+    h->nnz_in = got;
+    timer.mark("sliced ingest exchange");
+  }
   // ---- a4 geometry + stable sort
   BlockGeom g{};
   g.G = G;
@@ -782,6 +939,10 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   timer.mark("a4 alloc records");
   CU(h, k_block_sort(g, dB, h->d_perm_row, h->d_perm_col, h->d_in_u, h->d_in_v, h->d_in_r, nnz, su, sv, sr, dOff, st));
   timer.mark("a4 key+sort+decode");
+  if (h->sliced) {  // global block offsets = the sum of the ranks' (local) offsets
+    h->comm_counts[SITE_INGEST_BLOCKS] += 1;
+    CM(h, h->comm->allreduce(dOff, dOff, (size_t)nblk + 1, DType::i64, ROp::sum, st));
+  }
   h->block_off.assign(nblk + 1, 0);
   CU(h, cudaMemcpyAsync(h->block_off.data(), dOff, sizeof(int64_t) * (nblk + 1), cudaMemcpyDeviceToHost, st));
   CU(h, cudaStreamSynchronize(st));
@@ -804,7 +965,14 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   h->nblk_local = (h->shard_hi - h->shard_lo) * bps;
   h->rec0 = h->block_off[h->blk0];
   h->local_nnz = h->block_off[h->blk0 + h->nblk_local] - h->rec0;
-  if (h->world > 1) {
+  if (h->sliced) {  // the sorted records are exactly this shard's
+    if (h->local_nnz != nnz)
+      return fail(h, HCCMF_ESTATE, "sliced ingest: %lld records received, %lld in the shard's blocks",
+                  (long long)nnz, (long long)h->local_nnz);
+    h->d_u = su;
+    h->d_v = sv;
+    h->d_r = sr;
+  } else if (h->world > 1) {
     CU(h, dmalloc(h, &h->d_u, h->local_nnz));
     CU(h, dmalloc(h, &h->d_v, h->local_nnz));
     CU(h, dmalloc(h, &h->d_r, h->local_nnz));
@@ -928,12 +1096,16 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     a.lambda = h->lambda;
     a.vec_pref = (int32_t)h->opt_vec;
     a.prefetch = 1;
-    if (wave_slab)
-      CU(h, launch_wave_slab(a, h->d_blk_off, h->Br, h->d_progress, h->n, h->stream));
-    else
-      CU(h, launch_wave(a, h->d_blk_off, h->Br, h->d_progress, h->stream));
-    ++h->epoch;
-    return finish(h);
+    cudaError_t e = wave_slab ? launch_wave_slab(a, h->d_blk_off, h->Br, h->d_progress, h->n, h->stream)
+                              : launch_wave(a, h->d_blk_off, h->Br, h->d_progress, h->stream);
+    if (e == cudaSuccess) {
+      ++h->epoch;
+      return finish(h);
+    }
+    // the cooperative launch could not make every CTA co-resident (another workload holds
+    // SMs): nothing ran; the per-stratum launches below compute the same epoch
+    if (e != cudaErrorCooperativeLaunchTooLarge) CU(h, e);
+    cudaGetLastError();
   }
   Plan* pl = nullptr;
   hccmf_status st = build_plan(h, sched, sync, &pl);
@@ -955,13 +1127,11 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   };
   auto average = [&]() -> hccmf_status {  // the server's sync (L549-L557): Q = mean of the shards' Q
     if (dist && h->opt_wire16) {  // Strategy 2: the copies travel and come back as binary16
-      hccmf_status w = wire_reserve(h, (size_t)nk);
+      hccmf_status w = allreduce_q16(h, s);
       if (w != HCCMF_OK) return w;
-      CU(h, k_pack_half(h->d_Q, h->d_wire, nk, s));
-      NC(h, ncclAllReduce(h->d_wire, h->d_wire, (size_t)nk, ncclHalf, ncclAvg, h->comm, s));
-      CU(h, k_unpack_half(h->d_wire, h->d_Q, nk, s));
     } else if (dist) {
-      NC(h, ncclAllReduce(h->d_Q, h->d_Q, (size_t)nk, ncclFloat, ncclAvg, h->comm, s));
+      h->comm_counts[SITE_ALLREDUCE_Q] += 1;
+      CM(h, h->comm->allreduce(h->d_Q, h->d_Q, (size_t)nk, DType::f32, ROp::avg, s));
     } else if (h->opt_wire16) {
       CU(h, k_average_half(h->d_Qrep, nrep, nk, h->d_Q, s));
     } else {
@@ -1018,8 +1188,6 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   a.rec0 = h->rec0;
   a.epoch = h->epoch;
   const int L = sgd_lanes(h->k, (int)h->opt_vec);
-  // a ring stage races only on its column group's items
-  const int64_t hog_warps = auto_warps(h, eff_sync == HCCMF_SYNC_RING ? h->n / G : h->n);
   if (dist && eff_sync == HCCMF_SYNC_RING && sched == HCCMF_SCHED_HOGWILD) {
     const size_t ne = (size_t)G * (h->Bc / G);
     if (pl->launches.size() != ne) return fail(h, HCCMF_EINVAL, "ring plan: one launch per column block expected");
@@ -1111,7 +1279,8 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     a.n_tasks = ln.nt;
     a.counter = h->d_counters + li;
     // DET: one rating group per block of the stratum; HOGWILD: persistent grid
-    const int64_t warps = (sched == HCCMF_SCHED_DET) ? (ln.nt * L + 31) / 32 : hog_warps;
+    // Hogwild races only on the Q rows of the launch's column blocks (R14, R28)
+    const int64_t warps = (sched == HCCMF_SCHED_DET) ? (ln.nt * L + 31) / 32 : auto_warps(h, ln.items);
     CU(h, launch_sgd(a, warps, s));
     if (pipelined) {
       st = qh_flush();  // the block travels as fp32 (or binary16 wire) right after its launch
@@ -1187,7 +1356,10 @@ hccmf_status hccmf_rmse(hccmf_t h, const int32_t* u, const int32_t* v, const flo
   }
   CU(h, k_rmse(du, dv, dr, nt, h->d_perm_row, h->d_perm_col, h->d_P, h->row0, h->rows, h->d_Q, h->k, h->d_partials,
                h->d_scalar, s));
-  if (h->world > 1) NC(h, ncclAllReduce(h->d_scalar, h->d_scalar, 2, ncclDouble, ncclSum, h->comm, s));
+  if (h->world > 1) {
+    h->comm_counts[SITE_RMSE] += 1;
+    CM(h, h->comm->allreduce(h->d_scalar, h->d_scalar, 2, DType::f64, ROp::sum, s));
+  }
   double sc[2] = {0.0, 0.0};
   CU(h, cudaMemcpyAsync(sc, h->d_scalar, sizeof(sc), cudaMemcpyDeviceToHost, s));
   CU(h, cudaStreamSynchronize(s));
@@ -1209,15 +1381,16 @@ hccmf_status hccmf_get_factors(hccmf_t h, float* P, float* Q) {
     float* tmp = nullptr;
     if (h->world > 1) {  // final push of P (L1205-L1206): every shard's rows to every rank
       CU(h, cudaMallocAsync((void**)&full, sizeof(float) * mk, s));
-      NC(h, ncclGroupStart());
+      h->comm_counts[SITE_EXPORT_P] += 1;
+      CM(h, h->comm->group_start());
       for (int g = 0; g < h->G; ++g) {
         const int64_t a = h->bounds[g], b = h->bounds[g + 1];
         if (b > a) {
           const float* src = (g == h->rank) ? h->d_P : full + a * h->k;
-          NC(h, ncclBroadcast(src, full + a * h->k, (size_t)(b - a) * h->k, ncclFloat, g, h->comm, s));
+          CM(h, h->comm->broadcast(src, full + a * h->k, sizeof(float) * (size_t)(b - a) * h->k, g, s));
         }
       }
-      NC(h, ncclGroupEnd());
+      CM(h, h->comm->group_end());
     }
     CU(h, cudaMallocAsync((void**)&tmp, sizeof(float) * mk, s));
     CU(h, k_gather_rows(full, h->m, h->k, h->d_perm_row, 0, tmp, s));
@@ -1334,6 +1507,18 @@ hccmf_status hccmf_cost_model(int32_t p, int64_t m, int64_t n, int64_t nnz, int3
     *strategy = HCCMF_DP2;
   }
   return HCCMF_OK;
+}
+
+hccmf_status hccmf_probe_roundtrip(hccmf_t h, int32_t mode, int64_t warps, int32_t reps, double* ms) {
+  ENTER(h);
+  if (!ms || mode < 0 || mode > 2 || warps < 0 || reps < 1) return fail(h, HCCMF_EINVAL, "bad probe arguments");
+  if (h->state < 2) return fail(h, HCCMF_ESTATE, "probe needs partition");
+  if (h->k % 128 != 0) return fail(h, HCCMF_EINVAL, "probe needs k a multiple of 128");
+  const int64_t w = warps ? warps : auto_warps(h, h->n);
+  float t = 0.f;
+  CU(h, k_probe_roundtrip(mode, h->d_v, h->d_r, h->local_nnz, h->k, h->n, w, reps, &t, h->stream));
+  *ms = t;
+  return finish(h);
 }
 
 hccmf_status hccmf_get_info(hccmf_t h, hccmf_info* o) {

@@ -8,6 +8,7 @@
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
+#include <vector>
 
 #include <cub/cub.cuh>
 #include <thrust/iterator/counting_iterator.h>
@@ -251,6 +252,29 @@ __global__ void permute_tasks_kernel(const int64_t* idx, int64_t nt, const int64
   }
 }
 
+// sliced ingest: destination shard of every rating (key) and its input index (value)
+__global__ void shard_key_kernel(const int32_t* __restrict__ u, int64_t nnz, const int32_t* __restrict__ perm_row,
+                                 const int32_t* __restrict__ bounds, int32_t G, uint32_t* key, int64_t* idx,
+                                 unsigned long long* cnt) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t s = shard_of(bounds, G, perm_row[u[i]]);
+    key[i] = (uint32_t)s;
+    idx[i] = i;
+    atomicAdd(cnt + s, 1ull);
+  }
+}
+
+__global__ void gather_ratings_kernel(const int64_t* __restrict__ idx, int64_t nnz, const int32_t* __restrict__ u,
+                                      const int32_t* __restrict__ v, const float* __restrict__ r, int32_t* ou,
+                                      int32_t* ov, float* orr) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t j = idx[i];
+    ou[i] = u[j];
+    ov[i] = v[j];
+    orr[i] = r[j];
+  }
+}
+
 template <typename T>
 cudaError_t dalloc(T** p, size_t count, cudaStream_t st) {
   return cudaMallocAsync((void**)p, sizeof(T) * (count ? count : 1), st);
@@ -374,6 +398,44 @@ cudaError_t k_block_sort(const BlockGeom& g, const int32_t* bounds, const int32_
   CKR(cudaGetLastError());
   cudaFreeAsync(k0, st);
   cudaFreeAsync(k1, st);
+  return cudaGetLastError();
+}
+
+cudaError_t k_shard_split(const int32_t* u, const int32_t* v, const float* r, int64_t nnz, const int32_t* perm_row,
+                          const int32_t* bounds, int32_t G, int32_t* ou, int32_t* ov, float* orr, int64_t* counts,
+                          cudaStream_t st) {
+  for (int s = 0; s < G; ++s) counts[s] = 0;
+  if (nnz == 0) return cudaSuccess;
+  uint32_t *k0 = nullptr, *k1 = nullptr;
+  int64_t *i0 = nullptr, *i1 = nullptr;
+  unsigned long long* cnt = nullptr;
+  CKR(dalloc(&k0, nnz, st));
+  CKR(dalloc(&k1, nnz, st));
+  CKR(dalloc(&i0, nnz, st));
+  CKR(dalloc(&i1, nnz, st));
+  CKR(dalloc(&cnt, G, st));
+  CKR(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long) * G, st));
+  (note_launch(), shard_key_kernel<<<grid_for(nnz), kT, 0, st>>>(u, nnz, perm_row, bounds, G, k0, i0, cnt));
+  CKR(cudaGetLastError());
+  int bits = 0;
+  while ((1 << bits) < G) ++bits;
+  const int64_t* idx = i0;
+  if (bits > 0) {  // LSD radix sort: stable, so each shard keeps the input order
+    size_t tb = 0;
+    void* tmp = nullptr;
+    CKR(cub::DeviceRadixSort::SortPairs(nullptr, tb, k0, k1, i0, i1, nnz, 0, bits, st));
+    CKR(cudaMallocAsync(&tmp, tb, st));
+    CKR(cub::DeviceRadixSort::SortPairs(tmp, tb, k0, k1, i0, i1, nnz, 0, bits, st));
+    cudaFreeAsync(tmp, st);
+    idx = i1;
+  }
+  (note_launch(), gather_ratings_kernel<<<grid_for(nnz), kT, 0, st>>>(idx, nnz, u, v, r, ou, ov, orr));
+  CKR(cudaGetLastError());
+  std::vector<unsigned long long> h(G);
+  CKR(cudaMemcpyAsync(h.data(), cnt, sizeof(unsigned long long) * G, cudaMemcpyDeviceToHost, st));
+  CKR(cudaStreamSynchronize(st));
+  for (int s = 0; s < G; ++s) counts[s] = (int64_t)h[s];
+  for (void* p : {(void*)k0, (void*)k1, (void*)i0, (void*)i1, (void*)cnt}) cudaFreeAsync(p, st);
   return cudaGetLastError();
 }
 

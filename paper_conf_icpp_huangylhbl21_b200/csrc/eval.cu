@@ -198,6 +198,17 @@ __global__ void average_half_kernel(const float* reps, int32_t G, int64_t count,
   }
 }
 
+// Strategy 2 all-reduce on the wire (R25): W binary16 copies of one chunk, `stride`
+// halves apart, summed in fp64 in rank order; the mean is rounded once to binary16 --
+// the same function as average_half_kernel on the logical backend
+__global__ void mean_gathered_half_kernel(const __half* g, int32_t W, int64_t stride, int64_t count, __half* out) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < count; e += (int64_t)gridDim.x * blockDim.x) {
+    double s = 0.0;
+    for (int r = 0; r < W; ++r) s += (double)__half2float(g[(int64_t)r * stride + e]);
+    out[e] = __double2half(s / (double)W);
+  }
+}
+
 }  // namespace
 
 cudaError_t k_round_half(float* x, int64_t count, cudaStream_t st) {
@@ -217,6 +228,13 @@ cudaError_t k_unpack_half(const void* y, float* x, int64_t count, cudaStream_t s
 }
 cudaError_t k_average_half(const float* reps, int32_t G, int64_t count, float* out, cudaStream_t st) {
   (note_launch(), average_half_kernel<<<grid_for(count), kT, 0, st>>>(reps, G, count, out));
+  return cudaGetLastError();
+}
+
+cudaError_t k_mean_gathered_half(const void* g, int32_t W, int64_t stride, int64_t count, void* out, cudaStream_t st) {
+  if (count <= 0) return cudaSuccess;
+  (note_launch(), mean_gathered_half_kernel<<<grid_for(count), kT, 0, st>>>(reinterpret_cast<const __half*>(g), W, stride,
+                                                                            count, reinterpret_cast<__half*>(out)));
   return cudaGetLastError();
 }
 

@@ -2,13 +2,13 @@
 #pragma once
 
 #include <cuda_runtime.h>
-#include <nccl.h>
 #include <stdint.h>
 
 #include <atomic>
 #include <string>
 #include <vector>
 
+#include "comm.cuh"
 #include "hccmf.h"
 
 namespace hccmf {
@@ -43,6 +43,8 @@ struct Launch {
   int32_t qrep;
   int32_t stage;
   int32_t phase;  // all-reduce sub-epoch round (R22)
+  int64_t items;  // Q rows this launch's blocks may touch (distinct column blocks): the
+                  // Hogwild concurrency cap of DESIGN.md R14 is taken from it
 };
 
 struct Plan {
@@ -114,6 +116,11 @@ cudaError_t k_block_sort(const BlockGeom& g, const int32_t* bounds, const int32_
                          const int32_t* perm_col, const int32_t* u, const int32_t* v, const float* r,
                          int64_t nnz, int32_t* ou, int32_t* ov, float* orr, int64_t* block_off,
                          cudaStream_t st);
+// sliced ingest: stable split of n ratings by the shard owning perm_row[u] (bounds on the
+// device, G + 1); out_* receive them grouped by shard in input order, counts[G] (host)
+cudaError_t k_shard_split(const int32_t* u, const int32_t* v, const float* r, int64_t nnz, const int32_t* perm_row,
+                          const int32_t* bounds, int32_t G, int32_t* ou, int32_t* ov, float* orr, int64_t* counts,
+                          cudaStream_t st);
 cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* blk_off_local /*nb+1, local idx*/,
                           int64_t nb, int64_t target, int64_t heavy, int64_t** task_lo, int64_t** task_hi, int64_t* n_tasks,
                           cudaStream_t st);
@@ -133,7 +140,12 @@ cudaError_t k_round_half(float* x, int64_t count, cudaStream_t st);
 cudaError_t k_pack_half(const float* x, void* y /* __half */, int64_t count, cudaStream_t st);
 cudaError_t k_unpack_half(const void* y /* __half */, float* x, int64_t count, cudaStream_t st);
 cudaError_t k_average_half(const float* reps, int32_t G, int64_t count, float* out, cudaStream_t st);
+// W gathered binary16 copies (stride halves apart) -> fp64 mean rounded once to binary16
+cudaError_t k_mean_gathered_half(const void* g, int32_t W, int64_t stride, int64_t count, void* out, cudaStream_t st);
 constexpr int RMSE_BLOCKS = 592;
+// q_v round-trip ceiling probe (probe.cu): mean ms of one pass over the records
+cudaError_t k_probe_roundtrip(int mode, const int32_t* rv, const float* rr, int64_t nrec, int32_t k, int64_t n,
+                              int64_t warps, int reps, float* ms, cudaStream_t st);
 
 }  // namespace hccmf
 
@@ -146,7 +158,8 @@ struct hccmf_ctx {
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   int32_t rank = 0, world = 1;
-  ncclComm_t comm = nullptr;
+  hccmf::Comm* comm = nullptr;                  // NCCL or loopback (world > 1 / distributed handles)
+  int64_t comm_counts[hccmf::N_COMM_SITES] = {};// per-call-site executions (hccmf_comm_counts)
   cudaStream_t comm_stream = nullptr;           // ring transfers overlapped with compute
   std::vector<cudaEvent_t> ev_done, ev_recv;    // per (stage, column block)
   void* d_wire = nullptr;                       // binary16 staging (send | recv) for Strategy 2
@@ -158,8 +171,10 @@ struct hccmf_ctx {
   bool sync_stream = true;
   size_t device_bytes = 0;
 
-  // a1 input (global COO, device)
-  int64_t nnz = 0;
+  // a1 input (global COO, or this rank's slice of it: sliced ingest), device
+  int64_t nnz = 0;     // global ratings (after partition; = nnz_in until then unless sliced)
+  int64_t nnz_in = 0;  // ratings in d_in_*
+  bool sliced = false; // d_in_* is this rank's slice of the global COO (hccmf_load_ratings_slice)
   int32_t* d_in_u = nullptr;
   int32_t* d_in_v = nullptr;
   float* d_in_r = nullptr;

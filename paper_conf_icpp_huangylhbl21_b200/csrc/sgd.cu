@@ -1346,19 +1346,39 @@ bool wave_supported(int k, int vec_pref, int B) {
   return (int64_t)B * 2 <= (int64_t)sms * per_sm * (kThreads / 32);
 }
 
+// The wavefront kernels spin on progress counters of warps in other CTAs, so every CTA
+// must be resident at once: they are launched cooperatively, and the driver either
+// guarantees co-residency (whatever else the device runs) or fails the launch with
+// cudaErrorCooperativeLaunchTooLarge, on which the caller runs the per-stratum launches.
+template <typename... KArgs, typename... Args>
+cudaError_t launch_cooperative(void (*kernel)(KArgs...), unsigned blocks, unsigned threads, size_t smem,
+                               cudaStream_t st, Args... args) {
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(blocks);
+  cfg.blockDim = dim3(threads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  note_launch();
+  return cudaLaunchKernelEx(&cfg, kernel, args...);
+}
+
 cudaError_t launch_wave(const SgdArgs& a, const int64_t* off, int B, int* progress, cudaStream_t st) {
   int L, VEC;
   sgd_geometry(a.k, a.vec_pref, &L, &VEC);
   cudaError_t e = cudaMemsetAsync(progress, 0, sizeof(int) * B, st);
   if (e != cudaSuccess) return e;
-  const int64_t blocks = ((int64_t)B * 32 + kThreads - 1) / kThreads;
+  const unsigned blocks = (unsigned)(((int64_t)B * 32 + kThreads - 1) / kThreads);
   switch (VEC) {
-    case 1: (note_launch(), sgd_wave_kernel<1><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress)); break;
-    case 2: (note_launch(), sgd_wave_kernel<2><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress)); break;
-    case 4: (note_launch(), sgd_wave_kernel<4><<<(unsigned)blocks, kThreads, 0, st>>>(a, off, B, progress)); break;
+    case 1: return launch_cooperative(sgd_wave_kernel<1>, blocks, kThreads, 0, st, a, off, B, progress);
+    case 2: return launch_cooperative(sgd_wave_kernel<2>, blocks, kThreads, 0, st, a, off, B, progress);
+    case 4: return launch_cooperative(sgd_wave_kernel<4>, blocks, kThreads, 0, st, a, off, B, progress);
     default: return cudaErrorInvalidValue;
   }
-  return cudaGetLastError();
 }
 
 namespace {
@@ -1417,7 +1437,9 @@ cudaError_t launch_wave_slab(const SgdArgs& a, const int64_t* off, int B, int* p
 #define SLAB_CASE(V)                                                                                        \
   case V:                                                                                                   \
     if (!slab_geometry_t<V>(a.k, B, n, &wpc, &smem)) return cudaErrorInvalidConfiguration;                 \
-    (note_launch(), sgd_wave_slab_kernel<V><<<(unsigned)((B + wpc - 1) / wpc), wpc * 32, smem, st>>>(a, off, B, progress, n, wmax)); \
+    e = launch_cooperative(sgd_wave_slab_kernel<V>, (unsigned)((B + wpc - 1) / wpc), (unsigned)(wpc * 32), smem, st, \
+                           a, off, B, progress, n, wmax);                                                  \
+    if (e != cudaSuccess) return e;                                                                       \
     break;
   switch (VEC) {
     SLAB_CASE(1)

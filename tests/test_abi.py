@@ -59,3 +59,20 @@ def test_no_cpu_fallback_without_device():
     with pytest.raises(pkg.HccmfError) as ei:
         pkg.Model(10, 10, 8)
     assert ei.value.code == pkg.ECUDA
+
+
+def test_loopback_hub_lifecycle_without_device():
+    # the hub is host-only; a loopback handle needs a device and fails loudly without one
+    import paper_conf_icpp_huangylhbl21_b200 as pkg
+    L = pkg.lib()
+    hub = ctypes.c_void_p()
+    assert L.hccmf_hub_create(0, ctypes.byref(hub)) == pkg.EINVAL
+    assert L.hccmf_hub_create(3, ctypes.byref(hub)) == pkg.OK and hub.value
+    h = ctypes.c_void_p()
+    assert L.hccmf_create_loopback(10, 10, 8, 0.005, 0.01, hub, 3, 0, ctypes.byref(h)) == pkg.EINVAL  # rank >= world
+    assert L.hccmf_create_loopback(10, 10, 6, 0.005, 0.01, hub, 0, 0, ctypes.byref(h)) == pkg.EINVAL  # k % 4 != 0
+    if not os.path.exists("/dev/nvidia0"):
+        assert L.hccmf_create_loopback(10, 10, 8, 0.005, 0.01, hub, 1, 0, ctypes.byref(h)) == pkg.ECUDA
+    assert L.hccmf_comm_counts(None, None, 0, None) == pkg.EINVAL
+    L.hccmf_hub_destroy(hub)
+    L.hccmf_hub_destroy(None)

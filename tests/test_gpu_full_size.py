@@ -15,6 +15,7 @@ import os
 import numpy as np
 import pytest
 
+import bands
 import synth
 
 pytestmark = pytest.mark.gpu
@@ -85,7 +86,7 @@ def test_hogwild_band_full_size(pkg, c3, name, data, storage):
             curve.append(mdl.rmse(tu, tv, tr))
         if storage == "fp32":
             assert curve[0] == pytest.approx(ref["test_rmse"][0], rel=1e-6)  # same init, same data
-        assert abs(curve[E] - ref["test_rmse"][E]) <= 0.005, (curve, ref["test_rmse"])
+        bands.check(curve, ref["test_rmse"], f"{name} full size {storage} G=1")
 
 
 def test_c5_full_size_properties(pkg):

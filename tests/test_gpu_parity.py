@@ -8,6 +8,7 @@ Hogwild and multi-shard modes.
 import numpy as np
 import pytest
 
+import bands
 import golden_io
 import synth
 
@@ -268,6 +269,8 @@ def test_hogwild_single_group_is_the_serial_oracle(pkg, orc, atomic, k, task, de
 
 
 def _band(pkg, orc, cfg_name, frac, k, epochs, sync="none", G=1, Br=1, Bc=1, repeats=2, gamma=None):
+    """GPU and oracle test-RMSE curves (same data, same schedule, init seed 1), checked with the
+    shared bar of tests/bands.py (R15, R29) for every repeat."""
     cfg = synth.CONFIGS[cfg_name]
     if frac != 1.0:
         cfg = synth.scaled(cfg, frac)
@@ -275,37 +278,35 @@ def _band(pkg, orc, cfg_name, frac, k, epochs, sync="none", G=1, Br=1, Bc=1, rep
     (u, v, r), (tu, tv, tr) = synth.make(cfg)
     prob = orc.Problem(cfg.m, cfg.n, k, gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=Bc, seed=cfg.seed)
     prob.init(1)
+    want = [prob.rmse(tu, tv, tr)]
     for _ in range(epochs):
         prob.epoch("serial", sync)
-    want = prob.rmse(tu, tv, tr)
-    got = []
-    for _ in range(repeats):
+        want.append(prob.rmse(tu, tv, tr))
+    for rep in range(repeats):
         mdl = _gpu_problem(pkg, cfg.m, cfg.n, k, gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=Bc, seed=cfg.seed)
         mdl.init(1)
+        got = [mdl.rmse(tu, tv, tr)]
         for _ in range(epochs):
             mdl.train_epoch("hogwild", sync)
-        got.append(mdl.rmse(tu, tv, tr))
+            got.append(mdl.rmse(tu, tv, tr))
         mdl.close()
-    return want, got
+        bands.check(got, want, f"{cfg_name} frac={frac} k={k} sync={sync} G={G} grid={Br}x{Bc} rep={rep}")
 
 
 def test_hogwild_band_c1(pkg, orc):
     # BASELINE.json config 1: 5 epochs, 1 GPU vs the CPU oracle
-    want, got = _band(pkg, orc, "c1", 1.0, 16, 5, repeats=3)
-    assert all(abs(g - want) <= 0.005 for g in got), (want, got)
+    _band(pkg, orc, "c1", 1.0, 16, 5, repeats=3)
 
 
 def test_hogwild_band_c2_full(pkg, orc):
     # BASELINE.json config 2 at full size; band read at E = 20 epochs (R15)
-    want, got = _band(pkg, orc, "c2", 1.0, 32, 20, repeats=3)  # Hogwild bands run 3 times
-    assert all(abs(g - want) <= 0.005 for g in got), (want, got)
+    _band(pkg, orc, "c2", 1.0, 32, 20, repeats=3)  # Hogwild bands run 3 times
 
 
 @pytest.mark.parametrize("sync,G,Bc", [("ring", 4, 4), ("ring", 2, 8), ("allreduce", 2, 1)])
 def test_hogwild_logical_shards_band_c2(pkg, orc, sync, G, Bc):
     # multi-GPU schedules on G logical shards; the oracle runs the same schedule serially
-    want, got = _band(pkg, orc, "c2", 1.0, 32, 20, sync=sync, G=G, Br=1, Bc=Bc, repeats=1)
-    assert all(abs(g - want) <= 0.005 for g in got), (want, got)
+    _band(pkg, orc, "c2", 1.0, 32, 20, sync=sync, G=G, Br=1, Bc=Bc, repeats=1)
 
 
 @pytest.mark.parametrize("k,B,dup", [(128, 24, False), (256, 9, False), (128, 37, True), (512, 12, True),
@@ -388,17 +389,22 @@ def test_hogwild_allreduce_sub_epoch_sync_band_c2(pkg, orc, phases):
     mdl = _gpu_problem(pkg, cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=1, seed=cfg.seed)
     mdl.set_option("sync_phases", phases)
     mdl.init(1)
+    want, got = [prob.rmse(tu, tv, tr)], [mdl.rmse(tu, tv, tr)]
     for _ in range(20):
         prob.epoch_phased(phases)
         mdl.train_epoch("hogwild", "allreduce")
-    want, got = prob.rmse(tu, tv, tr), mdl.rmse(tu, tv, tr)
-    assert abs(got - want) <= 0.005, (want, got)
+        want.append(prob.rmse(tu, tv, tr))
+        got.append(mdl.rmse(tu, tv, tr))
+    bands.check(got, want, f"c2 allreduce phases={phases}")
 
 
 def test_distributed_handle_world1_matches_single(pkg, orc):
-    # the NCCL code paths (unique-id bootstrap through torch.distributed, ncclCommInitRank,
-    # ncclAllReduce(ncclAvg) for Q and {sum, count} of the RMSE, broadcasts in get_factors)
-    # on a one-rank communicator: results equal the single-process handle bit for bit
+    # the NCCL backend's bootstrap on one rank: the unique id travels through
+    # torch.distributed and ncclCommInitRank builds a one-rank communicator.  With world = 1
+    # and G = 1 no collective runs (every data-plane call site is guarded by world > 1 and
+    # the epochs degenerate to SYNC_NONE), so this pins the handle plumbing only: results
+    # equal the single-process handle bit for bit.  The multi-rank data plane itself runs in
+    # tests/test_gpu_loopback.py (every call site, G = 2..8 ranks on one GPU).
     import os
     import socket
     import torch.distributed as dist
@@ -466,11 +472,13 @@ def test_hogwild_ring_wire_fp16_band_c2(pkg, orc):
     mdl = _gpu_problem(pkg, cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=G, Br=1, Bc=Bc, seed=cfg.seed)
     mdl.set_option("wire_fp16", 1)
     mdl.init(1)
+    want, got = [prob.rmse(tu, tv, tr)], [mdl.rmse(tu, tv, tr)]
     for _ in range(20):
         prob.epoch_wire16("serial", "ring")
         mdl.train_epoch("hogwild", "ring")
-    want, got = prob.rmse(tu, tv, tr), mdl.rmse(tu, tv, tr)
-    assert abs(got - want) <= 0.005, (want, got)
+        want.append(prob.rmse(tu, tv, tr))
+        got.append(mdl.rmse(tu, tv, tr))
+    bands.check(got, want, "c2 ring G=4 Bc=8 wire16 (logical)")
 
 
 # ---------------------------------------- binary16 storage of Q (f1, R26)

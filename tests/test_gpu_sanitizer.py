@@ -1,0 +1,33 @@
+"""compute-sanitizer over the synchronisation-heavy kernels:
+memcheck (out-of-bounds / misaligned accesses, in the blocker and the SGD kernels), racecheck
+(shared-memory hazards: the slab wavefront's Q slabs and p_u ring, the record rings) and
+synccheck (barrier / warp-sync misuse) on tools/sanitize_workload.py.  Logs of the full runs
+are committed under profiles/r02_sanitizer_*.log."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+TOOL = shutil.which("compute-sanitizer") or "/usr/local/cuda/bin/compute-sanitizer"
+
+
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck"])
+def test_sanitizer_clean(tool):
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    if not os.path.exists(TOOL):
+        pytest.skip("compute-sanitizer not installed")
+    import __graft_entry__
+    __graft_entry__.build()
+    cmd = [TOOL, "--tool", tool, "--error-exitcode", "9", "--print-limit", "20", sys.executable,
+           os.path.join(ROOT, "tools", "sanitize_workload.py"), "--quick"]
+    p = subprocess.run(cmd, capture_output=True, text=True, timeout=1500, cwd=ROOT)
+    out = p.stdout + p.stderr
+    assert p.returncode == 0, out[-4000:]
+    assert "ERROR SUMMARY: 0 errors" in out, out[-4000:]
+    assert "jobs ok" in out

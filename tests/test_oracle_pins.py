@@ -275,6 +275,43 @@ def test_init_range_and_scale(orc):
     assert np.array_equal(P2[pr], P)
 
 
+def test_init_elements_hand_computed(orc):
+    # R5 element by element, from the published SplitMix64 (pinned above) written out here in
+    # pure Python: P[u][j] = U(H(seed, 3, u, j)) sqrt(1/k), Q[v][j] = U(H(seed, 4, v, j)) sqrt(1/k).
+    # Hand-computed words for seed 7 (u/v = 2, j = 5 and the swapped (5, 2)):
+    #   H(7,3,2,5) = 0x0cd83494f4c604e6 -> top 24 bits 841780    -> P[2][5] = 841780 2^-24 sqrt(1/8)
+    #   H(7,3,5,2) = 0x566fe5d8ffab1f03 -> 5664741               -> P[5][2]
+    #   H(7,4,2,5) = 0xd9d05e5045769262 -> 14274654              -> Q[2][5]
+    #   H(7,4,5,2) = 0x43141ffb2255f682 -> 4396063               -> Q[5][2]
+    # so swapped (row, column) arguments or swapped tags 3 / 4 change every one of them.
+    M, G = (1 << 64) - 1, 0x9E3779B97F4A7C15
+
+    def sm(x):
+        z = (x + G) & M
+        z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & M
+        z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & M
+        return z ^ (z >> 31)
+
+    assert [sm((i * G) & M) for i in range(1, 3)] == [0x6E789E6AA1B965F4, 0x06C45D188009454F]
+    H = lambda seed, tag, a, b: sm(sm(sm(seed ^ (tag << 56)) ^ a) ^ b)  # noqa: E731
+    assert H(7, 3, 2, 5) == 0x0CD83494F4C604E6 and H(7, 3, 5, 2) == 0x566FE5D8FFAB1F03
+    assert H(7, 4, 2, 5) == 0xD9D05E5045769262 and H(7, 4, 5, 2) == 0x43141FFB2255F682
+    k, sc = 8, math.sqrt(1.0 / 8)
+    m, n = 9, 7
+    pr, pc = orc.perm(11, 1, m), orc.perm(11, 2, n)  # stored permuted: row pr[u] holds user u
+    P, Q = orc.init(7, m, n, k, pr, pc)
+    assert P[pr[2], 5] == 841780 * 2.0 ** -24 * sc
+    assert P[pr[5], 2] == 5664741 * 2.0 ** -24 * sc
+    assert Q[pc[2], 5] == 14274654 * 2.0 ** -24 * sc
+    assert Q[pc[5], 2] == 4396063 * 2.0 ** -24 * sc
+    for u in range(m):
+        for j in range(k):
+            assert P[pr[u], j] == (H(7, 3, u, j) >> 40) * 2.0 ** -24 * sc
+    for v in range(n):
+        for j in range(k):
+            assert Q[pc[v], j] == (H(7, 4, v, j) >> 40) * 2.0 ** -24 * sc
+
+
 def test_phased_allreduce_pins(orc):
     # R22: phases = 1 is the plain all-reduce epoch (bit-exact); any phase count keeps
     # the all-reduce first-order limit (P step gamma, Q step gamma / G)

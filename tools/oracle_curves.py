@@ -9,6 +9,7 @@ one shard, grid (1, 1), shuffle seed = config seed, init seed 1, serial order.
     python tools/oracle_curves.py c1 c2 c3      # C3: ~4 min on one core
     python tools/oracle_curves.py c3:2048        # digest of the 2048 x 2048 DET partition
     python tools/oracle_curves.py det:c3:2048    # sampled P, Q rows after one DET epoch
+    python tools/oracle_curves.py ring:c3:8:8    # Hogwild-ring reference curve, G = 8, Bc = 8
 """
 import hashlib
 import json
@@ -76,8 +77,37 @@ def det_epoch_sample(name, B, rows=128):
     print(name, B, "det sample", path, f"{time.time() - t0:.0f}s", flush=True)
 
 
+def ring_curve(name, G, Bc):
+    """The oracle's serialisation of the G-shard Hogwild ring (R19: stage t, shard s,
+    its column blocks of group (s+t) mod G in order), grid (1, Bc), init seed 1: the reference
+    curve of the multi-rank band tests (tests/golden/oracle_curve_<name>_ring_G<G>_Bc<Bc>.json)."""
+    cfg = synth.CONFIGS[name]
+    (u, v, r), (tu, tv, tr) = synth.make(cfg)
+    t0 = time.time()
+    prob = oracle.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=G, Br=1, Bc=Bc, seed=cfg.seed)
+    prob.init(1)
+    digest = partition_digest(prob)
+    curve = [prob.rmse(tu, tv, tr)]
+    for _ in range(EPOCHS[name]):
+        prob.epoch("serial", "ring")
+        curve.append(prob.rmse(tu, tv, tr))
+    out = {"config": name, "workload": cfg.name, "epochs": EPOCHS[name], "G": G, "Bc": Bc, "test_rmse": curve,
+           f"partition_sha256_G{G}_grid_1x{Bc}": digest,
+           "note": "curve[0] = before training; curve[e] = after e oracle epochs in the ring serialisation "
+                   "(R19), shuffle seed = config seed, init seed 1",
+           "oracle_seconds": time.time() - t0}
+    path = os.path.join(ROOT, "tests", "golden", f"oracle_curve_{name}_ring_G{G}_Bc{Bc}.json")
+    with open(path, "w") as f:
+        json.dump(out, f, indent=1)
+    print(name, "ring", G, Bc, [round(x, 5) for x in curve], f"{out['oracle_seconds']:.0f}s", flush=True)
+
+
 def main(names):
     for name in names:
+        if name.startswith("ring:"):  # e.g. ring:c3:8:8
+            _, n_, G, Bc = name.split(":")
+            ring_curve(n_, int(G), int(Bc))
+            continue
         if name.startswith("det:"):  # e.g. det:c3:2048 -> sampled rows after one DET epoch
             _, n_, B = name.split(":")
             det_epoch_sample(n_, int(B))
