@@ -72,8 +72,9 @@ def parse():
     ap.add_argument("--task", type=int, default=0)
     ap.add_argument("--vec", type=int, default=0, help="float4 slots per lane (0 = library auto)")
     ap.add_argument("--depth", type=int, default=0, help="Hogwild q_v prefetch distance (0 = library auto)")
-    ap.add_argument("--det-wave", type=int, default=1, choices=[0, 1, 2],
-                    help="DET: 1 wavefront with Q slabs in shared memory, 2 wavefront, 0 per-stratum launches")
+    ap.add_argument("--det-wave", type=int, default=0, choices=[-1, 0, 1, 2, 3],
+                    help="DET: 0 library default, 1 wavefront with Q slabs in shared memory, 2 wavefront, "
+                         "3 chain-parallel wavefront (-1: per-stratum launches)")
     ap.add_argument("--impl", default="hccmf", choices=["hccmf", "reference"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -81,6 +82,7 @@ def parse():
     ap.add_argument("--storage", default="fp32", choices=["fp32", "fp16", "fp16sr"],
                     help="Q storage of the headline number (fp16 = binary16 Q, fp32 math, R26; "
                          "fp16sr = with stochastic rounding, R27)")
+    ap.add_argument("--col-balance", action="store_true", help="degree-balanced column blocks (R30)")
     ap.add_argument("--fp16-leg", default="fp16sr", choices=["fp16", "fp16sr", "none"],
                     help="secondary binary16-Q measurement added to the JSON line")
     return ap.parse_args()
@@ -289,7 +291,7 @@ class Ctx:
         self.args, self.rank, self.world, self.local, self.stream = args, rank, world, local, stream
 
 
-def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, sample_for_cpu=False):
+def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, sample_for_cpu=False, col_balance=False):
     """Generate `name`, partition, and measure each storage in `storages` (W warm-up + K timed
     steps from a fresh init); optionally the e2e job.  Returns a dict for the JSON line."""
     import torch
@@ -344,14 +346,14 @@ def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, samp
         mdl.set_option("vec", args.vec)
     if args.depth:
         mdl.set_option("prefetch_depth", args.depth)
-    if args.det_wave != 1:
-        mdl.set_option("det_wave", args.det_wave)
+    if args.det_wave:
+        mdl.set_option("det_wave", max(0, args.det_wave))
     torch.cuda.synchronize()
     t_prep = time.perf_counter()
     mdl.load_slice(du, dv, dr)
     del du, dv, dr
     torch.cuda.empty_cache()
-    mdl.partition(G, (Br, Bc), "DP0", seed=cfg.seed, storage=storages[0])
+    mdl.partition(G, (Br, Bc), "DP0", seed=cfg.seed, storage=storages[0], col_balance=col_balance)
     mdl.init(1)
     torch.cuda.synchronize()
     t_prep = time.perf_counter() - t_prep
@@ -411,6 +413,7 @@ def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, samp
             mdl.set_option("storage", STORAGE[storage])
             mdl.init(1)
         res["legs"][storage] = measure(storage)
+        res["det_path"] = mdl.info()["det_path"]
     mdl.close()
     torch.cuda.empty_cache()
 
@@ -446,7 +449,7 @@ def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, samp
         if args.vec:
             m2.set_option("vec", args.vec)
         m2.load_slice(pin[0], pin[1], pin[2])
-        m2.partition(G, (Br, Bc), "DP0", seed=cfg.seed, storage=storage)
+        m2.partition(G, (Br, Bc), "DP0", seed=cfg.seed, storage=storage, col_balance=col_balance)
         m2.init(1)
         for _ in range(E):
             m2.train_epoch(sched, sync)
@@ -505,7 +508,8 @@ def main():
     if args.storage == "fp32" and cfg.k % 128 == 0 and args.fp16_leg != "none":
         storages.append(args.fp16_leg)
     head = run_workload(cx, args.config, args.sched, storages, args.steps, not args.no_e2e,
-                        sample_for_cpu=(rank == 0 and world == 1 and not args.no_cpu_baseline))
+                        sample_for_cpu=(rank == 0 and world == 1 and not args.no_cpu_baseline),
+                        col_balance=args.col_balance)
     H = head["legs"][args.storage]
     info = head["info"]
     out = {"metric": METRIC, "value": H["value"], "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -514,6 +518,7 @@ def main():
            "config": {"workload": f"{cfg.name} ({args.config})", "m": cfg.m, "n": cfg.n, "nnz": head["nnz"],
                       "k": cfg.k, "test_ratings": head["nt"], "gamma": cfg.gamma, "lambda": cfg.lam,
                       "sched": args.sched, "sync": head["sync"], "grid": head["grid"], "storage": args.storage,
+                      "col_balance": bool(args.col_balance),
                       "parallelism": f"dp{world} (row shards, Q {head['sync']}; sliced ingest)",
                       "step": "1 SGD epoch over all nnz + Q sync + test RMSE",
                       "l2": "inputs larger than L2 (records %.2f GB > 126 MB); Q is L2-resident by design"
@@ -547,11 +552,12 @@ def main():
         torch.cuda.empty_cache()
     if "det" in legs:
         kd = min(args.steps, 3)
-        d = run_workload(cx, "c3", "det", ["fp32"], kd, False, det_grid=(2048, 2048))
+        d = run_workload(cx, "c3", "det", ["fp32"], kd, False, det_grid=(2048, 2048), col_balance=True)
         out["legs"]["det"] = dict(leg_json(d, "fp32", kd, args.warmup), workload=f"{d['cfg'].name} (c3)",
-                                  grid=[2048, 2048], sched="det",
-                                  note="serial-equivalent FPSGD strata (R19) as one wavefront launch per epoch; "
-                                       "bound by the hottest column block's serial chain")
+                                  grid=[2048, 2048], sched="det", det_path=d.get("det_path"), col_balance=True,
+                                  note="serial-equivalent FPSGD strata (R19) as one wavefront launch per epoch, "
+                                       "degree-balanced column blocks (R30); bound by the heaviest column "
+                                       "block's serial chain")
         d = None
         torch.cuda.empty_cache()
 

@@ -121,6 +121,13 @@ typedef struct {
                              grid every caller-facing call keeps its orientation (P is
                              still m x k, rmse takes (u, v)); get_partition, get_records
                              and hccmf_info describe the transposed problem. */
+    int32_t col_balance;  /* 0 (default): columns shuffled by the seeded hash (R8);
+                             1: degree-balanced column blocks (R30): items
+                             in order of (ratings desc, id asc) each take a slot of
+                             the least-loaded column block with a free slot (ties to
+                             the lowest block), so the heaviest column block -- the
+                             DET order's critical path -- carries about the heaviest
+                             item alone.  Rows keep the hash shuffle.             */
 } hccmf_partition_opts;
 
 typedef struct {
@@ -137,6 +144,9 @@ typedef struct {
     int32_t rank, world;     /* 0, 1 for a single-process handle                  */
     int64_t device_bytes;    /* device memory currently owned by the handle       */
     int32_t transposed;      /* 1: column grid (m, n, rows describe R^T)          */
+    int32_t det_path;        /* kernel of the last DET epoch: 0 per-stratum launches,
+                                1 slab wavefront, 2 register wavefront, 3 chain-parallel
+                                wavefront; -1 none yet                             */
 } hccmf_info;
 
 /* Tunables for hccmf_set_option (values are int64). */

@@ -49,6 +49,7 @@ def lib():
             "orc_hash": (u64, [u64, u64, u64, u64]),
             "orc_uniform": (f64, [u64]),
             "orc_perm": (ctypes.c_int, [u64, u64, i64, P]),
+            "orc_perm_balanced": (ctypes.c_int, [i64, i64, P, i32, P]),
             "orc_dp0": (None, [i32, P, P]),
             "orc_dp0_affine": (None, [i32, P, P, P]),
             "orc_dp1": (i32, [i32, P, P, P]),
@@ -113,6 +114,15 @@ def uniform(h: int) -> float:
 def perm(seed: int, tag: int, count: int) -> np.ndarray:
     out = np.empty(max(count, 0), dtype=np.int32)
     rc = lib().orc_perm(seed, tag, count, _p(out))
+    assert rc == 0
+    return out
+
+
+def perm_balanced(n: int, v, B: int) -> np.ndarray:
+    """Degree-balanced column permutation (R30): v' of every item."""
+    vv = _i32(v)
+    out = np.empty(n, dtype=np.int32)
+    rc = lib().orc_perm_balanced(n, len(vv), _p(vv), B, _p(out))
     assert rc == 0
     return out
 
@@ -282,12 +292,12 @@ def unpermute(perm_, Xp) -> np.ndarray:
 class Problem:
     """Convenience: the whole oracle pipeline for one problem (tests only)."""
 
-    def __init__(self, m, n, k, gamma, lam, u, v, r, G=1, Br=1, Bc=1, seed=0, x=None):
+    def __init__(self, m, n, k, gamma, lam, u, v, r, G=1, Br=1, Bc=1, seed=0, x=None, col_balance=0):
         self.m, self.n, self.k, self.gamma, self.lam = m, n, k, gamma, lam
         self.u, self.v, self.r = _i32(u), _i32(v), _f32(r)
         self.G, self.Br, self.Bc = G, Br, Bc
         self.perm_row = perm(seed, 1, m)
-        self.perm_col = perm(seed, 2, n)
+        self.perm_col = perm_balanced(n, self.v, Bc) if col_balance else perm(seed, 2, n)
         self.S = row_prefix(m, self.u, self.perm_row)
         self.x = np.full(G, 1.0 / G) if x is None else _f64(x)
         self.b = bounds(m, len(self.u), self.S, G, self.x)

@@ -88,6 +88,56 @@ int orc_perm(uint64_t seed, uint64_t tag, int64_t count, int32_t* perm)
 }
 
 /* ------------------------------------------------------------------------- */
+/* Degree-balanced column permutation (R30): "shuffling" exists to    */
+/* balance the blocks (L546); under the DET order every rating of a column      */
+/* block is serialised through the block's owners one row block after another,   */
+/* so the heaviest column block is the epoch's critical path.  Items are taken  */
+/* in order of (degree descending, id ascending); each goes to the column block  */
+/* with the least load (sum of degrees) among those with a free slot, ties to    */
+/* the lowest block index, and takes that block's next slot.  Column block c    */
+/* holds v' in [ceil(c n / B), ceil((c+1) n / B)) (a4), so it has that many     */
+/* slots.  deg[v] = number of ratings of item v (original ids).                 */
+/* ------------------------------------------------------------------------- */
+typedef struct { int64_t deg; int64_t id; } orc_degid;
+
+static int cmp_degid(const void* a, const void* b)
+{
+    const orc_degid* x = (const orc_degid*)a;
+    const orc_degid* y = (const orc_degid*)b;
+    if (x->deg != y->deg) return x->deg > y->deg ? -1 : 1;
+    if (x->id != y->id) return x->id < y->id ? -1 : 1;
+    return 0;
+}
+
+int orc_perm_balanced(int64_t n, int64_t nnz, const int32_t* v, int32_t B, int32_t* perm)
+{
+    if (n < 1 || B < 1 || nnz < 0) return -1;
+    orc_degid* it = (orc_degid*)malloc(sizeof(orc_degid) * (size_t)n);
+    int64_t* load = (int64_t*)calloc((size_t)B, sizeof(int64_t));
+    int64_t* used = (int64_t*)calloc((size_t)B, sizeof(int64_t));
+    if (!it || !load || !used) return -3;
+    for (int64_t x = 0; x < n; ++x) { it[x].deg = 0; it[x].id = x; }
+    for (int64_t i = 0; i < nnz; ++i) it[v[i]].deg += 1;
+    qsort(it, (size_t)n, sizeof(orc_degid), cmp_degid);
+    for (int64_t x = 0; x < n; ++x) {
+        int32_t best = -1;
+        for (int32_t c = 0; c < B; ++c) {
+            const int64_t start = ((int64_t)c * n + B - 1) / B, end = ((int64_t)(c + 1) * n + B - 1) / B;
+            if (used[c] >= end - start) continue;  /* no free slot */
+            if (best < 0 || load[c] < load[best]) best = c;
+        }
+        const int64_t start = ((int64_t)best * n + B - 1) / B;
+        perm[it[x].id] = (int32_t)(start + used[best]);
+        used[best] += 1;
+        load[best] += it[x].deg;
+    }
+    free(it);
+    free(load);
+    free(used);
+    return 0;
+}
+
+/* ------------------------------------------------------------------------- */
 /* Data partition strategies (section 3.3).                        */
 /* ------------------------------------------------------------------------- */
 

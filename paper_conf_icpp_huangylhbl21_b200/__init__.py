@@ -51,7 +51,7 @@ class PartitionOpts(ctypes.Structure):
     _fields_ = [("n_shards", ctypes.c_int32), ("grid_rows", ctypes.c_int32), ("grid_cols", ctypes.c_int32),
                 ("strategy", ctypes.c_int32), ("x", ctypes.c_void_p), ("t_meas", ctypes.c_void_p),
                 ("t_sync", ctypes.c_double), ("seed", ctypes.c_uint64), ("storage", ctypes.c_int32),
-                ("grid_dim", ctypes.c_int32)]
+                ("grid_dim", ctypes.c_int32), ("col_balance", ctypes.c_int32)]
 
 
 class Info(ctypes.Structure):
@@ -60,7 +60,7 @@ class Info(ctypes.Structure):
                 ("local_nnz", ctypes.c_int64), ("row0", ctypes.c_int64), ("rows", ctypes.c_int64),
                 ("n_blocks", ctypes.c_int64), ("n_tasks", ctypes.c_int64), ("key_bits", ctypes.c_int32),
                 ("rank", ctypes.c_int32), ("world", ctypes.c_int32), ("device_bytes", ctypes.c_int64),
-                ("transposed", ctypes.c_int32)]
+                ("transposed", ctypes.c_int32), ("det_path", ctypes.c_int32)]
 
     def as_dict(self):
         return {f: getattr(self, f) for f, _ in self._fields_}
@@ -303,16 +303,17 @@ class Model:
         return dict(zip(COMM_SITES, c.tolist()))
 
     def partition(self, n_shards=1, grid=(1, 1), strategy="DP0", seed=0, x=None, t_meas=None, t_sync=0.0,
-                  grid_dim="rows", storage="fp32"):
+                  grid_dim="rows", storage="fp32", col_balance=False):
         """grid_dim: "rows" (shards of users, Q moves), "cols" (shards of items, P moves) or
         "auto" (the paper's rule, L884-L886).  storage: "fp32"; "fp16" = Q held in IEEE
         binary16 during epochs, fp32 arithmetic, round to nearest (R26; k a multiple
-        of 128); "fp16sr" = the same with stochastic rounding of every q write (R27)."""
+        of 128); "fp16sr" = the same with stochastic rounding of every q write (R27).
+        col_balance: degree-balanced column blocks instead of the hash shuffle of columns (R30)."""
         px, kx = _buf(x, np.float64)
         pt, kt = _buf(t_meas, np.float64)
         o = PartitionOpts(int(n_shards), int(grid[0]), int(grid[1]), DP[strategy] if isinstance(strategy, str)
                           else int(strategy), px, pt, float(t_sync), int(seed), {"fp32": 0, "fp16": 1, "fp16sr": 2}[storage],
-                          {"rows": 0, "cols": 1, "auto": 2}[grid_dim])
+                          {"rows": 0, "cols": 1, "auto": 2}[grid_dim], int(bool(col_balance)))
         self._check(lib().hccmf_partition(self._h, ctypes.byref(o)))
         self.G, self.grid = int(n_shards), (int(grid[0]), int(grid[1]))
 

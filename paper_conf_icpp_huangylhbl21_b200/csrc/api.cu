@@ -3,6 +3,8 @@
 // launch plans for every (schedule, sync) pair, the ring / all-reduce Q
 // synchronisation over NCCL, and export.
 #include <algorithm>
+#include <functional>
+#include <queue>
 #include <chrono>
 #include <cmath>
 #include <cstdarg>
@@ -229,6 +231,7 @@ void free_partition(hccmf_t h) {
   h->n_counters = 0;
   dfree(h, h->d_blk_off, h->nblk_local + 1);
   dfree(h, h->d_progress, h->Br);
+  det_chain_free(&h->det_chain, h->stream);
   h->local_nnz = 0;
   h->rows = 0;
   h->blk_task_off.clear();
@@ -664,7 +667,7 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
       h->opt_phases = value;
       return HCCMF_OK;
     case HCCMF_OPT_DET_WAVE:
-      if (value < 0 || value > 2) return fail(h, HCCMF_EINVAL, "det_wave must be 0, 1 or 2");
+      if (value < 0 || value > 3) return fail(h, HCCMF_EINVAL, "det_wave must be 0, 1, 2 or 3");
       h->opt_wave = (int)value;
       return HCCMF_OK;
     case HCCMF_OPT_VEC:
@@ -810,7 +813,41 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   CU(h, dmalloc(h, &h->d_perm_row, m));
   CU(h, dmalloc(h, &h->d_perm_col, n));
   CU(h, k_perm(h->seed, 1, m, h->d_perm_row, st));
-  CU(h, k_perm(h->seed, 2, n, h->d_perm_col, st));
+  if (o->col_balance) {
+    // R30: degree-balanced column blocks -- item degrees (global under sliced ingest), then
+    // least-loaded placement in order of (degree desc, id asc), ties to the lowest block
+    unsigned long long* dDeg = nullptr;
+    CU(h, cudaMallocAsync((void**)&dDeg, sizeof(unsigned long long) * n, st));
+    CU(h, k_item_degree(h->d_in_v, h->nnz_in, n, dDeg, st));
+    if (h->sliced) {
+      h->comm_counts[SITE_INGEST_HIST] += 1;
+      CM(h, h->comm->allreduce(dDeg, dDeg, (size_t)n, DType::u64, ROp::sum, st));
+    }
+    std::vector<unsigned long long> deg(n);
+    CU(h, cudaMemcpyAsync(deg.data(), dDeg, sizeof(unsigned long long) * n, cudaMemcpyDeviceToHost, st));
+    CU(h, cudaStreamSynchronize(st));
+    cudaFreeAsync(dDeg, st);
+    std::vector<int32_t> order(n), pc(n);
+    for (int64_t x = 0; x < n; ++x) order[x] = (int32_t)x;
+    std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) { return deg[a] > deg[b]; });
+    const int64_t Bc = o->grid_cols;
+    std::vector<int64_t> used(Bc, 0);
+    using LB = std::pair<unsigned long long, int64_t>;  // (load, block): least load, then lowest block
+    std::priority_queue<LB, std::vector<LB>, std::greater<LB>> heap;
+    for (int64_t c = 0; c < Bc; ++c)
+      if (ceil_div((c + 1) * n, Bc) > ceil_div(c * n, Bc)) heap.push({0ull, c});
+    for (int64_t x = 0; x < n; ++x) {
+      const LB top = heap.top();
+      heap.pop();
+      const int64_t c = top.second, start = ceil_div(c * n, Bc), width = ceil_div((c + 1) * n, Bc) - start;
+      pc[order[x]] = (int32_t)(start + used[c]);
+      if (++used[c] < width) heap.push({top.first + deg[order[x]], c});
+    }
+    CU(h, cudaMemcpyAsync(h->d_perm_col, pc.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice, st));
+    CU(h, cudaStreamSynchronize(st));
+  } else {
+    CU(h, k_perm(h->seed, 2, n, h->d_perm_col, st));
+  }
 
   timer.mark("a2 shuffle");
   // ---- a3 row histogram, prefix, boundaries
@@ -1079,7 +1116,32 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     if (L != 32 || L * VEC * 4 != h->k)
       return fail(h, HCCMF_EINVAL, "binary16 Q storage needs one rating per warp (k a multiple of 128, vec = k/128)");
   }
-  const bool wave_slab = sched == HCCMF_SCHED_DET && G == 1 && h->opt_wave == 1 && h->storage == 0 &&
+  int chain_ng = 0, chain_su = 0;
+  if (sched == HCCMF_SCHED_DET && G == 1 && h->opt_wave == 3 && h->storage == 0 && h->Br == h->Bc && h->Br > 1 &&
+      h->local_nnz > 0 && det_chain_plan(h->k, h->Br, h->n, &chain_ng, &chain_su)) {
+    // DET as the chain-parallel wavefront: the same per-row update sequences as the strata (R19)
+    DetChain& dc = h->det_chain;
+    if (dc.B != h->Br || dc.NG != chain_ng || dc.SU != chain_su) {
+      det_chain_free(&dc, h->stream);
+      cudaError_t e = k_det_chain_schedule(h->d_u, h->d_v, h->d_r, h->d_blk_off, h->nblk_local, h->Bc, h->n, chain_ng,
+                                           chain_su, &dc, h->stream);
+      if (e != cudaSuccess) {
+        det_chain_free(&dc, h->stream);
+        CU(h, e);
+      }
+      dc.B = h->Br;
+    }
+    cudaError_t e = launch_wave_chain(dc, h->d_P, h->d_Q, h->row0, h->n, h->k, h->gamma, h->lambda, h->Br,
+                                      h->d_progress, h->stream);
+    if (e == cudaSuccess) {
+      h->det_path = 3;
+      ++h->epoch;
+      return finish(h);
+    }
+    if (e != cudaErrorCooperativeLaunchTooLarge) CU(h, e);
+    cudaGetLastError();
+  }
+  const bool wave_slab = sched == HCCMF_SCHED_DET && G == 1 && (h->opt_wave == 1 || h->opt_wave == 3) && h->storage == 0 &&
                          h->Br == h->Bc && h->Br > 1 && wave_slab_supported(h->k, (int)h->opt_vec, h->Br, h->n);
   if (wave_slab || (sched == HCCMF_SCHED_DET && G == 1 && h->opt_wave && h->storage == 0 && h->Br == h->Bc &&
                     h->Br > 1 && wave_supported(h->k, (int)h->opt_vec, h->Br))) {
@@ -1099,6 +1161,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     cudaError_t e = wave_slab ? launch_wave_slab(a, h->d_blk_off, h->Br, h->d_progress, h->n, h->stream)
                               : launch_wave(a, h->d_blk_off, h->Br, h->d_progress, h->stream);
     if (e == cudaSuccess) {
+      h->det_path = wave_slab ? 1 : 2;
       ++h->epoch;
       return finish(h);
     }
@@ -1110,6 +1173,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   Plan* pl = nullptr;
   hccmf_status st = build_plan(h, sched, sync, &pl);
   if (st != HCCMF_OK) return st;
+  if (sched == HCCMF_SCHED_DET) h->det_path = 0;
   const int eff_sync = (G == 1) ? HCCMF_SYNC_NONE : sync;
   const bool dist = h->world > 1;
   const int64_t nk = h->n * h->k;
@@ -1541,6 +1605,7 @@ hccmf_status hccmf_get_info(hccmf_t h, hccmf_info* o) {
   o->world = h->world;
   o->device_bytes = (int64_t)h->device_bytes;
   o->transposed = h->transposed ? 1 : 0;
+  o->det_path = h->det_path;
   return HCCMF_OK;
 }
 

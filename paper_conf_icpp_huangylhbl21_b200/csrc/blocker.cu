@@ -252,6 +252,11 @@ __global__ void permute_tasks_kernel(const int64_t* idx, int64_t nt, const int64
   }
 }
 
+__global__ void item_degree_kernel(const int32_t* __restrict__ v, int64_t nnz, unsigned long long* cnt) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nnz; i += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(cnt + v[i], 1ull);
+}
+
 // sliced ingest: destination shard of every rating (key) and its input index (value)
 __global__ void shard_key_kernel(const int32_t* __restrict__ u, int64_t nnz, const int32_t* __restrict__ perm_row,
                                  const int32_t* __restrict__ bounds, int32_t G, uint32_t* key, int64_t* idx,
@@ -341,6 +346,15 @@ cudaError_t k_row_prefix(const int32_t* u, int64_t nnz, const int32_t* perm_row,
   cudaFreeAsync(tmp, st);
   cudaFreeAsync(cnt, st);
   return cudaGetLastError();
+}
+
+cudaError_t k_item_degree(const int32_t* v, int64_t nnz, int64_t n, unsigned long long* deg, cudaStream_t st) {
+  CKR(cudaMemsetAsync(deg, 0, sizeof(unsigned long long) * n, st));
+  if (nnz) {
+    (note_launch(), item_degree_kernel<<<grid_for(nnz), kT, 0, st>>>(v, nnz, deg));
+    CKR(cudaGetLastError());
+  }
+  return cudaSuccess;
 }
 
 cudaError_t k_bound_search(const unsigned long long* S, int64_t m, const int64_t* targets, int32_t nt, int64_t* out,

@@ -89,6 +89,25 @@ cudaError_t launch_wave(const SgdArgs& a, const int64_t* off /* local block offs
 bool wave_slab_supported(int k, int vec_pref, int B, int64_t n);
 cudaError_t launch_wave_slab(const SgdArgs& a, const int64_t* off, int B, int* progress, int64_t n,
                              cudaStream_t st);
+// DET as the chain-parallel wavefront (detchain.cu): the per-partition schedule
+struct DetChain {
+  int32_t* cv = nullptr;       // records reordered group by group inside each segment
+  float* cr = nullptr;
+  uint32_t* meta = nullptr;    // p slot | dependency (group, index)
+  int64_t* blk_seg = nullptr;  // nblk + 1: segments of each block
+  int64_t* seg_lo = nullptr;   // nseg + 1: first record of each segment
+  int64_t* seg_run = nullptr;  // nseg + 1: first user run of each segment
+  uint16_t* seg_gend = nullptr;// 4 per segment: group ends inside the segment
+  int32_t* run_user = nullptr; // nrun: the user of each run
+  int64_t nseg = 0, nrun = 0, nrec = 0;
+  int NG = 0, SU = 0, B = 0;
+};
+bool det_chain_plan(int k, int B, int64_t n, int* NG, int* SU);
+cudaError_t k_det_chain_schedule(const int32_t* ru, const int32_t* rv, const float* rr, const int64_t* off,
+                                 int64_t nblk, int Bc, int64_t n, int NG, int SU, DetChain* out, cudaStream_t st);
+void det_chain_free(DetChain* d, cudaStream_t st);
+cudaError_t launch_wave_chain(const DetChain& d, float* P, float* Q, int64_t row0, int64_t n, int32_t k, float gamma,
+                              float lambda, int B, int* progress, cudaStream_t st);
 // lane geometry of the SGD kernel: L lanes per rating group, VEC float4 per lane
 void sgd_geometry(int k, int vec_pref, int* L, int* VEC);
 int sgd_lanes(int k, int vec_pref);
@@ -110,6 +129,7 @@ cudaError_t k_validate(const int32_t* u, const int32_t* v, const float* r, int64
 cudaError_t k_perm(uint64_t seed, uint64_t tag, int64_t count, int32_t* perm, cudaStream_t st);
 cudaError_t k_row_prefix(const int32_t* u, int64_t nnz, const int32_t* perm_row, int64_t m,
                          unsigned long long* S /* m+1 */, cudaStream_t st);
+cudaError_t k_item_degree(const int32_t* v, int64_t nnz, int64_t n, unsigned long long* deg /* n */, cudaStream_t st);
 cudaError_t k_bound_search(const unsigned long long* S, int64_t m, const int64_t* targets, int32_t nt,
                            int64_t* out, cudaStream_t st);
 cudaError_t k_block_sort(const BlockGeom& g, const int32_t* bounds, const int32_t* perm_row,
@@ -214,8 +234,10 @@ struct hccmf_ctx {
   double* d_scalar = nullptr;
   int64_t* d_blk_off = nullptr;  // local block offsets (DET wavefront), nblk_local + 1
   int* d_progress = nullptr;     // wavefront progress counters, Br
+  hccmf::DetChain det_chain;     // chain-parallel DET schedule (built at the first such epoch)
 
   bool transposed = false;  // column grid: internal rows are the caller's columns
+  int det_path = -1;        // kernel of the last DET epoch (hccmf_info.det_path)
   int q_ring_sched = -1;  // >= 0: distributed ring left only this rank's Q group valid
   std::vector<hccmf::Plan> plans;
 };

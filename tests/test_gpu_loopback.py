@@ -209,8 +209,8 @@ def test_loopback_wire16_allreduce_is_one_rounding(pkg, orc):
         assert np.array_equal(Q, Ql) and np.array_equal(P, Pl)
 
 
-@pytest.mark.parametrize("G,Br,Bc", [(2, 4, 8), (3, 5, 7), (4, 8, 32), (4, 1, 4)])
-def test_loopback_sliced_ingest_concatenates_to_single_process(pkg, orc, G, Br, Bc):
+@pytest.mark.parametrize("G,Br,Bc,bal", [(2, 4, 8, 0), (3, 5, 7, 0), (4, 8, 32, 0), (4, 1, 4, 0), (3, 2, 6, 1)])
+def test_loopback_sliced_ingest_concatenates_to_single_process(pkg, orc, G, Br, Bc, bal):
     # each rank loads 1/G (uneven, one empty) of the COO; the exchange + local sort reproduce the
     # single-process partition: perms, bounds, global block offsets and every shard's records
     cfg = synth.scaled(synth.CONFIGS["c2"], 0.02)
@@ -221,12 +221,12 @@ def test_loopback_sliced_ingest_concatenates_to_single_process(pkg, orc, G, Br, 
     edges = [0, *cuts.tolist(), nnz]
     if G >= 3:
         edges[2] = edges[1]  # rank 1 loads nothing
-    prob = orc.Problem(cfg.m, cfg.n, 32, cfg.gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=Bc, seed=9)
+    prob = orc.Problem(cfg.m, cfg.n, 32, cfg.gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=Bc, seed=9, col_balance=bal)
 
     def body(rank, mdl):
         a, b = edges[rank], edges[rank + 1]
         mdl.load_slice(u[a:b], v[a:b], r[a:b])
-        mdl.partition(G, (Br, Bc), seed=9)
+        mdl.partition(G, (Br, Bc), seed=9, col_balance=bool(bal))
         return mdl.get_partition(), mdl.records(), mdl.info(), mdl.comm_counts()
 
     res = run_ranks(pkg, G, cfg.m, cfg.n, 32, cfg.gamma, cfg.lam, body)
@@ -238,7 +238,7 @@ def test_loopback_sliced_ingest_concatenates_to_single_process(pkg, orc, G, Br, 
         assert inf["nnz"] == nnz and inf["local_nnz"] == hi - lo
         assert np.array_equal(gu, prob.ru[lo:hi]) and np.array_equal(gv, prob.rv[lo:hi])
         assert np.array_equal(gr.view(np.int32), prob.rr[lo:hi].view(np.int32))
-        assert cc["ingest_hist"] == 1 and cc["ingest_exchange"] == 1 and cc["ingest_blocks"] == 1
+        assert cc["ingest_hist"] == 1 + bal and cc["ingest_exchange"] == 1 and cc["ingest_blocks"] == 1
 
 
 def test_loopback_sliced_ingest_trains_like_replicated(pkg, orc):

@@ -27,10 +27,10 @@ def pkg():
 
 
 def _gpu_problem(pkg, m, n, k, gamma, lam, u, v, r, G=1, Br=1, Bc=1, seed=0, strategy="DP0", x=None, t_meas=None,
-                 t_sync=0.0):
+                 t_sync=0.0, col_balance=False):
     mdl = pkg.Model(m, n, k, gamma, lam)
     mdl.load(u, v, r)
-    mdl.partition(G, (Br, Bc), strategy, seed=seed, x=x, t_meas=t_meas, t_sync=t_sync)
+    mdl.partition(G, (Br, Bc), strategy, seed=seed, x=x, t_meas=t_meas, t_sync=t_sync, col_balance=col_balance)
     return mdl
 
 
@@ -338,6 +338,112 @@ def test_det_wavefront_equals_strata(pkg, orc, k, B, dup):
         assert np.array_equal(outs[0][0], o[0]) and np.array_equal(outs[0][1], o[1])
     Po, Qo = prob.factors()
     assert max(np.abs(outs[0][0] - Po).max(), np.abs(outs[0][1] - Qo).max()) <= 1e-4
+
+
+def test_partition_col_balance_bitexact(pkg, orc):
+    # R30: the degree-balanced column permutation (host least-loaded placement from the GPU
+    # item histogram) and the resulting blocks equal the oracle's bit for bit
+    rng = np.random.default_rng(17)
+    for trial in range(60):
+        m, n = int(rng.integers(1, 15)), int(rng.integers(1, 15))
+        nnz = int(rng.integers(0, 120))
+        G = int(rng.integers(1, min(m, 3) + 1))
+        Br, Bc = int(rng.integers(1, 5)), int(rng.integers(1, 6))
+        u, v, r = synth.tiny(m, n, nnz, seed=trial)
+        prob = orc.Problem(m, n, 4, 0.01, 0.01, u, v, r, G=G, Br=Br, Bc=Bc, seed=trial % 3, col_balance=1)
+        mdl = _gpu_problem(pkg, m, n, 4, 0.01, 0.01, u, v, r, G=G, Br=Br, Bc=Bc, seed=trial % 3, col_balance=True)
+        _check_partition(mdl, prob)
+        mdl.close()
+    cfg = synth.scaled(synth.CONFIGS["c2"], 0.05)
+    (u, v, r), _ = synth.make(cfg)
+    for G, Br, Bc in [(1, 16, 16), (2, 4, 8), (1, 1, 37)]:
+        prob = orc.Problem(cfg.m, cfg.n, 32, cfg.gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=Bc, seed=5, col_balance=1)
+        mdl = _gpu_problem(pkg, cfg.m, cfg.n, 32, cfg.gamma, cfg.lam, u, v, r, G=G, Br=Br, Bc=Bc, seed=5,
+                           col_balance=True)
+        _check_partition(mdl, prob)
+        mdl.close()
+
+
+@pytest.mark.parametrize("wave,B", [(1, 8), (1, 24), (0, 8), (3, 12)])
+def test_det_epoch_parity_col_balance(pkg, orc, wave, B):
+    # the DET order on degree-balanced column blocks (R30): every wavefront / the strata
+    # against the oracle's serial run of the same partition, 1e-4
+    cfg = synth.CONFIGS["c1"]
+    (u, v, r), _ = synth.make(cfg)
+    rng = np.random.default_rng(B)
+    v = (rng.zipf(1.4, len(u)) % cfg.n).astype(np.int32)  # skewed items: balancing moves them
+    prob = orc.Problem(cfg.m, cfg.n, 128, 0.02, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=6, col_balance=1)
+    prob.init(2)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    mdl = _gpu_problem(pkg, cfg.m, cfg.n, 128, 0.02, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=6, col_balance=True)
+    _check_partition(mdl, prob)
+    mdl.set_option("det_wave", wave)
+    mdl.set_factors(P0, Q0)
+    for _ in range(2):
+        mdl.train_epoch("det", "none")
+        prob.epoch("det", "none")
+    P, Q = mdl.factors()
+    Po, Qo = prob.factors()
+    assert max(np.abs(P - Po).max(), np.abs(Q - Qo).max()) <= 1e-4
+
+
+@pytest.mark.parametrize("k,B,skew,dup", [(128, 8, False, False), (128, 8, True, True), (128, 24, True, False),
+                                           (256, 12, True, True), (128, 37, False, True), (128, 3, True, False)])
+def test_det_chain_wavefront_parity(pkg, orc, k, B, skew, dup):
+    # det_wave 3: the chain-parallel wavefront (detchain.cu) keeps every P row's and Q row's
+    # update sequence of the DET order (R19) while 4 lane groups walk different item chains
+    # of a block: the oracle to 1e-4, deterministic (two runs bit-identical), one launch per
+    # epoch once the schedule is built.  skew: Zipf items (long chains, many users shared by
+    # several chains of a block: cross-group waits); dup: duplicated cells; B = 8 blocks
+    # hold ~125 users each (several shared-memory segments per block).
+    cfg = synth.CONFIGS["c1"]
+    (u, v, r), _ = synth.make(cfg)
+    if skew:
+        rng = np.random.default_rng(B)
+        v = (rng.zipf(1.4, len(u)) % cfg.n).astype(np.int32)
+    if dup:
+        u, v, r = (np.concatenate([x[:30000], x[:15000]]) for x in (u, v, r))
+    prob = orc.Problem(cfg.m, cfg.n, k, 0.02, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=6)
+    prob.init(2)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    outs = []
+    for rep in range(2):
+        mdl = _gpu_problem(pkg, cfg.m, cfg.n, k, 0.02, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=6)
+        mdl.set_option("det_wave", 3)
+        mdl.set_factors(P0, Q0)
+        mdl.train_epoch("det", "none")  # builds the chain schedule
+        assert mdl.info()["det_path"] == (3 if -(-cfg.n // B) <= 64 else 1)  # wmax > 64: the slab wavefront
+        l0 = pkg.kernel_launches()
+        mdl.train_epoch("det", "none")
+        assert pkg.kernel_launches() - l0 == 1
+        outs.append(mdl.factors())
+        mdl.close()
+    for _ in range(2):
+        prob.epoch("det", "none")
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
+    Po, Qo = prob.factors()
+    assert max(np.abs(outs[0][0] - Po).max(), np.abs(outs[0][1] - Qo).max()) <= 1e-4
+
+
+@pytest.mark.parametrize("m,n,nnz,B", [(50, 20, 3000, 37), (40, 300, 4000, 2), (300, 7, 2500, 5), (1, 9, 40, 3),
+                                       (9, 1, 40, 4), (30, 30, 0, 6)])
+def test_det_chain_wavefront_degenerate_grids(pkg, orc, m, n, nnz, B):
+    u, v, r = synth.tiny(m, n, nnz, seed=m + n + B)
+    prob = orc.Problem(m, n, 128, 0.02, 0.01, u, v, r, G=1, Br=B, Bc=B, seed=9)
+    prob.init(5)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    mdl = _gpu_problem(pkg, m, n, 128, 0.02, 0.01, u, v, r, G=1, Br=B, Bc=B, seed=9)
+    mdl.set_option("det_wave", 3)
+    mdl.set_factors(P0, Q0)
+    mdl.train_epoch("det", "none")
+    P, Q = mdl.factors()
+    mdl.close()
+    prob.epoch("det", "none")
+    Po, Qo = prob.factors()
+    assert max(np.abs(P - Po).max(), np.abs(Q - Qo).max()) <= 1e-4
 
 
 def test_column_grid_is_the_transposed_row_grid(pkg, orc):

@@ -159,3 +159,63 @@ def test_dp2_hidden_sync_ramp(orc):
     np.testing.assert_allclose(d, d[0], rtol=1e-12)
     # ramp step relative to the median time equals t_sync / T_med
     assert d[0] / pred[2] == pytest.approx(0.1, rel=1e-12)
+
+
+# ----------------------------------------- degree-balanced column blocks (R30)
+def _col_blocks(n, B):
+    return [(-(-c * n // B), -(-(c + 1) * n // B)) for c in range(B)]
+
+
+def test_balanced_perm_hand_example(orc):
+    # n = 5 items, B = 2 column blocks (slots [0, 3) and [3, 5)); degrees
+    # item: 0 1 2 3 4 -> 1 5 3 5 2.  Order (degree desc, id asc): 1 (5), 3 (5), 2 (3), 4 (2), 0 (1).
+    #   1 -> block 0 (loads 0, 0: tie -> lowest)     slot 0      loads (5, 0)
+    #   3 -> block 1                                  slot 3      loads (5, 5)
+    #   2 -> block 0 (tie)                            slot 1      loads (8, 5)
+    #   4 -> block 1                                  slot 4      loads (8, 7), block 1 full
+    #   0 -> block 0 (only free slot)                 slot 2      loads (9, 7)
+    v = np.array([0] + [1] * 5 + [2] * 3 + [3] * 5 + [4] * 2, np.int32)
+    assert list(orc.perm_balanced(5, v, 2)) == [2, 0, 1, 3, 4]
+    # B = 1: one block, slots in degree order
+    assert list(orc.perm_balanced(5, v, 1)) == [4, 0, 2, 1, 3]
+
+
+def test_balanced_perm_invariants(orc):
+    # a permutation whose blocks have exactly their a4 widths and whose loads add up to nnz;
+    # on skewed data its heaviest block is lighter than the hash shuffle's in aggregate (a
+    # reversed order or a max-load rule would make it heavier)
+    rng = np.random.default_rng(3)
+    tot_bal = tot_hash = 0
+    for trial in range(60):
+        n = int(rng.integers(1, 200))
+        B = int(rng.integers(1, min(n, 40) + 1))
+        nnz = int(rng.integers(0, 3000))
+        v = (rng.zipf(1.5, nnz) % n).astype(np.int32) if trial % 2 else rng.integers(0, n, nnz).astype(np.int32)
+        pc = orc.perm_balanced(n, v, B)
+        assert np.array_equal(np.sort(pc), np.arange(n))
+        deg = np.bincount(v, minlength=n)
+        widths = [b - a for a, b in _col_blocks(n, B)]
+        loads = np.array([deg[(pc >= a) & (pc < b)].sum() for a, b in _col_blocks(n, B)])
+        assert loads.sum() == nnz and sum(widths) == n
+        ph = orc.perm(7, 2, n)
+        tot_bal += loads.max()
+        tot_hash += max(deg[(ph >= a) & (ph < b)].sum() for a, b in _col_blocks(n, B))
+    assert tot_bal < tot_hash, (tot_bal, tot_hash)
+
+
+def test_balanced_perm_partition_is_a_valid_block_sort(orc):
+    # Problem(col_balance=1): the sort invariants of section 8(c) c1.4 hold with the new
+    # column ids (every rating kept once, each record inside its column block)
+    u, v, r = synth_tiny()
+    for B in (1, 2, 5):
+        prob = orc.Problem(40, 30, 4, 0.01, 0.01, u, v, r, G=1, Br=B, Bc=B, seed=3, col_balance=1)
+        assert np.array_equal(np.sort(prob.perm_col), np.arange(30))
+        cb = (prob.rv.astype(np.int64) * B) // 30
+        blocks = np.repeat(np.arange(B * B), np.diff(prob.off))
+        assert np.array_equal(blocks % B, cb)
+        assert sorted(zip(prob.perm_row[u], prob.perm_col[v])) == sorted(zip(prob.ru, prob.rv))
+
+
+def synth_tiny():
+    import synth
+    return synth.tiny(40, 30, 500, seed=11)

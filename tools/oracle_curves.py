@@ -10,6 +10,7 @@ one shard, grid (1, 1), shuffle seed = config seed, init seed 1, serial order.
     python tools/oracle_curves.py c3:2048        # digest of the 2048 x 2048 DET partition
     python tools/oracle_curves.py det:c3:2048    # sampled P, Q rows after one DET epoch
     python tools/oracle_curves.py ring:c3:8:8    # Hogwild-ring reference curve, G = 8, Bc = 8
+    python tools/oracle_curves.py det:c3:2048:bal  # the same DET sample with degree-balanced columns (R30)
 """
 import hashlib
 import json
@@ -35,20 +36,22 @@ def partition_digest(prob):
     return h.hexdigest()
 
 
-def det_digest(name, B):
+def det_digest(name, B, bal=0):
     cfg = synth.CONFIGS[name]
     (u, v, r), _ = synth.make(cfg)
-    prob = oracle.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=cfg.seed)
+    prob = oracle.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=cfg.seed,
+                          col_balance=bal)
     path = os.path.join(ROOT, "tests", "golden", f"oracle_curve_{name}.json")
     with open(path) as f:
         out = json.load(f)
-    out[f"partition_sha256_grid_{B}x{B}"] = partition_digest(prob)
+    key = f"partition_sha256_grid_{B}x{B}" + ("_bal" if bal else "")
+    out[key] = partition_digest(prob)
     with open(path, "w") as f:
         json.dump(out, f, indent=1)
-    print(name, B, out[f"partition_sha256_grid_{B}x{B}"], flush=True)
+    print(name, B, out[key], flush=True)
 
 
-def det_epoch_sample(name, B, rows=128):
+def det_epoch_sample(name, B, rows=128, bal=0):
     """One DET epoch (B x B grid, the bench's DET configuration: shuffle seed = config
     seed, init seed 1) by the oracle; stores `rows` sampled rows of P and of Q (the
     heaviest users / items first, then uniform draws) as float32 in
@@ -57,7 +60,8 @@ def det_epoch_sample(name, B, rows=128):
     cfg = synth.CONFIGS[name]
     (u, v, r), _ = synth.make(cfg)
     t0 = time.time()
-    prob = oracle.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=cfg.seed)
+    prob = oracle.Problem(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, u, v, r, G=1, Br=B, Bc=B, seed=cfg.seed,
+                          col_balance=bal)
     prob.init(1)
     prob.epoch("det", "none")
     P, Q = prob.factors()
@@ -70,10 +74,12 @@ def det_epoch_sample(name, B, rows=128):
         return np.sort(np.concatenate([top, rest])).astype(np.int64)
 
     iu, iv = pick(cu, cfg.m), pick(cv, cfg.n)
-    path = os.path.join(ROOT, "tests", "golden", f"oracle_det_{name}_B{B}.npz")
+    path = os.path.join(ROOT, "tests", "golden", f"oracle_det_{name}_B{B}{'_bal' if bal else ''}.npz")
     np.savez_compressed(path, users=iu, items=iv, P=P[iu].astype(np.float32), Q=Q[iv].astype(np.float32),
+                        digest=np.array(partition_digest(prob)),
                         note=np.array("oracle DET epoch 1 from init(1), shuffle seed = config seed, "
-                                      f"grid {B}x{B}; rows of P (users) and Q (items) in original ids"))
+                                      f"grid {B}x{B}{', degree-balanced columns (R30)' if bal else ''}; rows of P "
+                                      "(users) and Q (items) in original ids; digest = the partition's SHA-256"))
     print(name, B, "det sample", path, f"{time.time() - t0:.0f}s", flush=True)
 
 
@@ -108,13 +114,13 @@ def main(names):
             _, n_, G, Bc = name.split(":")
             ring_curve(n_, int(G), int(Bc))
             continue
-        if name.startswith("det:"):  # e.g. det:c3:2048 -> sampled rows after one DET epoch
-            _, n_, B = name.split(":")
-            det_epoch_sample(n_, int(B))
+        if name.startswith("det:"):  # e.g. det:c3:2048[:bal] -> sampled rows after one DET epoch
+            parts = name.split(":")
+            det_epoch_sample(parts[1], int(parts[2]), bal=int(len(parts) > 3 and parts[3] == "bal"))
             continue
-        if ":" in name:  # e.g. c3:2048 -> digest of the B x B DET partition only
-            n_, B = name.split(":")
-            det_digest(n_, int(B))
+        if ":" in name:  # e.g. c3:2048[:bal] -> digest of the B x B DET partition only
+            parts = name.split(":")
+            det_digest(parts[0], int(parts[1]), bal=int(len(parts) > 2 and parts[2] == "bal"))
             continue
         cfg = synth.CONFIGS[name]
         (u, v, r), (tu, tv, tr) = synth.make(cfg)

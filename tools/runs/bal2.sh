@@ -1,0 +1,5 @@
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "wavefront or balance" 2>&1 | tail -2
+run() { timeout 600 python bench.py --config c3 --sched det --legs "" --no-e2e --no-cpu-baseline --fp16-leg none --steps 3 --warmup 2 "$@" > gpurun_out/bal.json 2> gpurun_out/bal.err; python -c "import json,sys;d=json.load(open('gpurun_out/bal.json'));print(sys.argv[1:], round(d['ms_per_step'],2), round(d['value']/1e9,3), d['rmse']['test_per_epoch'][-1])" "$@"; tail -2 gpurun_out/bal.err; }
+run --grid 2048,2048 --det-wave 1 --col-balance
+run --grid 1536,1536 --det-wave 1 --col-balance
+run --grid 2048,2048 --det-wave 1
