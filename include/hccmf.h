@@ -207,6 +207,10 @@ typedef enum {
                                     item are corrected in registers, so a single
                                     warp stays serial; across warps D widens the
                                     read-to-write window (R14).         */
+    HCCMF_OPT_TIMELINE = 15,     /* 1: train_epoch records CUDA events around every SGD
+                                    launch (compute stream) and every Q transfer (comm
+                                    stream) of the epoch; hccmf_timeline reads them.
+                                    Default 0 (no events).                        */
     HCCMF_OPT_STORAGE = 14       /* Q storage from the next epoch on: 0 fp32, 1
                                     binary16, 2 binary16 with stochastic rounding
                                     (the partition option `storage`,
@@ -376,10 +380,20 @@ HCCMF_API hccmf_status hccmf_cost_model(int32_t p, int64_t m, int64_t n, int64_t
  * `warps` warps (0: the Hogwild epoch's automatic count for the whole of Q), one rating
  * ahead, doing per rating only the kernel's q_v traffic into a SCRATCH copy of Q (the
  * model is not touched): mode 0 fp32 vector reductions only (red.v4.f32), 1 binary16
- * load + dependent reduction (red.v2.f16x2), 2 fp32 load + dependent reduction.
+ * load + dependent reduction (red.v2.f16x2), 2 fp32 load + dependent reduction, 3 the
+ * q_v stream alone (loads of the model's Q), 4 the p_u stream alone (per user run one load
+ * of the row and one store of the same values: the model is left unchanged).  Modes 3-4
+ * let ncu report the L2 hit rate of the Q and of the P stream separately.
  * *ms = mean duration of one pass over `reps` timed passes (CUDA events on the handle's
  * stream, after one warm-up pass).  Needs partition; k a multiple of 128. */
 HCCMF_API hccmf_status hccmf_probe_roundtrip(hccmf_t h, int32_t mode, int64_t warps, int32_t reps, double* ms);
+
+/* The last train_epoch's timeline (HCCMF_OPT_TIMELINE = 1): up to `cap` rows of 5 doubles
+ * {kind, stage, column block, start ms, end ms}, times relative to the epoch's first
+ * event, measured with CUDA events on the stream each piece ran on.  kind: 0 SGD launch,
+ * 1 pipelined ring transfer of one column block (comm stream), 2 stage-wise ring
+ * transfer, 3 Q average (all-reduce).  *n = rows available.  Synchronises the streams. */
+HCCMF_API hccmf_status hccmf_timeline(hccmf_t h, double* rows, int64_t cap, int64_t* n);
 
 /* Library version string, e.g. "hccmf 0.1 sm_100a". */
 HCCMF_API const char* hccmf_version(void);

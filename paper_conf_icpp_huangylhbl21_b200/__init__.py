@@ -38,7 +38,7 @@ STATUS = {0: "OK", -1: "EINVAL", -2: "ERANGE", -3: "ENOMEM", -4: "ESTATE", -5: "
 SCHED = {"det": 0, "hogwild": 1}
 SYNC = {"none": 0, "ring": 1, "allreduce": 2}
 DP = {"DP0": 0, "DP1": 1, "DP2": 2}
-OPT = {"hogwild_warps": 1, "task_ratings": 2, "sync_stream": 3, "hogwild_atomic": 5, "conflict_ratio": 6, "heavy_first": 7, "vec": 8, "det_wave": 9, "sync_phases": 10, "wire_fp16": 11, "l2_persist": 12, "prefetch_depth": 13, "storage": 14}
+OPT = {"hogwild_warps": 1, "task_ratings": 2, "sync_stream": 3, "hogwild_atomic": 5, "conflict_ratio": 6, "heavy_first": 7, "vec": 8, "det_wave": 9, "sync_phases": 10, "wire_fp16": 11, "l2_persist": 12, "prefetch_depth": 13, "storage": 14, "timeline": 15}
 
 
 class HccmfError(RuntimeError):
@@ -102,6 +102,7 @@ def lib():
             "hccmf_comm_counts": (st, [P, P, i32, P]),
             "hccmf_load_ratings_slice": (st, [P, P, P, P, i64]),
             "hccmf_probe_roundtrip": (st, [P, i32, i64, i32, ctypes.POINTER(ctypes.c_double)]),
+            "hccmf_timeline": (st, [P, P, i64, P]),
             "hccmf_kernel_launches": (ctypes.c_int64, []),
             "hccmf_schedule": (st, [i32, i32, i32, i64, i32, i32, i32, P, P, P, P, P, P]),
             "hccmf_cost_model": (st, [i32, i64, i64, i64, i32, P, P, ctypes.c_double, i32, i32, i32,
@@ -290,9 +291,18 @@ class Model:
     def probe_roundtrip(self, mode="red_f32", warps=0, reps=3) -> float:
         """Mean ms of one pass of the q_v round-trip ceiling probe (hccmf_probe_roundtrip)."""
         out = ctypes.c_double()
-        m = {"red_f32": 0, "ldred_f16": 1, "ldred_f32": 2}[mode]
+        m = {"red_f32": 0, "ldred_f16": 1, "ldred_f32": 2, "q_stream": 3, "p_stream": 4}[mode]
         self._check(lib().hccmf_probe_roundtrip(self._h, m, int(warps), int(reps), ctypes.byref(out)))
         return out.value
+
+    def timeline(self):
+        """Rows {kind, stage, block, start ms, end ms} of the last epoch (HCCMF_OPT_TIMELINE)."""
+        n = ctypes.c_int64()
+        self._check(lib().hccmf_timeline(self._h, None, 0, ctypes.byref(n)))
+        rows = np.zeros((n.value, 5), np.float64)
+        if n.value:
+            self._check(lib().hccmf_timeline(self._h, rows.ctypes.data, n.value, ctypes.byref(n)))
+        return rows
 
     def comm_counts(self) -> dict:
         """How many times each data-plane call site ran on this handle (hccmf_comm_counts)."""

@@ -239,6 +239,30 @@ void free_partition(hccmf_t h) {
   h->h_task_hi.clear();
 }
 
+// ------------------------------------------------------------ timeline (HCCMF_OPT_TIMELINE)
+void timeline_clear(hccmf_t h) {
+  for (auto& r : h->timeline) {
+    cudaEventDestroy(r.a);
+    cudaEventDestroy(r.b);
+  }
+  h->timeline.clear();
+}
+// open a row: its start event is recorded now on `st`; returns the row index (-1: off)
+int timeline_begin(hccmf_t h, int kind, int stage, int block, cudaStream_t st) {
+  if (!h->opt_timeline) return -1;
+  hccmf_ctx::TimelineRow r{kind, stage, block, nullptr, nullptr};
+  if (cudaEventCreate(&r.a) != cudaSuccess || cudaEventCreate(&r.b) != cudaSuccess) {
+    cudaGetLastError();
+    return -1;
+  }
+  cudaEventRecord(r.a, st);
+  h->timeline.push_back(r);
+  return (int)h->timeline.size() - 1;
+}
+void timeline_end(hccmf_t h, int row, cudaStream_t st) {
+  if (row >= 0) cudaEventRecord(h->timeline[row].b, st);
+}
+
 // ------------------------------------------------------------ SGD plans
 // The a5/a6/a7 schedule as block lists (pure host logic, also exported through
 // hccmf_schedule so multi-process tests can run it without a device):
@@ -461,7 +485,10 @@ hccmf_status ring_exchange(hccmf_t h, int sched, int t) {
   ring_group_cols(h, sched, g_send, &sa, &sb);
   ring_group_cols(h, sched, g_recv, &ra, &rb);
   const int prev = (s - 1 + G) % G, next = (s + 1) % G;
-  return ring_transfer(h, sa, sb, ra, rb, prev, next, h->stream, SITE_RING_STAGE);
+  const int row = timeline_begin(h, 2, t, -1, h->stream);
+  hccmf_status st = ring_transfer(h, sa, sb, ra, rb, prev, next, h->stream, SITE_RING_STAGE);
+  timeline_end(h, row, h->stream);
+  return st;
 }
 
 // Hidden synchronisation (L1143-L1172) with asynchronous computing-transmission
@@ -481,7 +508,10 @@ hccmf_status ring_exchange_block(hccmf_t h, int t, int j, cudaStream_t cs) {
   rows((s + t) % G, &sa, &sb);
   rows((s + t + 1) % G, &ra, &rb);
   const int prev = (s - 1 + G) % G, next = (s + 1) % G;
-  return ring_transfer(h, sa, sb, ra, rb, prev, next, cs, SITE_RING_BLOCK);
+  const int row = timeline_begin(h, 1, t, j, cs);
+  hccmf_status st = ring_transfer(h, sa, sb, ra, rb, prev, next, cs, SITE_RING_BLOCK);
+  timeline_end(h, row, cs);
+  return st;
 }
 
 // after ring epochs rank s holds only group s of Q: broadcast every group from its owner
@@ -677,6 +707,10 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
     case HCCMF_OPT_HEAVY_FIRST:
       h->opt_heavy = value;
       return HCCMF_OK;
+    case HCCMF_OPT_TIMELINE:
+      h->opt_timeline = value != 0;
+      if (!h->opt_timeline) timeline_clear(h);
+      return HCCMF_OK;
     case HCCMF_OPT_CONFLICT_RATIO:
       if (value < 0) return fail(h, HCCMF_EINVAL, "conflict ratio must be >= 0");
       h->opt_conflict = value;
@@ -697,6 +731,7 @@ void hccmf_destroy(hccmf_t h) {
   dfree(h, h->d_partials, 2 * RMSE_BLOCKS);
   dfree(h, h->d_scalar, 2);
   if (h->d_wire) cudaFreeAsync(h->d_wire, h->stream);
+  timeline_clear(h);
   for (auto e : h->ev_done) cudaEventDestroy(e);
   for (auto e : h->ev_recv) cudaEventDestroy(e);
   if (h->comm_stream) {
@@ -1174,6 +1209,7 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
   hccmf_status st = build_plan(h, sched, sync, &pl);
   if (st != HCCMF_OK) return st;
   if (sched == HCCMF_SCHED_DET) h->det_path = 0;
+  timeline_clear(h);
   const int eff_sync = (G == 1) ? HCCMF_SYNC_NONE : sync;
   const bool dist = h->world > 1;
   const int64_t nk = h->n * h->k;
@@ -1190,6 +1226,13 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     return HCCMF_OK;
   };
   auto average = [&]() -> hccmf_status {  // the server's sync (L549-L557): Q = mean of the shards' Q
+    const int trow = timeline_begin(h, 3, -1, -1, s);
+    struct End {
+      hccmf_t h;
+      int row;
+      cudaStream_t s;
+      ~End() { timeline_end(h, row, s); }
+    } end_{h, trow, s};
     if (dist && h->opt_wire16) {  // Strategy 2: the copies travel and come back as binary16
       hccmf_status w = allreduce_q16(h, s);
       if (w != HCCMF_OK) return w;
@@ -1345,7 +1388,9 @@ hccmf_status hccmf_train_epoch(hccmf_t h, hccmf_sched sched, hccmf_sync sync) {
     // DET: one rating group per block of the stratum; HOGWILD: persistent grid
     // Hogwild races only on the Q rows of the launch's column blocks (R14, R28)
     const int64_t warps = (sched == HCCMF_SCHED_DET) ? (ln.nt * L + 31) / 32 : auto_warps(h, ln.items);
+    const int trow = timeline_begin(h, 0, ln.stage, pipelined ? jblk : (int)li, s);
     CU(h, launch_sgd(a, warps, s));
+    timeline_end(h, trow, s);
     if (pipelined) {
       st = qh_flush();  // the block travels as fp32 (or binary16 wire) right after its launch
       if (st != HCCMF_OK) return st;
@@ -1573,14 +1618,38 @@ hccmf_status hccmf_cost_model(int32_t p, int64_t m, int64_t n, int64_t nnz, int3
   return HCCMF_OK;
 }
 
+hccmf_status hccmf_timeline(hccmf_t h, double* rows, int64_t cap, int64_t* n) {
+  ENTER(h);
+  if (!n) return fail(h, HCCMF_EINVAL, "n is NULL");
+  *n = (int64_t)h->timeline.size();
+  if (h->timeline.empty() || !rows) return HCCMF_OK;
+  CU(h, cudaStreamSynchronize(h->stream));
+  if (h->comm_stream) CU(h, cudaStreamSynchronize(h->comm_stream));
+  const cudaEvent_t t0 = h->timeline[0].a;
+  for (int64_t i = 0; i < *n && i < cap; ++i) {
+    const auto& r = h->timeline[i];
+    float a = 0.f, b = 0.f;
+    CU(h, cudaEventElapsedTime(&a, t0, r.a));
+    CU(h, cudaEventElapsedTime(&b, t0, r.b));
+    double* o = rows + 5 * i;
+    o[0] = r.kind;
+    o[1] = r.stage;
+    o[2] = r.block;
+    o[3] = a;
+    o[4] = b;
+  }
+  return HCCMF_OK;
+}
+
 hccmf_status hccmf_probe_roundtrip(hccmf_t h, int32_t mode, int64_t warps, int32_t reps, double* ms) {
   ENTER(h);
-  if (!ms || mode < 0 || mode > 2 || warps < 0 || reps < 1) return fail(h, HCCMF_EINVAL, "bad probe arguments");
+  if (!ms || mode < 0 || mode > 4 || warps < 0 || reps < 1) return fail(h, HCCMF_EINVAL, "bad probe arguments");
   if (h->state < 2) return fail(h, HCCMF_ESTATE, "probe needs partition");
   if (h->k % 128 != 0) return fail(h, HCCMF_EINVAL, "probe needs k a multiple of 128");
   const int64_t w = warps ? warps : auto_warps(h, h->n);
   float t = 0.f;
-  CU(h, k_probe_roundtrip(mode, h->d_v, h->d_r, h->local_nnz, h->k, h->n, w, reps, &t, h->stream));
+  CU(h, k_probe_roundtrip(mode, h->d_u, h->d_v, h->d_r, h->local_nnz, h->k, h->n, h->d_P, h->row0, h->d_Q, w, reps, &t,
+                          h->stream));
   *ms = t;
   return finish(h);
 }

@@ -164,8 +164,9 @@ cudaError_t k_average_half(const float* reps, int32_t G, int64_t count, float* o
 cudaError_t k_mean_gathered_half(const void* g, int32_t W, int64_t stride, int64_t count, void* out, cudaStream_t st);
 constexpr int RMSE_BLOCKS = 592;
 // q_v round-trip ceiling probe (probe.cu): mean ms of one pass over the records
-cudaError_t k_probe_roundtrip(int mode, const int32_t* rv, const float* rr, int64_t nrec, int32_t k, int64_t n,
-                              int64_t warps, int reps, float* ms, cudaStream_t st);
+cudaError_t k_probe_roundtrip(int mode, const int32_t* ru, const int32_t* rv, const float* rr, int64_t nrec, int32_t k,
+                              int64_t n, float* P, int64_t row0, const float* Q, int64_t warps, int reps, float* ms,
+                              cudaStream_t st);
 
 }  // namespace hccmf
 
@@ -238,6 +239,13 @@ struct hccmf_ctx {
 
   bool transposed = false;  // column grid: internal rows are the caller's columns
   int det_path = -1;        // kernel of the last DET epoch (hccmf_info.det_path)
+  // HCCMF_OPT_TIMELINE: events of the last epoch {kind, stage, block, start, end}
+  struct TimelineRow {
+    int kind, stage, block;
+    cudaEvent_t a, b;
+  };
+  bool opt_timeline = false;
+  std::vector<TimelineRow> timeline;
   int q_ring_sched = -1;  // >= 0: distributed ring left only this rank's Q group valid
   std::vector<hccmf::Plan> plans;
 };

@@ -4,8 +4,12 @@
 //   mode 0: fp32 vector reductions only (red.v4.f32, 512 B at k = 128) -- the L2 atomic
 //           units that bind the fp32 kernel;
 //   mode 1: binary16 load + dependent reduction (ld 8 B + red.v2.f16x2 per lane);
-//   mode 2: fp32 load + dependent reduction.
-// The reductions go to a scratch copy of Q, never to the model.  bench.py divides the
+//   mode 2: fp32 load + dependent reduction;
+//   mode 3: the q_v stream alone, loads only (one row per rating);
+//   mode 4: the p_u stream alone: per user run one load of the row and one store of the
+//           same values back (the epoch's P traffic; the model is left unchanged).
+// Modes 3 and 4 exist for ncu (the L2 hit rate of the Q and of the P stream separately,
+// profiles/r02_ncu_l2_split.md).  The reductions go to a scratch copy of Q, never to the model.  bench.py divides the
 // SGD kernel's rate by this ceiling (roofline.binding_frac).
 #include <cuda_fp16.h>
 
@@ -94,6 +98,49 @@ __global__ void __launch_bounds__(256) roundtrip_kernel(const int32_t* __restric
   if (acc == 1.2345f) sink[0] = acc;
 }
 
+// modes 3 / 4: one stream of the epoch at a time (same record order and warp split)
+template <int MODE, int SLOTS>
+__global__ void __launch_bounds__(256) stream_kernel(const int32_t* __restrict__ ru, const int32_t* __restrict__ rv,
+                                                     int64_t nrec, const char* Q, char* P, int64_t row0, int rowb,
+                                                     int64_t per_warp, float* sink) {
+  const int lane = threadIdx.x & 31;
+  const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t lo = w * per_warp;
+  const int64_t hi = lo + per_warp < nrec ? lo + per_warp : nrec;
+  float acc = 0.f;
+  int cu = -1;
+  float4 pr[SLOTS];
+  for (int64_t j = lo; j < hi; ++j) {
+    if (MODE == 3) {
+      const int v = __ldcs(rv + j);
+#pragma unroll
+      for (int s = 0; s < SLOTS; ++s) {
+        const float4 x = __ldcg(reinterpret_cast<const float4*>(Q + (int64_t)v * rowb + (s * 32 + lane) * 16));
+        acc += x.x + x.y + x.z + x.w;
+      }
+    } else {
+      const int u = __ldcs(ru + j);
+      if (u != cu) {
+        if (cu >= 0) {
+#pragma unroll
+          for (int s = 0; s < SLOTS; ++s)
+            __stcg(reinterpret_cast<float4*>(P + (int64_t)(cu - row0) * rowb + (s * 32 + lane) * 16), pr[s]);
+        }
+#pragma unroll
+        for (int s = 0; s < SLOTS; ++s)
+          pr[s] = __ldcg(reinterpret_cast<const float4*>(P + (int64_t)(u - row0) * rowb + (s * 32 + lane) * 16));
+        cu = u;
+      }
+    }
+  }
+  if (MODE == 4 && cu >= 0) {
+#pragma unroll
+    for (int s = 0; s < SLOTS; ++s)
+      __stcg(reinterpret_cast<float4*>(P + (int64_t)(cu - row0) * rowb + (s * 32 + lane) * 16), pr[s]);
+  }
+  if (acc == 1.2345f) sink[0] = acc;
+}
+
 template <int MODE, int SLOTS>
 cudaError_t launch_probe(const int32_t* rv, const float* rr, int64_t nrec, char* Q, int rowb, int64_t warps,
                          float* sink, cudaStream_t st) {
@@ -105,8 +152,9 @@ cudaError_t launch_probe(const int32_t* rv, const float* rr, int64_t nrec, char*
 
 }  // namespace
 
-cudaError_t k_probe_roundtrip(int mode, const int32_t* rv, const float* rr, int64_t nrec, int32_t k, int64_t n,
-                              int64_t warps, int reps, float* ms, cudaStream_t st) {
+cudaError_t k_probe_roundtrip(int mode, const int32_t* ru, const int32_t* rv, const float* rr, int64_t nrec, int32_t k,
+                              int64_t n, float* P, int64_t row0, const float* Qm, int64_t warps, int reps, float* ms,
+                              cudaStream_t st) {
   *ms = 0.f;
   if (nrec <= 0 || warps <= 0) return cudaSuccess;
   // slots of 32 lanes: 16 B (fp32) or 8 B (binary16) each
@@ -123,11 +171,21 @@ cudaError_t k_probe_roundtrip(int mode, const int32_t* rv, const float* rr, int6
   cudaEvent_t a, b;
   cudaEventCreate(&a);
   cudaEventCreate(&b);
+  const int64_t pw = (nrec + warps - 1) / warps;
+  const unsigned blocks = (unsigned)((warps * 32 + 255) / 256);
   auto once = [&]() -> cudaError_t {
 #define PR(M, S) \
   if (mode == M && slots == S) return launch_probe<M, S>(rv, rr, nrec, Q, rowb, warps, sink, st);
     PR(0, 1) PR(0, 2) PR(0, 4) PR(1, 1) PR(1, 2) PR(1, 4) PR(2, 1) PR(2, 2) PR(2, 4)
 #undef PR
+#define PS(M, S)                                                                                             \
+  if (mode == M && slots == S) {                                                                             \
+    (note_launch(), stream_kernel<M, S><<<blocks, 256, 0, st>>>(ru, rv, nrec, reinterpret_cast<const char*>(Qm), \
+                                                              reinterpret_cast<char*>(P), row0, k * 4, pw, sink)); \
+    return cudaGetLastError();                                                                               \
+  }
+    PS(3, 1) PS(3, 2) PS(3, 4) PS(4, 1) PS(4, 2) PS(4, 4)
+#undef PS
     return cudaErrorInvalidValue;
   };
   e = once();  // warm-up

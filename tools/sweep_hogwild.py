@@ -2,7 +2,8 @@
 """Measure Hogwild epoch time and test RMSE vs concurrency (warps) and atomic q updates.
 
 GPU only (does not touch oracle/); compare the printed RMSEs with the oracle's serial
-RMSE printed by tests/test_gpu_band_full.py.  Usage:
+curve stored in tests/golden/oracle_curve_<cfg>.json (tools/oracle_curves.py; the band
+tests are tests/test_gpu_full_size.py and tests/test_gpu_parity.py).  Usage:
     python tools/sweep_hogwild.py --config c3 --epochs 5 --warps 148,592,2368,4736 --atomic 0,1
 """
 import argparse
