@@ -29,5 +29,8 @@ def test_sanitizer_clean(tool):
     p = subprocess.run(cmd, capture_output=True, text=True, timeout=1500, cwd=ROOT)
     out = p.stdout + p.stderr
     assert p.returncode == 0, out[-4000:]
-    assert "ERROR SUMMARY: 0 errors" in out, out[-4000:]
+    # memcheck / synccheck end with "ERROR SUMMARY: 0 errors", racecheck with
+    # "RACECHECK SUMMARY: 0 hazards displayed (0 errors, 0 warnings)"
+    assert ("ERROR SUMMARY: 0 errors" in out or "SUMMARY: 0 hazards displayed (0 errors, 0 warnings)" in out), \
+        out[-4000:]
     assert "jobs ok" in out
