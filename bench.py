@@ -421,12 +421,19 @@ def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, samp
     res["e2e"] = None
     if not want_e2e:
         return res
+    # pinned host buffers: this rank's COO slice (twice while it is copied) + P and Q; every rank of
+    # the node needs its own, and the decision must be the same on every rank (the job is collective)
+    need = (12 * (nnz_slice + nt) * 2 + 4 * (cfg.m + cfg.n) * cfg.k) * int(os.environ.get("LOCAL_WORLD_SIZE", 1))
+    ok = host_mem_available() >= need
+    if world > 1:
+        t = torch.tensor([1.0 if ok else 0.0], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MIN)
+        ok = t.item() > 0.5
+    if not ok:
+        res["e2e"] = {"value": None, "unit": UNIT, "skipped": f"host memory {host_mem_available() / 1e9:.0f} GB "
+                                                             f"< {need / 1e9:.0f} GB for the node's pinned COO + P, Q"}
+        return res
     if on_device:
-        need = 12 * (nnz_slice + nt) * 2 + 4 * (cfg.m + cfg.n) * cfg.k
-        if host_mem_available() < need:
-            res["e2e"] = {"value": None, "unit": UNIT, "skipped": f"host memory {host_mem_available() / 1e9:.0f} GB "
-                                                                 f"< {need / 1e9:.0f} GB for pinned COO + P, Q"}
-            return res
         (du, dv, dr), (dtu2, dtv2, dtr2) = synth.make_device(cfg, device=f"cuda:{local}", part=(rank, world))
         u, v, r, tu, tv, tr = (x.cpu().numpy() for x in (du, dv, dr, dtu2, dtv2, dtr2))
         del du, dv, dr, dtu2, dtv2, dtr2

@@ -162,8 +162,9 @@ typedef enum {
                                     atomic model, no lost updates); 0: plain stores
                                     (racing writers may overwrite: the paper's
                                     "coverage", L1680-L1686)                      */
-    HCCMF_OPT_CONFLICT_RATIO = 6,/* auto Hogwild concurrency: at most n / value
-                                    rating groups in flight (default 3; 0 = no cap) */
+    HCCMF_OPT_CONFLICT_RATIO = 6,/* > 0: auto Hogwild concurrency is at most (items a
+                                    launch can touch) / value rating groups (round-1
+                                    rule); 0 (default): the staleness budget below  */
     HCCMF_OPT_HEAVY_FIRST = 7,   /* Hogwild task order inside a block: tasks with more
                                     than `value` ratings run first, longest first
                                     (no late heavy user stretches the epoch); the
@@ -207,6 +208,12 @@ typedef enum {
                                     item are corrected in registers, so a single
                                     warp stays serial; across warps D widens the
                                     read-to-write window (R14).         */
+    HCCMF_OPT_STALENESS = 16,    /* auto Hogwild concurrency (R32): at most
+                                    items * kappa / (gamma (r_rms + lambda)) rating
+                                    groups in flight per launch, items = the Q rows the
+                                    launch can touch, r_rms = sqrt(mean r^2) of the
+                                    shard, kappa = value * 1e-4 (default 80 -> 0.008);
+                                    0 = no cap (resident warps only)              */
     HCCMF_OPT_TIMELINE = 15,     /* 1: train_epoch records CUDA events around every SGD
                                     launch (compute stream) and every Q transfer (comm
                                     stream) of the epoch; hccmf_timeline reads them.

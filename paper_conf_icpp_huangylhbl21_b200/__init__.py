@@ -38,7 +38,7 @@ STATUS = {0: "OK", -1: "EINVAL", -2: "ERANGE", -3: "ENOMEM", -4: "ESTATE", -5: "
 SCHED = {"det": 0, "hogwild": 1}
 SYNC = {"none": 0, "ring": 1, "allreduce": 2}
 DP = {"DP0": 0, "DP1": 1, "DP2": 2}
-OPT = {"hogwild_warps": 1, "task_ratings": 2, "sync_stream": 3, "hogwild_atomic": 5, "conflict_ratio": 6, "heavy_first": 7, "vec": 8, "det_wave": 9, "sync_phases": 10, "wire_fp16": 11, "l2_persist": 12, "prefetch_depth": 13, "storage": 14, "timeline": 15}
+OPT = {"hogwild_warps": 1, "task_ratings": 2, "sync_stream": 3, "hogwild_atomic": 5, "conflict_ratio": 6, "heavy_first": 7, "vec": 8, "det_wave": 9, "sync_phases": 10, "wire_fp16": 11, "l2_persist": 12, "prefetch_depth": 13, "storage": 14, "timeline": 15, "staleness": 16}
 
 
 class HccmfError(RuntimeError):

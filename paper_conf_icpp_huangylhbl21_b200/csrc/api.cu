@@ -408,19 +408,34 @@ hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
   return HCCMF_OK;
 }
 
-// Hogwild concurrency (R14): the number of rating groups in flight sets
-// the staleness of q_v reads, so it is capped at n / opt_conflict groups, and at 32
-// resident warps per SM.
+// Hogwild concurrency (R14, R28, R32): the rating groups in flight set how stale a
+// q_v read can be.  A read that misses tau concurrent updates of its item is a delayed gradient
+// step; on the per-rating quadratic in q_v (curvature ~ |p_u|^2 + lambda, and |p_u|^2 grows to
+// the rating scale) the delay is harmless while tau * gamma * (r_rms + lambda) stays small.  With
+// the items of a launch hit uniformly, tau ~ groups / items, so the cap is
+//   groups <= items * kappa / (gamma (r_rms + lambda)),   kappa = opt_staleness * 1e-4 (0.008),
+// calibrated on the measured stability edge (C4, ratings 0..100, lambda 1: stable at
+// tau gamma (r_rms + lambda) = 0.0077 and 0.0097, divergent at 0.0155; C3 runs at 0.0048).
+// opt_conflict > 0 replaces it by the fixed items / opt_conflict of round 1.  Never more
+// than 32 resident warps per SM.
 int64_t auto_warps(hccmf_t h, int64_t items_in_play) {
   if (h->opt_warps > 0) return h->opt_warps;
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
-  int64_t w = (int64_t)sms * 32;
+#ifndef HCCMF_WARPS_PER_SM
+#define HCCMF_WARPS_PER_SM 32  // resident warps of the warp-per-rating kernel (64 registers: 4 CTAs of 8)
+#endif
+  int64_t w = (int64_t)sms * HCCMF_WARPS_PER_SM;
+  const int64_t groups_per_warp = hogwild_groups_per_warp(h->k, (int)h->opt_vec);
+  int64_t groups = -1;
   if (h->opt_conflict > 0) {
-    const int64_t groups_per_warp = hogwild_groups_per_warp(h->k, (int)h->opt_vec);
-    const int64_t cap = std::max<int64_t>(1, (items_in_play / h->opt_conflict) / groups_per_warp);
-    w = std::min(w, cap);
+    groups = items_in_play / h->opt_conflict;
+  } else if (h->opt_staleness > 0) {
+    const double denom = (double)h->gamma * (h->r_rms + (double)h->lambda);
+    const double g = denom > 0.0 ? (double)items_in_play * (double)h->opt_staleness * 1e-4 / denom : 1e18;
+    groups = (int64_t)std::min(g, 1e15);
   }
+  if (groups >= 0) w = std::min(w, std::max<int64_t>(1, groups / groups_per_warp));
   return w;
 }
 
@@ -710,6 +725,10 @@ hccmf_status hccmf_set_option(hccmf_t h, int32_t option, int64_t value) {
     case HCCMF_OPT_TIMELINE:
       h->opt_timeline = value != 0;
       if (!h->opt_timeline) timeline_clear(h);
+      return HCCMF_OK;
+    case HCCMF_OPT_STALENESS:
+      if (value < 0) return fail(h, HCCMF_EINVAL, "staleness budget must be >= 0");
+      h->opt_staleness = value;
       return HCCMF_OK;
     case HCCMF_OPT_CONFLICT_RATIO:
       if (value < 0) return fail(h, HCCMF_EINVAL, "conflict ratio must be >= 0");
@@ -1066,6 +1085,16 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   h->rows = (int64_t)h->bounds[h->shard_hi] - h->row0;
 
   timer.mark("local shard");
+  {  // rating scale of the shard (R32: the Hogwild staleness budget)
+    double* dss = nullptr;
+    CU(h, cudaMallocAsync((void**)&dss, sizeof(double), st));
+    CU(h, k_sum_sq(h->d_r, h->local_nnz, dss, st));
+    double ss = 0.0;
+    CU(h, cudaMemcpyAsync(&ss, dss, sizeof(double), cudaMemcpyDeviceToHost, st));
+    CU(h, cudaStreamSynchronize(st));
+    cudaFreeAsync(dss, st);
+    h->r_rms = h->local_nnz > 0 ? std::sqrt(ss / (double)h->local_nnz) : 0.0;
+  }
   // ---- Hogwild tasks: user-aligned runs of ~opt_task ratings inside each block
   std::vector<int64_t> loc_off(h->nblk_local + 1);
   for (int64_t j = 0; j <= h->nblk_local; ++j) loc_off[j] = h->block_off[h->blk0 + j] - h->rec0;

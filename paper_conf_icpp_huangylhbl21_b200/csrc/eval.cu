@@ -238,6 +238,23 @@ cudaError_t k_mean_gathered_half(const void* g, int32_t W, int64_t stride, int64
   return cudaGetLastError();
 }
 
+namespace {
+__global__ void sum_sq_kernel(const float* __restrict__ r, int64_t n, double* out) {
+  double s = 0.0;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    s += (double)r[i] * (double)r[i];
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if ((threadIdx.x & 31) == 0) atomicAdd(out, s);
+}
+}  // namespace
+
+cudaError_t k_sum_sq(const float* r, int64_t n, double* out, cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(out, 0, sizeof(double), st);
+  if (e != cudaSuccess || n <= 0) return e;
+  (note_launch(), sum_sq_kernel<<<grid_for(n), kT, 0, st>>>(r, n, out));
+  return cudaGetLastError();
+}
+
 cudaError_t k_init_factors(uint64_t seed, uint64_t tag, int64_t rows_total, int32_t k, const int32_t* perm,
                            int64_t row0, int64_t rows, float* X, cudaStream_t st) {
   if (rows_total == 0) return cudaSuccess;

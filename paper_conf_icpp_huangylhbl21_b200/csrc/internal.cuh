@@ -156,6 +156,8 @@ cudaError_t k_rmse(const int32_t* tu, const int32_t* tv, const float* tr, int64_
                    const int32_t* perm_col, const float* P, int64_t row0, int64_t rows, const float* Q, int32_t k,
                    double* partials /*2*RMSE_BLOCKS*/, double* out2 /*sum, count*/, cudaStream_t st);
 cudaError_t k_average(const float* reps, int32_t G, int64_t count, float* out, cudaStream_t st);
+// sum of r^2 over n ratings (fp64, one value on the device)
+cudaError_t k_sum_sq(const float* r, int64_t n, double* out, cudaStream_t st);
 cudaError_t k_round_half(float* x, int64_t count, cudaStream_t st);
 cudaError_t k_pack_half(const float* x, void* y /* __half */, int64_t count, cudaStream_t st);
 cudaError_t k_unpack_half(const void* y /* __half */, float* x, int64_t count, cudaStream_t st);
@@ -188,7 +190,9 @@ struct hccmf_ctx {
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 3, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1, opt_wire16 = 0, opt_l2persist = 0, opt_depth = 0;
+  int64_t opt_staleness = 80;  // Hogwild staleness budget, units of 1e-4 (R32); 0: no cap
+  double r_rms = 0.0;          // sqrt(mean r^2) of the local records (R32)
+  int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 0, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1, opt_wire16 = 0, opt_l2persist = 0, opt_depth = 0;
   bool sync_stream = true;
   size_t device_bytes = 0;
 

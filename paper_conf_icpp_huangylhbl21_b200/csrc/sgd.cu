@@ -43,6 +43,9 @@ constexpr int kThreads = 256;
 #ifndef HCCMF_WARP_UNROLL  // 2-rating steps per record-ring loop iteration (Hogwild, k = 128 j)
 #define HCCMF_WARP_UNROLL 8
 #endif
+#ifndef HCCMF_WARP_MINB1  // CTAs of 8 warps per SM the k = 128 warp kernel is compiled for (registers)
+#define HCCMF_WARP_MINB1 4
+#endif
 #ifndef HCCMF_NARROW_UNROLL  // R-rating rounds per loop iteration (Hogwild, k = 32 / 64)
 #define HCCMF_NARROW_UNROLL 1
 #endif
@@ -1073,7 +1076,7 @@ __global__ void __launch_bounds__(kThreads) sgd_narrow_kernel(SgdArgs a) {
 #define HCCMF_WARP_MINB 1
 #endif
 template <int VEC, bool ATOMIC, int D, int QM>  // QM: 0 fp32 Q, 1 binary16 RN, 2 binary16 SR
-__global__ void __launch_bounds__(kThreads, (VEC == 1 ? 4 : HCCMF_WARP_MINB)) sgd_warp_kernel(SgdArgs a) {
+__global__ void __launch_bounds__(kThreads, (VEC == 1 ? HCCMF_WARP_MINB1 : HCCMF_WARP_MINB)) sgd_warp_kernel(SgdArgs a) {
   constexpr unsigned FM = 0xffffffffu;
   WarpSgd<VEC, ATOMIC> w(a);
   __shared__ int4 sring[kThreads / 32][64];

@@ -268,6 +268,33 @@ def test_hogwild_single_group_is_the_serial_oracle(pkg, orc, atomic, k, task, de
     assert max(np.abs(P - Po).max(), np.abs(Q - Qo).max()) <= 1e-4
 
 
+@pytest.mark.parametrize("Bc,scale", [(2, 1.0), (3, 1.0), (8, 1.0), (8, 20.0), (5, 20.0)])
+def test_hogwild_single_group_column_phases(pkg, orc, Bc, scale):
+    # grid (1, Bc): one launch per column-block phase (C4's configuration); one warp walks every
+    # phase's tasks in record order, so the epoch IS the oracle's serial run of the sorted
+    # records (blocks (0, 0), (0, 1), ..).  scale 20: ratings on C4's 0..100 range.
+    cfg = synth.CONFIGS["c1"]
+    (u, v, r), _ = synth.make(cfg)
+    r = (r * scale).astype(np.float32)
+    prob = orc.Problem(cfg.m, cfg.n, 128, 0.005, 1.0, u, v, r, G=1, Br=1, Bc=Bc, seed=3)
+    prob.init(4)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    mdl = pkg.Model(cfg.m, cfg.n, 128, 0.005, 1.0)
+    mdl.set_option("heavy_first", -1)
+    mdl.load(u, v, r)
+    mdl.partition(1, (1, Bc), seed=3)
+    mdl.set_option("hogwild_warps", 1)
+    mdl.set_factors(P0, Q0)
+    for _ in range(2):
+        mdl.train_epoch("hogwild", "none")
+        prob.epoch("serial", "none")
+    P, Q = mdl.factors()
+    Po, Qo = prob.factors()
+    assert np.isfinite(P).all() and np.isfinite(Q).all()
+    assert max(np.abs(P - Po).max(), np.abs(Q - Qo).max()) <= 1e-4 * max(1.0, scale)
+
+
 def _band(pkg, orc, cfg_name, frac, k, epochs, sync="none", G=1, Br=1, Bc=1, repeats=2, gamma=None):
     """GPU and oracle test-RMSE curves (same data, same schedule, init seed 1), checked with the
     shared bar of tests/bands.py (R15, R29) for every repeat."""
@@ -301,6 +328,14 @@ def test_hogwild_band_c1(pkg, orc):
 def test_hogwild_band_c2_full(pkg, orc):
     # BASELINE.json config 2 at full size; band read at E = 20 epochs (R15)
     _band(pkg, orc, "c2", 1.0, 32, 20, repeats=3)  # Hogwild bands run 3 times
+
+
+@pytest.mark.parametrize("Bc", [1, 4])
+def test_hogwild_band_c4_scaled(pkg, orc, Bc):
+    # C4's rating scale (0..100, lambda 1) at 5 % size (12.6 M ratings, 31 K items): at the full
+    # resident concurrency (4,736 warps, 6.6 items per warp) this diverged to NaN in epoch 1;
+    # the staleness budget (R32) sizes the concurrency from gamma (r_rms + lambda) and holds the band
+    _band(pkg, orc, "c4", 0.05, 128, 5, Bc=Bc, repeats=2)
 
 
 @pytest.mark.parametrize("sync,G,Bc", [("ring", 4, 4), ("ring", 2, 8), ("allreduce", 2, 1)])
