@@ -219,3 +219,22 @@ def test_balanced_perm_partition_is_a_valid_block_sort(orc):
 def synth_tiny():
     import synth
     return synth.tiny(40, 30, 500, seed=11)
+
+
+def test_rotated_row_order_hand_computed(orc):
+    # R21 with a non-zero seed, by hand: one user (m = 1, so u' = 0), items 0..4 rated 1..5.
+    # perm_col(seed 11): H(11, 2, v, 0) = aa53.., 0b7b.., 9a38.., abbb.., 8fbc.. (v = 0..4) -> ranks
+    # v' = [3, 0, 2, 4, 1]; H(11, 5, 0, 0) = 0x21917a0b7eba4497: mod 5 = 2, mod 3 = 2, mod 2 = 1.
+    # One block (w = 5): o = (v' + 2) mod 5 -> the row runs v' = 3, 4, 0, 1, 2 (items 0, 3, 1, 4, 2).
+    # Two column blocks: [0, 3) with rotation 2 -> o = (v' + 2) mod 3 -> v' 1, 2, 0; [3, 5) with rotation 1
+    # -> o = (v' - 3 + 1) mod 2 -> v' 4, 3.
+    u = np.zeros(5, np.int32)
+    v = np.arange(5, dtype=np.int32)
+    r = np.arange(1, 6, dtype=np.float32)
+    p1 = orc.Problem(1, 5, 4, 0.01, 0.01, u, v, r, G=1, Br=1, Bc=1, seed=11)
+    assert list(p1.perm_col) == [3, 0, 2, 4, 1]
+    assert list(p1.rv) == [3, 4, 0, 1, 2] and list(p1.rr) == [1.0, 4.0, 2.0, 5.0, 3.0]
+    p2 = orc.Problem(1, 5, 4, 0.01, 0.01, u, v, r, G=1, Br=1, Bc=2, seed=11)
+    assert list(p2.rv) == [1, 2, 0, 4, 3] and list(p2.off) == [0, 3, 5]
+    p0 = orc.Problem(1, 5, 4, 0.01, 0.01, u, v, r, G=1, Br=1, Bc=1, seed=0)  # seed 0: plain order
+    assert list(p0.rv) == [0, 1, 2, 3, 4]
