@@ -905,9 +905,12 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
 
   timer.mark("a2 shuffle");
   // ---- a3 row histogram, prefix, boundaries
+  // (one shard: the bounds are [0, m] whatever the histogram -- skip it, C5: 3.1 B atomics)
   unsigned long long* dS = nullptr;
-  CU(h, cudaMallocAsync((void**)&dS, sizeof(unsigned long long) * (m + 1), st));
-  CU(h, k_row_prefix(h->d_in_u, nnz, h->d_perm_row, m, dS, st));
+  if (G > 1) {
+    CU(h, cudaMallocAsync((void**)&dS, sizeof(unsigned long long) * (m + 1), st));
+    CU(h, k_row_prefix(h->d_in_u, nnz, h->d_perm_row, m, dS, st));
+  }
   if (h->sliced) {  // the global prefix is the sum of the ranks' prefixes
     h->comm_counts[SITE_INGEST_HIST] += 1;
     CM(h, h->comm->allreduce(dS, dS, (size_t)m + 1, DType::u64, ROp::sum, st));
@@ -937,7 +940,7 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
     cudaFreeAsync(dR, st);
     for (int s = 1; s < G; ++s) h->bounds[s] = (int32_t)std::max<int64_t>(h->bounds[s - 1], rstar[s - 1]);
   }
-  cudaFreeAsync(dS, st);
+  if (dS) cudaFreeAsync(dS, st);
   int32_t* dB = nullptr;
   CU(h, cudaMallocAsync((void**)&dB, sizeof(int32_t) * (G + 1), st));
   CU(h, cudaMemcpyAsync(dB, h->bounds.data(), sizeof(int32_t) * (G + 1), cudaMemcpyHostToDevice, st));

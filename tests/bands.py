@@ -20,18 +20,21 @@ import os
 import numpy as np
 
 
-def check(gpu, ora, tag, final_epoch=None):
+def check(gpu, ora, tag, final_epoch=None, scale=1.0):
+    """scale: the band is 0.005 per 4 rating units (the 1..5-star range of C2/C3, SURVEY 8(c3));
+    C4's 0..100 range gives scale 25 (band 0.125), R29."""
     gpu, ora = np.asarray(gpu, float), np.asarray(ora, float)
+    band = 0.005 * scale
     E = len(ora) - 1 if final_epoch is None else final_epoch
     assert len(gpu) >= E + 1, (tag, len(gpu), E)
     gap = gpu[:E + 1] - ora[:E + 1]
     allow = np.full(E + 1, np.inf)
     for e in range(2, E + 1):
-        allow[e] = max(0.005, 0.5 * (ora[e - 1] - ora[e]))
+        allow[e] = max(band, 0.5 * (ora[e - 1] - ora[e]))
     rec = {"tag": tag, "epochs": E, "gap": [round(float(x), 5) for x in gap],
            "allow": [None if not np.isfinite(a) else round(float(a), 5) for a in allow],
            "oracle": [round(float(x), 5) for x in ora[:E + 1]], "gpu": [round(float(x), 5) for x in gpu[:E + 1]],
-           "final_ok": bool(abs(gap[E]) <= 0.005), "one_sided_ok": bool(np.all(gap[2:] <= allow[2:]))}
+           "band": band, "final_ok": bool(abs(gap[E]) <= band), "one_sided_ok": bool(np.all(gap[2:] <= allow[2:]))}
     path = os.environ.get("HCCMF_BAND_REPORT")
     if path:
         with open(path, "a") as f:
