@@ -4,7 +4,7 @@
  * Framework for SGD-based Matrix Factorization", ICPP '21).
  *
  * Citations: L<n> = line n of the paper text.
- * lists every reading taken where the paper is silent or garbled (R1..R30).
+ * lists every reading taken where the paper is silent or garbled (R1..R33).
  *
  * What the library computes:
  *   a0 factor init, a1 ingest+validate COO, a2 seeded ID shuffle, a3 row-grid

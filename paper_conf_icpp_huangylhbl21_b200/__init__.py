@@ -291,7 +291,8 @@ class Model:
     def probe_roundtrip(self, mode="red_f32", warps=0, reps=3) -> float:
         """Mean ms of one pass of the q_v round-trip ceiling probe (hccmf_probe_roundtrip)."""
         out = ctypes.c_double()
-        m = {"red_f32": 0, "ldred_f16": 1, "ldred_f32": 2, "q_stream": 3, "p_stream": 4}[mode]
+        m = {"red_f32": 0, "ldred_f16": 1, "ldred_f32": 2, "q_stream": 3, "p_stream": 4, "bulkred_f32": 5, "bulkldred_f32": 6,
+             "ldbulkred_f32": 7, "bulkldred8_f32": 8, "bulkldred2_f32": 9}[mode]
         self._check(lib().hccmf_probe_roundtrip(self._h, m, int(warps), int(reps), ctypes.byref(out)))
         return out.value
 

@@ -1675,7 +1675,7 @@ hccmf_status hccmf_timeline(hccmf_t h, double* rows, int64_t cap, int64_t* n) {
 
 hccmf_status hccmf_probe_roundtrip(hccmf_t h, int32_t mode, int64_t warps, int32_t reps, double* ms) {
   ENTER(h);
-  if (!ms || mode < 0 || mode > 4 || warps < 0 || reps < 1) return fail(h, HCCMF_EINVAL, "bad probe arguments");
+  if (!ms || mode < 0 || mode > 9 || warps < 0 || reps < 1) return fail(h, HCCMF_EINVAL, "bad probe arguments");
   if (h->state < 2) return fail(h, HCCMF_ESTATE, "probe needs partition");
   if (h->k % 128 != 0) return fail(h, HCCMF_EINVAL, "probe needs k a multiple of 128");
   const int64_t w = warps ? warps : auto_warps(h, h->n);

@@ -2,8 +2,10 @@
 
 Hogwild is nondeterministic, so it is held to the oracle's test-RMSE curve in the same
 schedule, not to its factors:
-  * final: |gpu[E] - oracle[E]| <= 0.005 (at the epoch E where the oracle's
-    curve has flattened, R15);
+  * final: gpu[E] <= oracle[E] + 0.005 ("reach test RMSE within 0.005 of the
+    oracle's", at the epoch E where the oracle's curve has flattened, R15), and not below
+    oracle[E] - 4 x 0.005 (a sanity floor: R33 -- Hogwild's interleaved users are a better-mixed
+    SGD order than the oracle's row-sorted serial sweep and may end lower, e.g. C4 at lambda 1);
   * every epoch e >= 2, one-sided: gpu[e] <= oracle[e] + max(0.005, 0.5 (oracle[e-1] -
     oracle[e])) -- never worse than the oracle by more than 0.005, or, in the steep phase,
     than half an epoch of the oracle's own progress (R29: concurrent rating groups read q_v
@@ -34,7 +36,7 @@ def check(gpu, ora, tag, final_epoch=None, scale=1.0):
     rec = {"tag": tag, "epochs": E, "gap": [round(float(x), 5) for x in gap],
            "allow": [None if not np.isfinite(a) else round(float(a), 5) for a in allow],
            "oracle": [round(float(x), 5) for x in ora[:E + 1]], "gpu": [round(float(x), 5) for x in gpu[:E + 1]],
-           "band": band, "final_ok": bool(abs(gap[E]) <= band), "one_sided_ok": bool(np.all(gap[2:] <= allow[2:]))}
+           "band": band, "final_ok": bool(-4 * band <= gap[E] <= band), "one_sided_ok": bool(np.all(gap[2:] <= allow[2:]))}
     path = os.environ.get("HCCMF_BAND_REPORT")
     if path:
         with open(path, "a") as f:
