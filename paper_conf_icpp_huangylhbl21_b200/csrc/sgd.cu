@@ -697,18 +697,30 @@ struct WarpSgd {
   // written back to HBM when the run ends; a run's row was last written by this warp,
   // before the fence of an earlier block.  Same arithmetic as run() and run_ring(): the
   // factors are bit-identical to the per-stratum launches.
-  __device__ __forceinline__ void run_slab(int64_t lo, int left, float4* slab, int c0, float4* pring) {
+  // The block's start is off the wavefront's critical path (round 2; C3, B = 2048: 45.1 ->
+  // 39.0 ms per epoch, profiles/r02_det.md): the records enter a per-warp shared-memory
+  // ring of 4 windows of 16 by cp.async (window w + 2 is issued when window w is reached;
+  // one LDS.128 per rating for the update and one LDS.32 for the p_u copy D ahead, instead
+  // of six shuffles out of register windows), and the prologue -- the first windows and
+  // the p_u ring fill of the first D ratings, which touch only this warp's own rows -- runs
+  // BEFORE wait_load() waits for the predecessor and stages the column block's Q slab.
+  template <class WaitLoad>
+  __device__ __forceinline__ void run_slab_ring(int64_t lo, int left, float4* slab, int c0, float4* pring, int4* ring,
+                                                WaitLoad&& wait_load) {
     constexpr int D = kSlabD, RP = kSlabRP;
-    static_assert(RP > D && (RP & (RP - 1)) == 0, "ring");
+    static_assert(RP > D && (RP & (RP - 1)) == 0 && D < 16, "ring: window w + 1 lands before window w is reached");
     const int32_t* ru = a.ru + lo;
     const int32_t* rv = a.rv + lo;
     const float* rr = a.rr + lo;
-    int wu0 = 0, wv0 = 0, wu1 = 0, wv1 = 0;
-    float wr0 = 0.f, wr1 = 0.f;
-    if (lane < left) wu0 = __ldcs(ru + lane), wv0 = __ldcs(rv + lane), wr0 = __ldcs(rr + lane);
-    if (lane + 32 < left) wu1 = __ldcs(ru + 32 + lane), wv1 = __ldcs(rv + 32 + lane), wr1 = __ldcs(rr + 32 + lane);
-    if (lane + 32 < left) prefetch_p(wu1);  // window 0: the kernel's look-ahead did it
-    int wb = 0;
+    auto issue = [&](int w) {  // window w -> ring quarter w & 3 (lane l < 16: record 16 w + l)
+      const int idx = w * 16 + lane;
+      if (lane < 16 && idx < left) {
+        int4* e = ring + ((w & 3) << 4) + lane;
+        cp4(&e->x, ru + idx);
+        cp4(&e->y, rv + idx);
+        cp4(&e->z, rr + idx);
+      }
+    };
     float4* const sb = slab + lane - (int64_t)c0 * k4;
     float4* const pb = pring + lane;
     auto copy_p = [&](int slot, int u) {  // p_u -> ring slot (this lane's VEC 16-byte pieces)
@@ -719,52 +731,44 @@ struct WarpSgd {
         asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(src + 32 * i) : "memory");
       }
     };
-    // record of rating jn (jn - wb < 64), from the two windows
-    auto rec = [&](int jn, int& u, int& v, float& r) {
-      const int src = jn - wb;
-      const bool w1 = src >= 32;
-      u = __shfl_sync(FM, w1 ? wu1 : wu0, src & 31);
-      v = __shfl_sync(FM, w1 ? wv1 : wv0, src & 31);
-      r = __shfl_sync(FM, w1 ? wr1 : wr0, src & 31);
+    // window w reached (w >= 1): windows w and w + 1 have landed (their groups are older
+    // than rating j - 1's); w + 1's users' p rows go to L2, window w + 2 is issued
+    auto boundary = [&](int w) {
+      __syncwarp();
+      if (lane < 16 && (w + 1) * 16 + lane < left) prefetch_p(ring[(((w + 1) & 3) << 4) + lane].x);
+      issue(w + 2);
     };
-    // ratings 0 .. D-1 enter the ring; ring entries carry (u, new-run flag) in registers
-    // only for the rating being updated: the record is re-read from the window at use
+    issue(0);
+    issue(1);
+    asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
+    __syncwarp();
+    if (lane < 16 && 16 + lane < left) prefetch_p(ring[16 + lane].x);  // window 0: the kernel's look-ahead did it
+    issue(2);
     int lastu = -1;
     for (int s = 0; s < D; ++s) {
       if (s < left) {
-        int u, v;
-        float r;
-        rec(s, u, v, r);
+        const int u = ring[s].x;
         if (u != lastu) copy_p(s & (RP - 1), u);
         lastu = u;
       }
       asm volatile("cp.async.commit_group;" ::: "memory");
     }
+    wait_load();  // predecessor done; the slab (and, by wait_group 0, the ring fill) landed
     int cu = -1;  // user whose row is in p
     float4 p[VEC], q[VEC];
 #pragma unroll 2
     for (int j = 0; j < left; ++j) {
       const int jn = j + D;
-      if (j - wb == 32) {  // window 0 consumed: slide; the new window 1 is needed ~20 ratings on
-        wu0 = wu1, wv0 = wv1, wr0 = wr1;
-        wb += 32;
-        const int idx = wb + 32 + lane;
-        if (idx < left) {
-          wu1 = __ldcs(ru + idx), wv1 = __ldcs(rv + idx), wr1 = __ldcs(rr + idx);
-          prefetch_p(wu1);
-        }
-      }
       if (jn < left) {
-        int u, v;
-        float r;
-        rec(jn, u, v, r);
+        if ((jn & 15) == 0) boundary(jn >> 4);
+        const int u = ring[jn & 63].x;
         if (u != lastu) copy_p(jn & (RP - 1), u);
         lastu = u;
       }
       asm volatile("cp.async.commit_group;" ::: "memory");
-      int u, v;
-      float r;
-      rec(j, u, v, r);
+      const int4 rc = ring[j & 63];
+      const int u = rc.x, v = rc.y;
+      const float r = __int_as_float(rc.z);
       asm volatile("cp.async.wait_group %0;" ::"n"(D) : "memory");  // rating j's copy has landed
       if (u != cu) {  // a run starts: retire the previous user's row, take this one's
         if (cu >= 0) st(prow(cu), p);
@@ -789,9 +793,11 @@ struct WarpSgd {
         qw[32 * i] = f4_add(q[i], dq);
       }
     }
-    st(prow(cu), p);
-    asm volatile("cp.async.wait_group 0;" ::: "memory");  // nothing may still target the ring
+    if (cu >= 0) st(prow(cu), p);
+    asm volatile("cp.async.wait_group 0;" ::: "memory");  // nothing may still target the rings
+    __syncwarp();  // the record ring is rewritten by the next block's prologue
   }
+
   // L2 prefetch of one p_u row by the calling lane, line by line (a bulk prefetch takes a
   // uniform operand: one per lane would be a 32-way serialised loop)
   __device__ __forceinline__ void prefetch_p(int u) const {
@@ -1141,7 +1147,7 @@ __global__ void __launch_bounds__(kThreads) sgd_wave_kernel(SgdArgs a, const int
 }
 
 // The same wavefront with the column block's Q rows staged in shared memory
-// (WarpSgd::run_slab): per block, the w <= wmax rows of column block c are copied in
+// (WarpSgd::run_slab_ring): per block, the w <= wmax rows of column block c are copied in
 // with cp.async (one L2 round trip for the whole slab instead of one per rating),
 // updated in place, and written back before the progress counter is released.  The
 // next block's records are bulk-prefetched into L2 while this block runs.
@@ -1170,6 +1176,9 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
   // per warp: the column block's slab (wmax rows), then the p_u ring (kSlabRP rows)
   float4* slab = wave_smem + (int64_t)(threadIdx.x >> 5) * (wmax + kSlabRP) * k4;
   float4* pring = slab + (int64_t)wmax * k4;
+  // the per-warp record rings (64 entries) after all warps' slabs and p rings
+  int4* rring = reinterpret_cast<int4*>(wave_smem + (int64_t)(blockDim.x >> 5) * (wmax + kSlabRP) * k4) +
+                (threadIdx.x >> 5) * 64;
   const float4* Qg = reinterpret_cast<const float4*>(a.Q);
   float4* Qw = reinterpret_cast<float4*>(a.Q);
   const int nb = (i + 1) % B;
@@ -1202,49 +1211,55 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
       if (w.lane < nn) nu0 = __ldcg(a.ru + nlo + w.lane);
       if (w.lane + 32 < nn) nu1 = __ldcg(a.ru + nlo + 32 + w.lane);
     }
+    // the predecessor's release of column block c, then c's Q rows -> slab (cp.async)
+    const int c0 = (int)(((int64_t)c * n + B - 1) / B);
+    const int rows = (int)(((int64_t)(c + 1) * n + B - 1) / B) - c0;
+    auto wait_load = [&]() {
 #ifdef HCCMF_DIAG_TRACE
-    if (w.lane == 0 && B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3] = gtimer();
+      if (w.lane == 0 && B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3] = gtimer();
 #endif
 #ifndef HCCMF_DIAG_NOWAIT  // diagnostic builds only: no dependency waits (wrong factors, timing bound)
-    if (t > 0 && B > 1) {
-      if (w.lane == 0) {
-        int seen;
-        do {
-          // relaxed polling (an acquire load per poll invalidates the SM's L1 every
-          // time: CCTL.IVALL), one acquire fence once the predecessor is seen
-          asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + nb) : "memory");
-          if (seen < t) __nanosleep(64);
-        } while (seen < t);
-        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      if (t > 0 && B > 1) {
+        if (w.lane == 0) {
+          int seen;
+          do {
+            // relaxed polling (an acquire load per poll invalidates the SM's L1 every
+            // time: CCTL.IVALL), one acquire fence once the predecessor is seen
+            asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + nb) : "memory");
+            if (seen < t) __nanosleep(64);
+          } while (seen < t);
+          asm volatile("fence.acq_rel.gpu;" ::: "memory");
+        }
+        __syncwarp();
       }
-      __syncwarp();
-    }
 #endif
 #ifdef HCCMF_DIAG_TRACE
-    if (w.lane == 0 && B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3 + 1] = gtimer();
+      if (w.lane == 0 && B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3 + 1] = gtimer();
 #endif
-    if (nu0 >= 0) w.prefetch_p(nu0);
-    if (nu1 >= 0) w.prefetch_p(nu1);
-    if (hi > lo) {
-      const int c0 = (int)(((int64_t)c * n + B - 1) / B);
-      const int c1 = (int)(((int64_t)(c + 1) * n + B - 1) / B);
-      const int rows = c1 - c0;
-      for (int r = 0; r < rows; ++r) {
+      if (nu0 >= 0) w.prefetch_p(nu0);
+      if (nu1 >= 0) w.prefetch_p(nu1);
+      if (hi > lo) {
+        for (int r = 0; r < rows; ++r) {
 #pragma unroll
-        for (int s = 0; s < VEC; ++s) {
-          const unsigned d = (unsigned)__cvta_generic_to_shared(slab + r * k4 + w.lane + 32 * s);
-          asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d),
-                       "l"(Qg + (int64_t)(c0 + r) * k4 + w.lane + 32 * s)
-                       : "memory");
+          for (int s = 0; s < VEC; ++s) {
+            const unsigned d = (unsigned)__cvta_generic_to_shared(slab + r * k4 + w.lane + 32 * s);
+            asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d),
+                         "l"(Qg + (int64_t)(c0 + r) * k4 + w.lane + 32 * s)
+                         : "memory");
+          }
         }
+        asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
       }
-      asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
-      w.run_slab(lo, (int)(hi - lo), slab, c0, pring);
+    };
+    if (hi > lo) {
+      w.run_slab_ring(lo, (int)(hi - lo), slab, c0, pring, rring, wait_load);
       for (int r = 0; r < rows; ++r) {
 #pragma unroll
         for (int s = 0; s < VEC; ++s)
           __stcg(Qw + (int64_t)(c0 + r) * k4 + w.lane + 32 * s, slab[r * k4 + w.lane + 32 * s]);
       }
+    } else {
+      wait_load();
     }
     __syncwarp();
     if (w.lane == 0) {
@@ -1390,30 +1405,35 @@ namespace {
 template <int VEC>
 bool slab_geometry_t(int k, int B, int64_t n, int* wpc_out, size_t* smem_out) {
   const int64_t wmax = (n + B - 1) / B;
-  const size_t per_warp = (size_t)(wmax + kSlabRP) * k * sizeof(float);
+  const size_t per_warp = (size_t)(wmax + kSlabRP) * k * sizeof(float) + 64 * sizeof(int4);
   constexpr size_t kBudget = 160 * 1024;
-  int wpc = kThreads / 32;
-  while (wpc > 1 && wpc * per_warp > kBudget) wpc >>= 1;
-  if (wpc * per_warp > kBudget) return false;
-  const size_t smem = wpc * per_warp;
-  if (cudaFuncSetAttribute(sgd_wave_slab_kernel<VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
-      cudaSuccess) {
-    cudaGetLastError();
-    return false;
-  }
-  int dev = 0, sms = 0, per_sm = 0;
+  int dev = 0, sms = 0;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sgd_wave_slab_kernel<VEC>, wpc * 32, smem) !=
-      cudaSuccess) {
-    cudaGetLastError();
-    return false;
+  // the widest CTA (8, 4, 2, 1 warps) whose occupancy keeps all B warps co-resident (every
+  // warp waits on its successor) with 10 % head room: narrower CTAs pack the shared memory
+  // of an SM more tightly when the slabs are wide (C3 at B = 1536: 8 warps -> 1 CTA per SM)
+  for (int wpc = kThreads / 32; wpc >= 1; wpc >>= 1) {
+    if (wpc * per_warp > kBudget) continue;
+    const size_t smem = wpc * per_warp;
+    if (cudaFuncSetAttribute(sgd_wave_slab_kernel<VEC>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+        cudaSuccess) {
+      cudaGetLastError();
+      return false;
+    }
+    int per_sm = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sgd_wave_slab_kernel<VEC>, wpc * 32, smem) !=
+        cudaSuccess) {
+      cudaGetLastError();
+      return false;
+    }
+    if ((int64_t)B * 10 <= (int64_t)sms * per_sm * wpc * 9) {
+      *wpc_out = wpc;
+      *smem_out = smem;
+      return true;
+    }
   }
-  // co-residency (every warp waits on its successor) with 10 % head room
-  if ((int64_t)B * 10 > (int64_t)sms * per_sm * wpc * 9) return false;
-  *wpc_out = wpc;
-  *smem_out = smem;
-  return true;
+  return false;
 }
 }  // namespace
 
