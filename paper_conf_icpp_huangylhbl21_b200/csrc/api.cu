@@ -230,7 +230,7 @@ void free_partition(hccmf_t h) {
   dfree(h, h->d_counters, h->n_counters);
   h->n_counters = 0;
   dfree(h, h->d_blk_off, h->nblk_local + 1);
-  dfree(h, h->d_progress, h->Br);
+  dfree(h, h->d_progress, (size_t)h->Br * kProgressStride);
   det_chain_free(&h->det_chain, h->stream);
   h->local_nnz = 0;
   h->rows = 0;
@@ -1112,7 +1112,7 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   // local block offsets stay on the device for the DET wavefront
   CU(h, dmalloc(h, &h->d_blk_off, h->nblk_local + 1));
   CU(h, cudaMemcpyAsync(h->d_blk_off, loc_off.data(), sizeof(int64_t) * (h->nblk_local + 1), cudaMemcpyHostToDevice, st));
-  CU(h, dmalloc(h, &h->d_progress, h->Br));
+  CU(h, dmalloc(h, &h->d_progress, (size_t)h->Br * kProgressStride));
   h->h_task_lo.resize(nt);
   h->h_task_hi.resize(nt);
   if (nt) {

@@ -285,7 +285,7 @@ __global__ void __launch_bounds__(NW * 32) sgd_wave_chain_kernel(ChainArgs a, in
       if (tid == 0) {
         int seen;
         do {
-          asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + nb) : "memory");
+          asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + (int64_t)nb * kProgressStride) : "memory");
           if (seen < t) __nanosleep(64);
         } while (seen < t);
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
@@ -392,7 +392,7 @@ __global__ void __launch_bounds__(NW * 32) sgd_wave_chain_kernel(ChainArgs a, in
     __syncthreads();
     if (tid == 0) {
       asm volatile("fence.acq_rel.gpu;" ::: "memory");
-      asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(progress + i), "r"(t + 1) : "memory");
+      asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(progress + (int64_t)i * kProgressStride), "r"(t + 1) : "memory");
 #ifdef HCCMF_DIAG_TRACE
       if (B <= 2048) {
         g_chain_trace[((int64_t)i * B + t) * 4 + 2] = ctimer();
@@ -550,7 +550,7 @@ cudaError_t launch_wave_chain(const DetChain& d, float* P, float* Q, int64_t row
   a.seg_gend = d.seg_gend;
   a.run_user = d.run_user;
   const int wmax = (int)((n + B - 1) / B);
-  cudaError_t e = cudaMemsetAsync(progress, 0, sizeof(int) * B, st);
+  cudaError_t e = cudaMemsetAsync(progress, 0, sizeof(int) * kProgressStride * (size_t)B, st);
   if (e != cudaSuccess) return e;
   int SU = 0, ng = 0, v = 0;
   size_t smem = 0;

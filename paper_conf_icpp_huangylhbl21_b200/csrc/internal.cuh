@@ -13,6 +13,10 @@
 
 namespace hccmf {
 
+// DET wavefront progress counters: one per 128-byte line (counter i at progress[i * kProgressStride]),
+// so the warps polling their successors spread over L2 slices instead of hammering a few lines
+constexpr int kProgressStride = 32;
+
 // every <<<...>>> launch site of the library is written (note_launch(), kernel<<<...>>>(...))
 // so hccmf_kernel_launches() reports what actually ran (bench.py's gpu_launches)
 inline std::atomic<long long> g_kernel_launches{0};

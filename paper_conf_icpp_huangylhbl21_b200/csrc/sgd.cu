@@ -756,6 +756,7 @@ struct WarpSgd {
     wait_load();  // predecessor done; the slab (and, by wait_group 0, the ring fill) landed
     int cu = -1;  // user whose row is in p
     float4 p[VEC], q[VEC];
+    int4 rc = ring[0];  // rating j's record, read one rating ahead (off the q_v chain)
 #pragma unroll 2
     for (int j = 0; j < left; ++j) {
       const int jn = j + D;
@@ -766,9 +767,9 @@ struct WarpSgd {
         lastu = u;
       }
       asm volatile("cp.async.commit_group;" ::: "memory");
-      const int4 rc = ring[j & 63];
       const int u = rc.x, v = rc.y;
       const float r = __int_as_float(rc.z);
+      rc = ring[(j + 1) & 63];  // visible since its window's boundary (j + 1 < jn)
       asm volatile("cp.async.wait_group %0;" ::"n"(D) : "memory");  // rating j's copy has landed
       if (u != cu) {  // a run starts: retire the previous user's row, take this one's
         if (cu >= 0) st(prow(cu), p);
@@ -1128,7 +1129,7 @@ __global__ void __launch_bounds__(kThreads) sgd_wave_kernel(SgdArgs a, const int
         do {
           // relaxed polling (an acquire load per poll invalidates the SM's L1 every
           // time: CCTL.IVALL), one acquire fence once the predecessor is seen
-          asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + nb) : "memory");
+          asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + (int64_t)nb * kProgressStride) : "memory");
           if (seen < t) __nanosleep(64);
         } while (seen < t);
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
@@ -1141,7 +1142,7 @@ __global__ void __launch_bounds__(kThreads) sgd_wave_kernel(SgdArgs a, const int
     __syncwarp();
     if (w.lane == 0) {
       asm volatile("fence.acq_rel.gpu;" ::: "memory");  // the warp's writes (ordered by __syncwarp) first
-      asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(progress + i), "r"(t + 1) : "memory");
+      asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(progress + (int64_t)i * kProgressStride), "r"(t + 1) : "memory");
     }
   }
 }
@@ -1225,7 +1226,7 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
           do {
             // relaxed polling (an acquire load per poll invalidates the SM's L1 every
             // time: CCTL.IVALL), one acquire fence once the predecessor is seen
-            asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + nb) : "memory");
+            asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + (int64_t)nb * kProgressStride) : "memory");
             if (seen < t) __nanosleep(64);
           } while (seen < t);
           asm volatile("fence.acq_rel.gpu;" ::: "memory");
@@ -1264,7 +1265,7 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
     __syncwarp();
     if (w.lane == 0) {
       asm volatile("fence.acq_rel.gpu;" ::: "memory");  // the warp's writes (ordered by __syncwarp) first
-      asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(progress + i), "r"(t + 1) : "memory");
+      asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(progress + (int64_t)i * kProgressStride), "r"(t + 1) : "memory");
 #ifdef HCCMF_DIAG_TRACE
       if (B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3 + 2] = gtimer();
 #endif
@@ -1388,7 +1389,7 @@ cudaError_t launch_cooperative(void (*kernel)(KArgs...), unsigned blocks, unsign
 cudaError_t launch_wave(const SgdArgs& a, const int64_t* off, int B, int* progress, cudaStream_t st) {
   int L, VEC;
   sgd_geometry(a.k, a.vec_pref, &L, &VEC);
-  cudaError_t e = cudaMemsetAsync(progress, 0, sizeof(int) * B, st);
+  cudaError_t e = cudaMemsetAsync(progress, 0, sizeof(int) * kProgressStride * (size_t)B, st);
   if (e != cudaSuccess) return e;
   const unsigned blocks = (unsigned)(((int64_t)B * 32 + kThreads - 1) / kThreads);
   switch (VEC) {
@@ -1454,7 +1455,7 @@ cudaError_t launch_wave_slab(const SgdArgs& a, const int64_t* off, int B, int* p
   int L, VEC, wpc = 0;
   size_t smem = 0;
   sgd_geometry(a.k, a.vec_pref, &L, &VEC);
-  cudaError_t e = cudaMemsetAsync(progress, 0, sizeof(int) * B, st);
+  cudaError_t e = cudaMemsetAsync(progress, 0, sizeof(int) * kProgressStride * (size_t)B, st);
   if (e != cudaSuccess) return e;
   const int wmax = (int)((n + B - 1) / B);
 #define SLAB_CASE(V)                                                                                        \
