@@ -769,7 +769,7 @@ struct WarpSgd {
       asm volatile("cp.async.commit_group;" ::: "memory");
       const int u = rc.x, v = rc.y;
       const float r = __int_as_float(rc.z);
-      rc = ring[(j + 1) & 63];  // visible since its window's boundary (j + 1 < jn)
+      if (j + 1 < left) rc = ring[(j + 1) & 63];  // visible since its window's boundary (j + 1 < jn)
       asm volatile("cp.async.wait_group %0;" ::"n"(D) : "memory");  // rating j's copy has landed
       if (u != cu) {  // a run starts: retire the previous user's row, take this one's
         if (cu >= 0) st(prow(cu), p);
