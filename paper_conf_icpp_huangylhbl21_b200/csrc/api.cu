@@ -235,8 +235,6 @@ void free_partition(hccmf_t h) {
   h->local_nnz = 0;
   h->rows = 0;
   h->blk_task_off.clear();
-  h->h_task_lo.clear();
-  h->h_task_hi.clear();
 }
 
 // ------------------------------------------------------------ timeline (HCCMF_OPT_TIMELINE)
@@ -364,21 +362,27 @@ hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
                                     sched == HCCMF_SCHED_HOGWILD ? (int)h->opt_phases : 1);
   if (msg) return fail(h, HCCMF_EINVAL, "%s", msg);
   pl.phases = sched == HCCMF_SCHED_HOGWILD ? (int)h->opt_phases : 1;
-  std::vector<int64_t> lo, hi;
+  // DET: one task per non-empty block, from the host block offsets.  HOGWILD: the blocks'
+  // task ranges of the device task list, gathered on the device (segment tables only)
+  std::vector<int64_t> lo, hi, seg_src, seg_dst;
+  int64_t total = 0;
   for (const BlockLaunch& L : bl) {
-    const int64_t t0 = (int64_t)lo.size();
+    const int64_t t0 = total;
     for (int64_t b : L.blocks) {
-      if (sched == HCCMF_SCHED_DET) {  // one task per non-empty block
+      if (sched == HCCMF_SCHED_DET) {
         const int64_t a = h->block_off[b] - h->rec0, e = h->block_off[b + 1] - h->rec0;
         if (e > a) {
           lo.push_back(a);
           hi.push_back(e);
+          ++total;
         }
-      } else {  // the block's user-aligned tasks
+      } else {
         const int64_t j = b - h->blk0;
-        for (int64_t t = h->blk_task_off[j]; t < h->blk_task_off[j + 1]; ++t) {
-          lo.push_back(h->h_task_lo[t]);
-          hi.push_back(h->h_task_hi[t]);
+        const int64_t cnt = h->blk_task_off[j + 1] - h->blk_task_off[j];
+        if (cnt > 0) {
+          seg_src.push_back(h->blk_task_off[j]);
+          seg_dst.push_back(total);
+          total += cnt;
         }
       }
     }
@@ -388,14 +392,17 @@ hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
     cbs.erase(std::unique(cbs.begin(), cbs.end()), cbs.end());
     int64_t items = 0;
     for (int64_t cb : cbs) items += ceil_div((cb + 1) * h->n, h->Bc) - ceil_div(cb * h->n, h->Bc);
-    pl.launches.push_back(Launch{t0, (int64_t)lo.size() - t0, L.qrep, L.stage, L.phase, items});
+    pl.launches.push_back(Launch{t0, total - t0, L.qrep, L.stage, L.phase, items});
   }
-  pl.n_tasks = (int64_t)lo.size();
+  pl.n_tasks = total;
   CU(h, dmalloc(h, &pl.d_lo, pl.n_tasks));
   CU(h, dmalloc(h, &pl.d_hi, pl.n_tasks));
-  if (pl.n_tasks) {
+  if (sched == HCCMF_SCHED_DET && pl.n_tasks) {
     CU(h, cudaMemcpyAsync(pl.d_lo, lo.data(), sizeof(int64_t) * pl.n_tasks, cudaMemcpyHostToDevice, h->stream));
     CU(h, cudaMemcpyAsync(pl.d_hi, hi.data(), sizeof(int64_t) * pl.n_tasks, cudaMemcpyHostToDevice, h->stream));
+  } else if (pl.n_tasks) {
+    CU(h, k_gather_tasks(seg_src.data(), seg_dst.data(), (int64_t)seg_src.size(), total, h->d_task_lo, h->d_task_hi,
+                         pl.d_lo, pl.d_hi, h->stream));
   }
   if ((int64_t)pl.launches.size() > h->n_counters) {
     dfree(h, h->d_counters, h->n_counters);
@@ -1113,20 +1120,9 @@ hccmf_status hccmf_partition(hccmf_t h, const hccmf_partition_opts* o) {
   CU(h, dmalloc(h, &h->d_blk_off, h->nblk_local + 1));
   CU(h, cudaMemcpyAsync(h->d_blk_off, loc_off.data(), sizeof(int64_t) * (h->nblk_local + 1), cudaMemcpyHostToDevice, st));
   CU(h, dmalloc(h, &h->d_progress, (size_t)h->Br * kProgressStride));
-  h->h_task_lo.resize(nt);
-  h->h_task_hi.resize(nt);
-  if (nt) {
-    CU(h, cudaMemcpyAsync(h->h_task_lo.data(), h->d_task_lo, sizeof(int64_t) * nt, cudaMemcpyDeviceToHost, st));
-    CU(h, cudaMemcpyAsync(h->h_task_hi.data(), h->d_task_hi, sizeof(int64_t) * nt, cudaMemcpyDeviceToHost, st));
-  }
-  CU(h, cudaStreamSynchronize(st));
-  // tasks are grouped by block (LPT order inside a block): count per block
+  // tasks are grouped by block (LPT order inside a block): the first task of every block
   h->blk_task_off.assign(h->nblk_local + 1, 0);
-  for (int64_t t = 0; t < nt; ++t) {
-    const int64_t j = std::upper_bound(loc_off.begin(), loc_off.end(), h->h_task_lo[t]) - loc_off.begin() - 1;
-    h->blk_task_off[j + 1] += 1;
-  }
-  for (int64_t j = 0; j < h->nblk_local; ++j) h->blk_task_off[j + 1] += h->blk_task_off[j];
+  CU(h, k_task_block_offsets(h->d_task_lo, nt, h->d_blk_off, h->nblk_local, h->blk_task_off.data(), st));
 
   timer.mark("hogwild tasks");
   // ---- factors

@@ -543,4 +543,69 @@ cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* off, i
   return cudaSuccess;
 }
 
+// ---- task index per block and plan gathering, without a host copy of the tasks
+namespace {
+__device__ __forceinline__ int64_t block_of(const int64_t* off, int64_t nb, int64_t lo) {
+  int64_t a = 0, b = nb;  // largest j in [0, nb) with off[j] <= lo
+  while (b - a > 1) {
+    const int64_t mid = (a + b) >> 1;
+    if (off[mid] <= lo) a = mid; else b = mid;
+  }
+  return a;
+}
+__global__ void task_block_start_kernel(const int64_t* __restrict__ task_lo, int64_t nt, const int64_t* __restrict__ off,
+                                        int64_t nb, int64_t* __restrict__ start) {
+  for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nt; t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = block_of(off, nb, task_lo[t]);
+    if (t == 0 || block_of(off, nb, task_lo[t - 1]) != b) start[b] = t;
+  }
+}
+__global__ void gather_tasks_kernel(const int64_t* __restrict__ seg_src, const int64_t* __restrict__ seg_dst,
+                                    int64_t nseg, int64_t total, const int64_t* __restrict__ lo,
+                                    const int64_t* __restrict__ hi, int64_t* __restrict__ olo, int64_t* __restrict__ ohi) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    int64_t a = 0, b = nseg;  // segment s with seg_dst[s] <= i < seg_dst[s + 1]
+    while (b - a > 1) {
+      const int64_t mid = (a + b) >> 1;
+      if (seg_dst[mid] <= i) a = mid; else b = mid;
+    }
+    const int64_t src = seg_src[a] + (i - seg_dst[a]);
+    olo[i] = lo[src];
+    ohi[i] = hi[src];
+  }
+}
+}  // namespace
+
+cudaError_t k_task_block_offsets(const int64_t* task_lo, int64_t nt, const int64_t* off, int64_t nb, int64_t* blk_task_off,
+                                 cudaStream_t st) {
+  int64_t* d = nullptr;
+  CKR(dalloc(&d, nb + 1, st));
+  CKR(cudaMemsetAsync(d, 0xff, sizeof(int64_t) * (nb + 1), st));  // -1: no task starts there
+  if (nt > 0) (note_launch(), task_block_start_kernel<<<grid_for(nt), kT, 0, st>>>(task_lo, nt, off, nb, d));
+  CKR(cudaGetLastError());
+  CKR(cudaMemcpyAsync(blk_task_off, d, sizeof(int64_t) * (nb + 1), cudaMemcpyDeviceToHost, st));
+  CKR(cudaStreamSynchronize(st));
+  cudaFreeAsync(d, st);
+  blk_task_off[nb] = nt;  // a block without tasks starts where the next one does
+  for (int64_t j = nb - 1; j >= 0; --j)
+    if (blk_task_off[j] < 0) blk_task_off[j] = blk_task_off[j + 1];
+  return cudaSuccess;
+}
+
+cudaError_t k_gather_tasks(const int64_t* seg_src, const int64_t* seg_dst, int64_t nseg, int64_t total,
+                           const int64_t* lo, const int64_t* hi, int64_t* olo, int64_t* ohi, cudaStream_t st) {
+  if (total <= 0 || nseg <= 0) return cudaSuccess;
+  int64_t *ds = nullptr, *dd = nullptr;
+  CKR(dalloc(&ds, nseg, st));
+  CKR(dalloc(&dd, nseg, st));
+  CKR(cudaMemcpyAsync(ds, seg_src, sizeof(int64_t) * nseg, cudaMemcpyHostToDevice, st));
+  CKR(cudaMemcpyAsync(dd, seg_dst, sizeof(int64_t) * nseg, cudaMemcpyHostToDevice, st));
+  (note_launch(), gather_tasks_kernel<<<grid_for(total), kT, 0, st>>>(ds, dd, nseg, total, lo, hi, olo, ohi));
+  CKR(cudaGetLastError());
+  CKR(cudaStreamSynchronize(st));  // the host segment tables are the caller's
+  cudaFreeAsync(ds, st);
+  cudaFreeAsync(dd, st);
+  return cudaSuccess;
+}
+
 }  // namespace hccmf

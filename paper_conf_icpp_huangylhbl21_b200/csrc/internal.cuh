@@ -148,6 +148,14 @@ cudaError_t k_shard_split(const int32_t* u, const int32_t* v, const float* r, in
 cudaError_t k_build_tasks(const int32_t* ru, int64_t nrec, const int64_t* blk_off_local /*nb+1, local idx*/,
                           int64_t nb, int64_t target, int64_t heavy, int64_t** task_lo, int64_t** task_hi, int64_t* n_tasks,
                           cudaStream_t st);
+// blk_task_off (host, nb + 1): the first task of every block (tasks are grouped by block; a
+// block without tasks starts where the next one does), computed on the device
+cudaError_t k_task_block_offsets(const int64_t* task_lo, int64_t nt, const int64_t* blk_off_local /*device, nb+1*/,
+                                 int64_t nb, int64_t* blk_task_off, cudaStream_t st);
+// plan task lists: segment s copies tasks [seg_src[s], +len) to [seg_dst[s], seg_dst[s+1]) (host
+// tables, seg_dst ascending, the last segment ends at total)
+cudaError_t k_gather_tasks(const int64_t* seg_src, const int64_t* seg_dst, int64_t nseg, int64_t total,
+                           const int64_t* lo, const int64_t* hi, int64_t* olo, int64_t* ohi, cudaStream_t st);
 
 // ------------------------------------------------------------ eval/export
 cudaError_t k_init_factors(uint64_t seed, uint64_t tag, int64_t rows_total, int32_t k, const int32_t* perm,
@@ -227,7 +235,6 @@ struct hccmf_ctx {
   int64_t n_tasks = 0;
   int64_t* d_task_lo = nullptr;
   int64_t* d_task_hi = nullptr;
-  std::vector<int64_t> h_task_lo, h_task_hi;  // host copies for plan building
 
   // factors
   int64_t row0 = 0, rows = 0;
