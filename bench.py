@@ -276,10 +276,14 @@ def roofline(cfg, name, storage, sched, info, kmean_ms, step_ms, peak, peak_src,
     if sched == "hogwild":
         roof["binding_unit"] = b["unit"]
         if probe:
-            mode, pms = probe
+            mode, pms = probe[:2]
             roof["binding_ceiling"] = {"probe": mode, "ms": pms, "updates_per_s": nnz_l / (pms / 1e3),
                                        "source": "hccmf_probe_roundtrip: same records and warps, q_v traffic only"}
             roof["binding_frac"] = pms / kmean_ms
+            if len(probe) > 2:  # fp32: q_v load + dependent vector reduction, one rating ahead, no arithmetic
+                roof["roundtrip_ceiling"] = {"probe": "ldred_f32", "ms": probe[2],
+                                             "updates_per_s": nnz_l / (probe[2] / 1e3)}
+                roof["roundtrip_frac"] = probe[2] / kmean_ms
     else:
         roof["binding_unit"] = ("the hottest column block's serial dependency chain (wavefront; "
                                 "profiles/r01_det_wavefront.md)")
@@ -402,6 +406,8 @@ def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, samp
         if sched == "hogwild" and cfg.k % 128 == 0:
             mode = PROBE_MODE["fp32" if storage == "fp32" else "fp16"]
             probe = (mode, mdl.probe_roundtrip(mode, warps=args.warps, reps=3))
+            if storage == "fp32":  # the load + dependent reduction round trip as well (the kernel's own pattern)
+                probe = probe + (mdl.probe_roundtrip("ldred_f32", warps=args.warps, reps=3),)
         roof = roofline(cfg, name, storage, sched, info, kmean, ms / steps, peak, peak_src, probe)
         return {"value": nnz * steps / (ms / 1e3), "ms": ms, "roofline": roof, "clocks": clk,
                 "curve": curve + rms, "launches": launches}
