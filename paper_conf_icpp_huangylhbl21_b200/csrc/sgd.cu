@@ -757,20 +757,18 @@ struct WarpSgd {
     int cu = -1;  // user whose row is in p
     float4 p[VEC], q[VEC];
     int4 rc = ring[0];  // rating j's record, read one rating ahead (off the q_v chain)
+    // Issue order matters (one warp issues in order): rating j's operands are requested
+    // first, the look-ahead for rating j + D (whose user read -> compare -> copy would
+    // otherwise stall the warp right after the previous q_v write) goes under the
+    // dot-product reduction.
 #pragma unroll 2
     for (int j = 0; j < left; ++j) {
-      const int jn = j + D;
-      if (jn < left) {
-        if ((jn & 15) == 0) boundary(jn >> 4);
-        const int u = ring[jn & 63].x;
-        if (u != lastu) copy_p(jn & (RP - 1), u);
-        lastu = u;
-      }
-      asm volatile("cp.async.commit_group;" ::: "memory");
       const int u = rc.x, v = rc.y;
       const float r = __int_as_float(rc.z);
-      if (j + 1 < left) rc = ring[(j + 1) & 63];  // visible since its window's boundary (j + 1 < jn)
-      asm volatile("cp.async.wait_group %0;" ::"n"(D) : "memory");  // rating j's copy has landed
+#ifndef HCCMF_DIAG_NO_DEPBAR
+      // groups 0 .. j + D - 1 are committed: at most D - 1 pending = rating j's copy landed
+      asm volatile("cp.async.wait_group %0;" ::"n"(D - 1) : "memory");
+#endif
       if (u != cu) {  // a run starts: retire the previous user's row, take this one's
         if (cu >= 0) st(prow(cu), p);
 #pragma unroll
@@ -780,12 +778,27 @@ struct WarpSgd {
       float4* qw = sb + v * k4;
 #pragma unroll
       for (int i = 0; i < VEC; ++i) q[i] = qw[32 * i];  // after the previous write: serial order
+      if (j + 1 < left) rc = ring[(j + 1) & 63];  // visible since its window's boundary (j + 1 < j + D)
       float2 dd = make_float2(0.f, 0.f);
 #pragma unroll
       for (int i = 0; i < VEC; ++i) dd = f4_dot2(p[i], q[i], dd);
       float d = dd.x + dd.y;
+      {  // look-ahead of rating j + D: its window boundary, its user's p_u copy, one commit group
+        const int jn = j + D;
+        if (jn < left) {
+          if ((jn & 15) == 0) boundary(jn >> 4);
+          const int un = ring[jn & 63].x;
+          if (un != lastu) copy_p(jn & (RP - 1), un);
+          lastu = un;
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+      }
+#ifdef HCCMF_DIAG_SHFL_LEVELS  // diagnostic builds only: fewer reduction levels (wrong factors)
+      for (int o = 1 << (HCCMF_DIAG_SHFL_LEVELS - 1); o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
+#else
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
+#endif
       const float ge = g * (r - d);
 #pragma unroll
       for (int i = 0; i < VEC; ++i) {
