@@ -731,6 +731,17 @@ struct WarpSgd {
         asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(src + 32 * i) : "memory");
       }
     };
+    // the same copy, issued only if `go` (a predicated cp.async: no branch in the loop)
+    auto copy_p_if = [&](int slot, int u, bool go) {
+      const float4* src = prow(u);
+#pragma unroll
+      for (int i = 0; i < VEC; ++i) {
+        const unsigned d = (unsigned)__cvta_generic_to_shared(pb + slot * k4 + 32 * i);
+        asm volatile("{\n\t.reg .pred P;\n\tsetp.ne.b32 P, %2, 0;\n\t@P cp.async.cg.shared.global [%0], [%1], 16;\n\t}" ::"r"(d),
+                     "l"(src + 32 * i), "r"((int)go)
+                     : "memory");
+      }
+    };
     // window w reached (w >= 1): windows w and w + 1 have landed (their groups are older
     // than rating j - 1's); w + 1's users' p rows go to L2, window w + 2 is issued
     auto boundary = [&](int w) {
@@ -756,11 +767,13 @@ struct WarpSgd {
     wait_load();  // predecessor done; the slab (and, by wait_group 0, the ring fill) landed
     int cu = -1;  // user whose row is in p
     float4 p[VEC], q[VEC];
-    int4 rc = ring[0];  // rating j's record, read one rating ahead (off the q_v chain)
-    // Issue order matters (one warp issues in order): rating j's operands are requested
-    // first, the look-ahead for rating j + D (whose user read -> compare -> copy would
-    // otherwise stall the warp right after the previous q_v write) goes under the
-    // dot-product reduction.
+    int4 rc = ring[0];       // rating j's record, read one rating ahead (off the q_v chain)
+    int un = ring[D].x;      // the user of rating j + D, read one rating ahead as well
+    // Issue order matters (one warp issues in order, and on the wavefront's critical path
+    // it is alone): rating j's operands are requested first, the look-ahead of rating
+    // j + D (compare, predicated p_u copy, commit) sits between the reduction's first two
+    // levels, and the next look-ahead's user is read right after this rating's q_v write
+    // (a window boundary is handled one rating early so that read always finds it).
 #pragma unroll 2
     for (int j = 0; j < left; ++j) {
       const int u = rc.x, v = rc.y;
@@ -783,22 +796,21 @@ struct WarpSgd {
 #pragma unroll
       for (int i = 0; i < VEC; ++i) dd = f4_dot2(p[i], q[i], dd);
       float d = dd.x + dd.y;
-      {  // look-ahead of rating j + D: its window boundary, its user's p_u copy, one commit group
-        const int jn = j + D;
-        if (jn < left) {
-          if ((jn & 15) == 0) boundary(jn >> 4);
-          const int un = ring[jn & 63].x;
-          if (un != lastu) copy_p(jn & (RP - 1), un);
-          lastu = un;
-        }
-        asm volatile("cp.async.commit_group;" ::: "memory");
-      }
 #ifdef HCCMF_DIAG_SHFL_LEVELS  // diagnostic builds only: fewer reduction levels (wrong factors)
-      for (int o = 1 << (HCCMF_DIAG_SHFL_LEVELS - 1); o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
+      for (int o = 1 << (HCCMF_DIAG_SHFL_LEVELS - 1); o > 0; o >>= 1) {
 #else
 #pragma unroll
-      for (int o = 16; o > 0; o >>= 1) d += __shfl_xor_sync(FM, d, o);
+      for (int o = 16; o > 0; o >>= 1) {
 #endif
+        d += __shfl_xor_sync(FM, d, o);
+        if (o == 16) {  // look-ahead of rating j + D: its user's p_u copy, one commit group
+          const int jn = j + D;
+          const bool go = jn < left && un != lastu;
+          copy_p_if(jn & (RP - 1), go ? un : lastu, go);
+          if (go) lastu = un;
+          asm volatile("cp.async.commit_group;" ::: "memory");
+        }
+      }
       const float ge = g * (r - d);
 #pragma unroll
       for (int i = 0; i < VEC; ++i) {
@@ -806,6 +818,9 @@ struct WarpSgd {
         p[i] = f4_fma(ge, q[i], f4_scale(c1, p[i]));
         qw[32 * i] = f4_add(q[i], dq);
       }
+      const int jn1 = j + 1 + D;  // the next look-ahead's rating
+      if (jn1 < left && (jn1 & 15) == 0) boundary(jn1 >> 4);
+      un = ring[jn1 & 63].x;  // beyond the block: a stale entry, never copied
     }
     if (cu >= 0) st(prow(cu), p);
     asm volatile("cp.async.wait_group 0;" ::: "memory");  // nothing may still target the rings
