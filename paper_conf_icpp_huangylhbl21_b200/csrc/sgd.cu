@@ -364,6 +364,15 @@ struct WarpSgd {
 #pragma unroll
     for (int i = 0; i < VEC; ++i) __stcg(const_cast<float4*>(r) + 32 * i, x[i]);
   }
+  // the same store, performed only if `go` (predicated: no branch)
+  __device__ __forceinline__ void st_if(const float4* r, const float4 (&x)[VEC], bool go) const {
+#pragma unroll
+    for (int i = 0; i < VEC; ++i)
+      asm volatile("{\n\t.reg .pred P;\n\tsetp.ne.b32 P, %5, 0;\n\t@P st.global.cg.v4.f32 [%0], {%1, %2, %3, %4};\n\t}" ::"l"(
+                       r + 32 * i),
+                   "f"(x[i].x), "f"(x[i].y), "f"(x[i].z), "f"(x[i].w), "r"((int)go)
+                   : "memory");
+  }
 
   // bulk L2 prefetch of one rating's p_u and q_v rows (cp.async.bulk.prefetch, sm_90+)
   __device__ __forceinline__ void prefetch_rows(int u, int v) const {
@@ -782,15 +791,20 @@ struct WarpSgd {
       // groups 0 .. j + D - 1 are committed: at most D - 1 pending = rating j's copy landed
       asm volatile("cp.async.wait_group %0;" ::"n"(D - 1) : "memory");
 #endif
-      if (u != cu) {  // a run starts: retire the previous user's row, take this one's
-        if (cu >= 0) st(prow(cu), p);
-#pragma unroll
-        for (int i = 0; i < VEC; ++i) p[i] = pb[(j & (RP - 1)) * k4 + 32 * i];
-        cu = u;
-      }
       float4* qw = sb + v * k4;
 #pragma unroll
       for (int i = 0; i < VEC; ++i) q[i] = qw[32 * i];  // after the previous write: serial order
+      {  // a run starts: retire the previous user's row, take this one's (branch-free: every
+         // rating's row was copied; inside a run the registers hold the current row)
+        const bool newrun = u != cu;
+        float4 pr[VEC];
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) pr[i] = pb[(j & (RP - 1)) * k4 + 32 * i];
+        st_if(prow(cu < 0 ? u : cu), p, newrun && cu >= 0);
+#pragma unroll
+        for (int i = 0; i < VEC; ++i) p[i] = newrun ? pr[i] : p[i];
+        cu = u;
+      }
       if (j + 1 < left) rc = ring[(j + 1) & 63];  // visible since its window's boundary (j + 1 < j + D)
       float2 dd = make_float2(0.f, 0.f);
 #pragma unroll
@@ -805,9 +819,8 @@ struct WarpSgd {
         d += __shfl_xor_sync(FM, d, o);
         if (o == 16) {  // look-ahead of rating j + D: its user's p_u copy, one commit group
           const int jn = j + D;
-          const bool go = jn < left && un != lastu;
-          copy_p_if(jn & (RP - 1), go ? un : lastu, go);
-          if (go) lastu = un;
+          const bool go = jn < left;
+          copy_p_if(jn & (RP - 1), un, go);
           asm volatile("cp.async.commit_group;" ::: "memory");
         }
       }
