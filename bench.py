@@ -55,6 +55,9 @@ PROBE_MODE = {"fp32": "red_f32", "fp16": "ldred_f16"}
 UNIT = "updates/s"
 FALLBACK_HBM_GBS = 6650.0
 DEVICE_GEN_NNZ = 1_000_000_000
+# the C3 DET leg: a B x B grid on degree-balanced column blocks (R30); 1024-1536 measure alike
+# (29.7-30.4 ms per epoch, profiles/r02_det.md), 1536 has its full-size oracle sample
+DET_B = 1536
 
 
 def parse():
@@ -565,9 +568,9 @@ def main():
         torch.cuda.empty_cache()
     if "det" in legs:
         kd = min(args.steps, 3)
-        d = run_workload(cx, "c3", "det", ["fp32"], kd, False, det_grid=(2048, 2048), col_balance=True)
+        d = run_workload(cx, "c3", "det", ["fp32"], kd, False, det_grid=(DET_B, DET_B), col_balance=True)
         out["legs"]["det"] = dict(leg_json(d, "fp32", kd, args.warmup), workload=f"{d['cfg'].name} (c3)",
-                                  grid=[2048, 2048], sched="det", det_path=d.get("det_path"), col_balance=True,
+                                  grid=[DET_B, DET_B], sched="det", det_path=d.get("det_path"), col_balance=True,
                                   note="serial-equivalent FPSGD strata (R19) as one wavefront launch per epoch, "
                                        "degree-balanced column blocks (R30); bound by the heaviest column "
                                        "block's serial chain")

@@ -146,19 +146,20 @@ def test_c3_det_epoch_full_size(pkg, c3):
     assert np.abs(Q[ref["items"]] - ref["Q"]).max() <= 1e-4
 
 
-def test_c3_det_epoch_full_size_col_balance(pkg, c3):
-    # bench.py's DET leg: 2048 x 2048 grid on degree-balanced column blocks (R30), the slab
-    # wavefront, one launch: partition digest bit-exact and sampled rows (heaviest users and
-    # items included) within 1e-4 of the oracle's DET epoch on the same partition
-    path = os.path.join(GOLDEN, "oracle_det_c3_B2048_bal.npz")
+@pytest.mark.parametrize("B", [1536, 2048])
+def test_c3_det_epoch_full_size_col_balance(pkg, c3, B):
+    # bench.py's DET leg (B = 1536; 2048 as well): B x B grid on degree-balanced column blocks
+    # (R30), the slab wavefront, one launch: partition digest bit-exact and sampled rows
+    # (heaviest users and items included) within 1e-4 of the oracle's DET epoch on the same partition
+    path = os.path.join(GOLDEN, f"oracle_det_c3_B{B}_bal.npz")
     if not os.path.exists(path):
-        pytest.skip("tools/oracle_curves.py det:c3:2048:bal not run")
+        pytest.skip(f"tools/oracle_curves.py det:c3:{B}:bal not run")
     ref = np.load(path)
     cfg = synth.CONFIGS["c3"]
     (u, v, r), _ = c3
     mdl = pkg.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam)
     mdl.load(u, v, r)
-    mdl.partition(1, (2048, 2048), seed=cfg.seed, col_balance=True)
+    mdl.partition(1, (B, B), seed=cfg.seed, col_balance=True)
     assert _digest(mdl) == str(ref["digest"])
     mdl.init(1)
     l0 = pkg.kernel_launches()
