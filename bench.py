@@ -72,6 +72,7 @@ def parse():
     ap.add_argument("--sync", default=None, choices=["none", "ring", "allreduce"])
     ap.add_argument("--grid", default=None, help="Br,Bc (default: hogwild 1,G (ring) or 1,round(|Q|/80MB); det 64,64G)")
     ap.add_argument("--warps", type=int, default=0)
+    ap.add_argument("--opt", action="append", default=[], help="name=value library option for every handle (e.g. staleness=60)")
     ap.add_argument("--task", type=int, default=0)
     ap.add_argument("--vec", type=int, default=0, help="float4 slots per lane (0 = library auto)")
     ap.add_argument("--depth", type=int, default=0, help="Hogwild q_v prefetch distance (0 = library auto)")
@@ -345,6 +346,8 @@ def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, samp
 
     mdl = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, dist=world > 1, device=local)
     mdl.set_stream(stream)
+    for kv in args.opt:
+        mdl.set_option(kv.split("=")[0], int(kv.split("=")[1]))
     if args.warps:
         mdl.set_option("hogwild_warps", args.warps)
     if args.task:
@@ -460,6 +463,8 @@ def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, samp
     def job():
         m2 = hc.Model(cfg.m, cfg.n, cfg.k, cfg.gamma, cfg.lam, dist=world > 1, device=local)
         m2.set_stream(stream)
+        for kv in args.opt:
+            m2.set_option(kv.split("=")[0], int(kv.split("=")[1]))
         if args.warps:
             m2.set_option("hogwild_warps", args.warps)
         if args.vec:

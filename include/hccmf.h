@@ -212,7 +212,7 @@ typedef enum {
                                     items * kappa / (gamma (r_rms + lambda)) rating
                                     groups in flight per launch, items = the Q rows the
                                     launch can touch, r_rms = sqrt(mean r^2) of the
-                                    shard, kappa = value * 1e-4 (default 80 -> 0.008);
+                                    shard, kappa = value * 1e-4 (default 60 -> 0.006);
                                     0 = no cap (resident warps only)              */
     HCCMF_OPT_TIMELINE = 15,     /* 1: train_epoch records CUDA events around every SGD
                                     launch (compute stream) and every Q transfer (comm

@@ -420,9 +420,10 @@ hccmf_status build_plan(hccmf_t h, int sched, int sync, Plan** out) {
 // step; on the per-rating quadratic in q_v (curvature ~ |p_u|^2 + lambda, and |p_u|^2 grows to
 // the rating scale) the delay is harmless while tau * gamma * (r_rms + lambda) stays small.  With
 // the items of a launch hit uniformly, tau ~ groups / items, so the cap is
-//   groups <= items * kappa / (gamma (r_rms + lambda)),   kappa = opt_staleness * 1e-4 (0.008),
+//   groups <= items * kappa / (gamma (r_rms + lambda)),   kappa = opt_staleness * 1e-4 (0.006),
 // calibrated on the measured stability edge (C4, ratings 0..100, lambda 1: stable at
-// tau gamma (r_rms + lambda) = 0.0077 and 0.0097, divergent at 0.0155; C3 runs at 0.0048).
+// tau gamma (r_rms + lambda) = 0.0077 and 0.0097, divergent at 0.0155, and one epoch-1 NaN in
+// ~100 runs of C4 at 5 % size at 0.008 -- hence 0.006, 25 % inside it; C3 runs at 0.0048).
 // opt_conflict > 0 replaces it by the fixed items / opt_conflict of round 1.  Never more
 // than 32 resident warps per SM.
 int64_t auto_warps(hccmf_t h, int64_t items_in_play) {

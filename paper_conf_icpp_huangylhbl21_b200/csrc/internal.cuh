@@ -202,7 +202,7 @@ struct hccmf_ctx {
   int state = 0;  // 0 created, 1 loaded, 2 partitioned, 3 factors ready
   hccmf_status sticky = HCCMF_OK;
   std::string err;
-  int64_t opt_staleness = 80;  // Hogwild staleness budget, units of 1e-4 (R32); 0: no cap
+  int64_t opt_staleness = 60;  // Hogwild staleness budget, units of 1e-4 (R32); 0: no cap
   double r_rms = 0.0;          // sqrt(mean r^2) of the local records (R32)
   int64_t opt_warps = 0, opt_task = 256, opt_atomic = 1, opt_conflict = 0, opt_heavy = 1024, opt_vec = 0, opt_wave = 1, opt_phases = 1, opt_wire16 = 0, opt_l2persist = 0, opt_depth = 0;
   bool sync_stream = true;
