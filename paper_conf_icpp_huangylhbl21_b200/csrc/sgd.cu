@@ -714,8 +714,11 @@ struct WarpSgd {
   // the p_u ring fill of the first D ratings, which touch only this warp's own rows -- runs
   // BEFORE wait_load() waits for the predecessor and stages the column block's Q slab.
   template <class WaitLoad>
+  // The last run's p_u row is NOT stored here: it is returned in (last_u, last_p) and the
+  // caller stores it after releasing the column block, so the release fence does not wait
+  // for it (P rows are this warp's own; the next block's copies follow it in program order).
   __device__ __forceinline__ void run_slab_ring(int64_t lo, int left, float4* slab, int c0, float4* pring, int4* ring,
-                                                WaitLoad&& wait_load) {
+                                                WaitLoad&& wait_load, int& last_u, float4 (&last_p)[VEC]) {
     constexpr int D = kSlabD, RP = kSlabRP;
     static_assert(RP > D && (RP & (RP - 1)) == 0 && D < 16, "ring: window w + 1 lands before window w is reached");
     const int32_t* ru = a.ru + lo;
@@ -835,7 +838,9 @@ struct WarpSgd {
       if (jn1 < left && (jn1 & 15) == 0) boundary(jn1 >> 4);
       un = ring[jn1 & 63].x;  // beyond the block: a stale entry, never copied
     }
-    if (cu >= 0) st(prow(cu), p);
+    last_u = cu;
+#pragma unroll
+    for (int i = 0; i < VEC; ++i) last_p[i] = p[i];
     asm volatile("cp.async.wait_group 0;" ::: "memory");  // nothing may still target the rings
     __syncwarp();  // the record ring is rewritten by the next block's prologue
   }
@@ -1235,6 +1240,8 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(b0), "r"(bytes) : "memory");
   };
   const int64_t* row_off = off + (int64_t)i * B;  // block (i, c) = row_off[c] .. row_off[c + 1]
+  int last_u = -1;
+  float4 last_p[VEC];
   prefetch_records(row_off[i], row_off[i + 1]);
   if (B > 1) prefetch_records(row_off[(i + 1) % B], row_off[(i + 1) % B + 1]);
   for (int t = 0; t < B; ++t) {
@@ -1294,7 +1301,7 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
       }
     };
     if (hi > lo) {
-      w.run_slab_ring(lo, (int)(hi - lo), slab, c0, pring, rring, wait_load);
+      w.run_slab_ring(lo, (int)(hi - lo), slab, c0, pring, rring, wait_load, last_u, last_p);
       for (int r = 0; r < rows; ++r) {
 #pragma unroll
         for (int s = 0; s < VEC; ++s)
@@ -1310,6 +1317,10 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
 #ifdef HCCMF_DIAG_TRACE
       if (B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3 + 2] = gtimer();
 #endif
+    }
+    if (last_u >= 0) {  // the block's last p_u run, after the release (see run_slab_ring)
+      w.st(w.prow(last_u), last_p);
+      last_u = -1;
     }
   }
 }
