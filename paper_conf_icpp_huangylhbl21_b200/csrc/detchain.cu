@@ -288,7 +288,9 @@ __global__ void __launch_bounds__(NW * 32) sgd_wave_chain_kernel(ChainArgs a, in
           asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + (int64_t)nb * kProgressStride) : "memory");
           if (seen < t) __nanosleep(64);
         } while (seen < t);
-        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+        // acquire pattern (relaxed read + fence.acquire: CCTL.IVALL, no MEMBAR -- a full
+        // fence here would also wait for this warp's own outstanding copies and prefetches)
+        asm volatile("fence.acquire.gpu;" ::: "memory");
       }
       __syncthreads();
     }

@@ -1178,7 +1178,9 @@ __global__ void __launch_bounds__(kThreads) sgd_wave_kernel(SgdArgs a, const int
           asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + (int64_t)nb * kProgressStride) : "memory");
           if (seen < t) __nanosleep(64);
         } while (seen < t);
-        asm volatile("fence.acq_rel.gpu;" ::: "memory");
+        // acquire pattern (relaxed read + fence.acquire: CCTL.IVALL, no MEMBAR -- a full
+        // fence here would also wait for this warp's own outstanding copies and prefetches)
+        asm volatile("fence.acquire.gpu;" ::: "memory");
       }
       __syncwarp();
     }
@@ -1187,7 +1189,7 @@ __global__ void __launch_bounds__(kThreads) sgd_wave_kernel(SgdArgs a, const int
     if (hi > lo) w.run(lo, (int)(hi - lo));
     __syncwarp();
     if (w.lane == 0) {
-      asm volatile("fence.acq_rel.gpu;" ::: "memory");  // the warp's writes (ordered by __syncwarp) first
+      asm volatile("fence.release.gpu;" ::: "memory");  // the warp's writes (ordered by __syncwarp) first
       asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(progress + (int64_t)i * kProgressStride), "r"(t + 1) : "memory");
     }
   }
@@ -1277,7 +1279,9 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
             asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + (int64_t)nb * kProgressStride) : "memory");
             if (seen < t) __nanosleep(64);
           } while (seen < t);
-          asm volatile("fence.acq_rel.gpu;" ::: "memory");
+          // acquire pattern (relaxed read + fence.acquire: CCTL.IVALL, no MEMBAR -- a full
+          // fence here would also wait for this warp's own outstanding copies and prefetches)
+          asm volatile("fence.acquire.gpu;" ::: "memory");
         }
         __syncwarp();
       }
@@ -1285,8 +1289,6 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
 #ifdef HCCMF_DIAG_TRACE
       if (w.lane == 0 && B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3 + 1] = gtimer();
 #endif
-      if (nu0 >= 0) w.prefetch_p(nu0);
-      if (nu1 >= 0) w.prefetch_p(nu1);
       if (hi > lo) {
         for (int r = 0; r < rows; ++r) {
 #pragma unroll
@@ -1299,6 +1301,9 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
         }
         asm volatile("cp.async.commit_group;\n\tcp.async.wait_group 0;" ::: "memory");
       }
+      // the next block's first 64 users' p_u rows -> L2 (its prologue copies hit there)
+      if (nu0 >= 0) w.prefetch_p(nu0);
+      if (nu1 >= 0) w.prefetch_p(nu1);
     };
     if (hi > lo) {
       w.run_slab_ring(lo, (int)(hi - lo), slab, c0, pring, rring, wait_load, last_u, last_p);
@@ -1312,7 +1317,7 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
     }
     __syncwarp();
     if (w.lane == 0) {
-      asm volatile("fence.acq_rel.gpu;" ::: "memory");  // the warp's writes (ordered by __syncwarp) first
+      asm volatile("fence.release.gpu;" ::: "memory");  // the warp's writes (ordered by __syncwarp) first
       asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(progress + (int64_t)i * kProgressStride), "r"(t + 1) : "memory");
 #ifdef HCCMF_DIAG_TRACE
       if (B <= 2048) g_wave_trace[((int64_t)i * B + t) * 3 + 2] = gtimer();
