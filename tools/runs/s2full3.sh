@@ -1,14 +1,12 @@
-export HCCMF_BAND_REPORT=$PWD/gpurun_out/band_report_s2d.jsonl
+export HCCMF_BAND_REPORT=$PWD/gpurun_out/band_report_s2e.jsonl
 rm -f $HCCMF_BAND_REPORT
-timeout 2400 python -m pytest tests -m gpu -q --durations=5 > gpurun_out/gputest_s2d.log 2>&1
-echo "pytest rc=$?"; tail -6 gpurun_out/gputest_s2d.log
-timeout 900 python tools/rank_rate.py --config c5 --G 1 2 4 8 2>&1 | tail -5
-timeout 900 python tools/rank_rate.py --config c3 --G 1 2 4 8 2>&1 | tail -5
-timeout 1500 python bench.py > gpurun_out/bench_s2d.json 2> gpurun_out/bench_s2d.err
-echo "bench rc=$?"; tail -3 gpurun_out/bench_s2d.err
+timeout 2400 python -m pytest tests -m gpu -q --durations=5 > gpurun_out/gputest_s2e.log 2>&1
+echo "pytest rc=$?"; tail -6 gpurun_out/gputest_s2e.log
+timeout 1500 python bench.py > gpurun_out/bench_s2e.json 2> gpurun_out/bench_s2e.err
+echo "bench rc=$?"; tail -3 gpurun_out/bench_s2e.err
 python - <<'PY'
 import json
-d=json.load(open('gpurun_out/bench_s2d.json'))
+d=json.load(open('gpurun_out/bench_s2e.json'))
 r=d['roofline']
 print('C5', round(d['value']/1e9,3), round(d['ms_per_step'],1), d['clocks'], 'frac', round(r['frac'],4), 'bfrac', round(r['binding_frac'],3), 'rtfrac', round(r.get('roundtrip_frac',0),3))
 print('fp16', round(d['storage_fp16']['value']/1e9,3), d['storage_fp16']['roofline']['binding_frac'])
