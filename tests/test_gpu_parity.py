@@ -295,6 +295,32 @@ def test_hogwild_single_group_column_phases(pkg, orc, Bc, scale):
     assert max(np.abs(P - Po).max(), np.abs(Q - Qo).max()) <= 1e-4 * max(1.0, scale)
 
 
+@pytest.mark.parametrize("m,n,nnz,Bc", [(40, 7, 300, 12), (300, 5, 2500, 9), (30, 64, 0, 4), (1, 50, 200, 70)])
+def test_hogwild_single_group_empty_blocks(pkg, orc, m, n, nnz, Bc):
+    # grid (1, Bc) with empty column blocks (Bc > items, or no ratings at all): the per-block
+    # task offsets and the plan's task lists are built on the device (no host copy of the
+    # tasks); one warp walks them in record order = the oracle's serial epoch, 1e-4
+    u, v, r = synth.tiny(m, n, nnz, seed=m + n + Bc)
+    prob = orc.Problem(m, n, 128, 0.02, 0.01, u, v, r, G=1, Br=1, Bc=Bc, seed=7)
+    prob.init(2)
+    P0, Q0 = [x.astype(np.float32) for x in prob.factors()]
+    prob.set_factors(P0, Q0)
+    mdl = pkg.Model(m, n, 128, 0.02, 0.01)
+    mdl.set_option("heavy_first", -1)
+    mdl.set_option("task_ratings", 7)  # several tasks per block
+    mdl.load(u, v, r)
+    mdl.partition(1, (1, Bc), seed=7)
+    mdl.set_option("hogwild_warps", 1)
+    mdl.set_factors(P0, Q0)
+    for _ in range(2):
+        mdl.train_epoch("hogwild", "none")
+        prob.epoch("serial", "none")
+    P, Q = mdl.factors()
+    Po, Qo = prob.factors()
+    mdl.close()
+    assert max(np.abs(P - Po).max(initial=0.0), np.abs(Q - Qo).max(initial=0.0)) <= 1e-4
+
+
 def _band(pkg, orc, cfg_name, frac, k, epochs, sync="none", G=1, Br=1, Bc=1, repeats=2, gamma=None):
     """GPU and oracle test-RMSE curves (same data, same schedule, init seed 1), checked with the
     shared bar of tests/bands.py (R15, R29) for every repeat."""
