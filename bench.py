@@ -291,8 +291,46 @@ def roofline(cfg, name, storage, sched, info, kmean_ms, step_ms, peak, peak_src,
                 roof["roundtrip_frac"] = probe[2] / kmean_ms
     else:
         roof["binding_unit"] = ("the hottest column block's serial dependency chain (wavefront; "
-                                "profiles/r01_det_wavefront.md)")
+                                "profiles/r02_det.md)")
+        if probe:  # latency roof: the heaviest column block's ratings x one warp's uncontended chain
+            roof["binding_ceiling"] = probe
+            roof["binding_frac"] = probe["ms"] / kmean_ms
     return roof
+
+
+def det_latency_ceiling(hc, mdl, cfg, Br, Bc):
+    """The DET epoch's latency bound, measured in this run: every rating of the heaviest column
+    block passes through its successive owners in order, so the epoch takes at least (its ratings) x
+    (one warp's per-rating time on a same-item chain with no other warps around).  The chain time
+    comes from a 2 x 2 wavefront whose column blocks hold one item each (tools/det_chain_latency.py)."""
+    import torch
+    _, off, _, _ = mdl.get_partition()
+    per_block = np.diff(off).reshape(Br, Bc)
+    crit = int(per_block.sum(axis=0).max())
+    nr = 1 << 20
+    rng = np.random.default_rng(1)
+    u = np.arange(nr, dtype=np.int32)
+    v = rng.integers(0, 2, nr).astype(np.int32)
+    r = rng.uniform(1, 5, nr).astype(np.float32)
+    m2 = hc.Model(nr, 2, cfg.k, cfg.gamma, cfg.lam)
+    m2.load(u, v, r)
+    m2.partition(1, (2, 2), seed=3)
+    m2.init(1)
+    s = torch.cuda.Stream()
+    m2.set_stream(s)
+    ts = []
+    for _ in range(3):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        m2.train_epoch("det", "none")
+        e1.record(s)
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    m2.close()
+    ns = float(np.median(ts[1:])) * 1e6 / (nr / 2)  # two warps, each over half the ratings
+    return {"critical_ratings": crit, "chain_ns_per_rating": ns, "ms": crit * ns / 1e6,
+            "source": "heaviest column block's ratings x one warp's same-item chain (2 x 2 wavefront, one item "
+                      "per column block), measured in this run"}
 
 
 def hogwild_phases(cfg):
@@ -422,6 +460,8 @@ def run_workload(cx, name, sched, storages, steps, want_e2e, det_grid=None, samp
             probe = (mode, mdl.probe_roundtrip(mode, warps=args.warps, reps=3))
             if storage == "fp32":  # the load + dependent reduction round trip as well (the kernel's own pattern)
                 probe = probe + (mdl.probe_roundtrip("ldred_f32", warps=args.warps, reps=3),)
+        if sched == "det" and world == 1 and cfg.k % 128 == 0:
+            probe = det_latency_ceiling(hc, mdl, cfg, Br, Bc)
         roof = roofline(cfg, name, storage, sched, info, kmean, ms / steps, peak, peak_src, probe)
         return {"value": nnz * steps / (ms / 1e3), "ms": ms, "roofline": roof, "clocks": clk,
                 "curve": curve + rms, "launches": launches}
