@@ -56,9 +56,9 @@ PROBE_MODE = {"fp32": "red_f32", "fp16": "ldred_f16"}
 UNIT = "updates/s"
 FALLBACK_HBM_GBS = 6650.0
 DEVICE_GEN_NNZ = 1_000_000_000
-# the C3 DET leg: a B x B grid on degree-balanced column blocks (R30); 1024-1536 measure alike
-# (29.7-30.4 ms per epoch, profiles/r02_det.md), 1536 has its full-size oracle sample
-DET_B = 1536
+# the C3 DET leg: a B x B grid on degree-balanced column blocks (R30); 1024-1536 measure alike,
+# 1184 the fastest by ~0.5 ms (profiles/r02_det.md); it has its full-size oracle sample
+DET_B = 1184
 
 
 def parse():

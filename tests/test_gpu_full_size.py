@@ -146,9 +146,9 @@ def test_c3_det_epoch_full_size(pkg, c3):
     assert np.abs(Q[ref["items"]] - ref["Q"]).max() <= 1e-4
 
 
-@pytest.mark.parametrize("B", [1536, 2048])
+@pytest.mark.parametrize("B", [1184, 1536, 2048])
 def test_c3_det_epoch_full_size_col_balance(pkg, c3, B):
-    # bench.py's DET leg (B = 1536; 2048 as well): B x B grid on degree-balanced column blocks
+    # bench.py's DET leg (B = 1184; 1536 and 2048 as well): B x B grid on degree-balanced column blocks
     # (R30), the slab wavefront, one launch: partition digest bit-exact and sampled rows
     # (heaviest users and items included) within 1e-4 of the oracle's DET epoch on the same partition
     path = os.path.join(GOLDEN, f"oracle_det_c3_B{B}_bal.npz")
