@@ -390,7 +390,10 @@ HCCMF_API hccmf_status hccmf_cost_model(int32_t p, int64_t m, int64_t n, int64_t
  * load + dependent reduction (red.v2.f16x2), 2 fp32 load + dependent reduction, 3 the
  * q_v stream alone (loads of the model's Q), 4 the p_u stream alone (per user run one load
  * of the row and one store of the same values: the model is left unchanged).  Modes 3-4
- * let ncu report the L2 hit rate of the Q and of the P stream separately.
+ * let ncu report the L2 hit rate of the Q and of the P stream separately.  Modes 5-9 move
+ * the row through the TMA bulk-copy engine (profiles/r02_probe_tma.md): 5 bulk reductions
+ * only, 7 per-lane load + bulk reduction, 6 / 8 / 9 bulk load 3 / 7 / 1 ratings ahead + a
+ * dependent bulk reduction (k = 128 only).
  * *ms = mean duration of one pass over `reps` timed passes (CUDA events on the handle's
  * stream, after one warm-up pass).  Needs partition; k a multiple of 128. */
 HCCMF_API hccmf_status hccmf_probe_roundtrip(hccmf_t h, int32_t mode, int64_t warps, int32_t reps, double* ms);
