@@ -706,17 +706,17 @@ struct WarpSgd {
   // written back to HBM when the run ends; a run's row was last written by this warp,
   // before the fence of an earlier block.  Same arithmetic as run() and run_ring(): the
   // factors are bit-identical to the per-stratum launches.
-  // The block's start is off the wavefront's critical path (round 2; C3, B = 2048: 45.1 ->
-  // 39.0 ms per epoch, profiles/r02_det.md): the records enter a per-warp shared-memory
-  // ring of 4 windows of 16 by cp.async (window w + 2 is issued when window w is reached;
-  // one LDS.128 per rating for the update and one LDS.32 for the p_u copy D ahead, instead
-  // of six shuffles out of register windows), and the prologue -- the first windows and
-  // the p_u ring fill of the first D ratings, which touch only this warp's own rows -- runs
-  // BEFORE wait_load() waits for the predecessor and stages the column block's Q slab.
+  // Round 2 (C3 DET epoch 45.1 -> 29.3 ms, profiles/r02_det.md).  The block's start is off
+  // the wavefront's critical path: the records enter a per-warp shared-memory ring of 4
+  // windows of 16 by cp.async (window w + 2 is issued when window w is reached; one LDS.128
+  // per rating for the update and one LDS.32 for the p_u copy D ahead, instead of six
+  // shuffles out of register windows), and the prologue -- the first windows and the p_u
+  // ring fill of the first D ratings, which touch only this warp's own rows -- runs BEFORE
+  // wait_load() waits for the predecessor and stages the column block's Q slab.  The last
+  // run's p_u row is NOT stored here: it is returned in (last_u, last_p) and the caller
+  // stores it after releasing the column block, so the release fence does not wait for it
+  // (P rows are this warp's own; the next block's copies follow it in program order).
   template <class WaitLoad>
-  // The last run's p_u row is NOT stored here: it is returned in (last_u, last_p) and the
-  // caller stores it after releasing the column block, so the release fence does not wait
-  // for it (P rows are this warp's own; the next block's copies follow it in program order).
   __device__ __forceinline__ void run_slab_ring(int64_t lo, int left, float4* slab, int c0, float4* pring, int4* ring,
                                                 WaitLoad&& wait_load, int& last_u, float4 (&last_p)[VEC]) {
     constexpr int D = kSlabD, RP = kSlabRP;
