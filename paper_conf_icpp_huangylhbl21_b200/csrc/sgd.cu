@@ -325,7 +325,10 @@ __global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
 // per-step liveness predicates).  Same pipeline as Group: rating j+1's record and
 // q row are in flight while rating j is updated.
 // DET slab wavefront: p_u copy distance (ratings) and ring slots (> distance, power of 2)
-constexpr int kSlabD = 12, kSlabRP = 16;
+#ifndef HCCMF_SLAB_D  // diagnostic builds may move the p_u copy distance (< 16)
+#define HCCMF_SLAB_D 12
+#endif
+constexpr int kSlabD = HCCMF_SLAB_D, kSlabRP = 16;
 
 template <int VEC, bool ATOMIC>
 struct WarpSgd {
