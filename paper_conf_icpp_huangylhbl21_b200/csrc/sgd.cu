@@ -325,6 +325,10 @@ __global__ void __launch_bounds__(kThreads) sgd_kernel(SgdArgs a) {
 // per-step liveness predicates).  Same pipeline as Group: rating j+1's record and
 // q row are in flight while rating j is updated.
 // DET slab wavefront: p_u copy distance (ratings) and ring slots (> distance, power of 2)
+#ifndef HCCMF_POLL_NS  // the slab wavefront's pause between polls of its predecessor's counter
+#define HCCMF_POLL_NS 64
+#endif
+constexpr unsigned kPollNs = HCCMF_POLL_NS;
 #ifndef HCCMF_SLAB_D  // diagnostic builds may move the p_u copy distance (< 16)
 #define HCCMF_SLAB_D 12
 #endif
@@ -1280,7 +1284,7 @@ __global__ void __launch_bounds__(kThreads, 2) sgd_wave_slab_kernel(SgdArgs a, c
             // relaxed polling (an acquire load per poll invalidates the SM's L1 every
             // time: CCTL.IVALL), one acquire fence once the predecessor is seen
             asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(seen) : "l"(progress + (int64_t)nb * kProgressStride) : "memory");
-            if (seen < t) __nanosleep(64);
+            if (seen < t && kPollNs) __nanosleep(kPollNs);
           } while (seen < t);
           // acquire pattern (relaxed read + fence.acquire: CCTL.IVALL, no MEMBAR -- a full
           // fence here would also wait for this warp's own outstanding copies and prefetches)
