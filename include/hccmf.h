@@ -395,7 +395,9 @@ HCCMF_API hccmf_status hccmf_cost_model(int32_t p, int64_t m, int64_t n, int64_t
  * only, 7 per-lane load + bulk reduction, 6 / 8 / 9 bulk load 3 / 7 / 1 ratings ahead + a
  * dependent bulk reduction (k = 128 only).
  * *ms = mean duration of one pass over `reps` timed passes (CUDA events on the handle's
- * stream, after one warm-up pass).  Needs partition; k a multiple of 128. */
+ * stream, after one warm-up pass).  On a one-shard grid (1, Bc > 1) -- a Hogwild epoch of Bc
+ * column-block phases -- the probe runs phase by phase with each phase's records and warp
+ * count and *ms is the sum.  Needs partition; k a multiple of 128. */
 HCCMF_API hccmf_status hccmf_probe_roundtrip(hccmf_t h, int32_t mode, int64_t warps, int32_t reps, double* ms);
 
 /* The last train_epoch's timeline (HCCMF_OPT_TIMELINE = 1): up to `cap` rows of 5 doubles

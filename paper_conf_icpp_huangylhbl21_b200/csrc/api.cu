@@ -1675,6 +1675,22 @@ hccmf_status hccmf_probe_roundtrip(hccmf_t h, int32_t mode, int64_t warps, int32
   if (!ms || mode < 0 || mode > 9 || warps < 0 || reps < 1) return fail(h, HCCMF_EINVAL, "bad probe arguments");
   if (h->state < 2) return fail(h, HCCMF_ESTATE, "probe needs partition");
   if (h->k % 128 != 0) return fail(h, HCCMF_EINVAL, "probe needs k a multiple of 128");
+  if (h->G == 1 && h->Br == 1 && h->Bc > 1) {
+    // the Hogwild epoch's column-block phases (one launch each, e.g. C4): the same phases with
+    // their own records and warp counts, one after the other; *ms is their sum
+    double sum = 0.0;
+    for (int64_t cb = 0; cb < h->Bc; ++cb) {
+      const int64_t lo = h->block_off[h->blk0 + cb] - h->rec0, hi = h->block_off[h->blk0 + cb + 1] - h->rec0;
+      const int64_t items = ceil_div((cb + 1) * h->n, h->Bc) - ceil_div(cb * h->n, h->Bc);
+      if (hi <= lo) continue;
+      float t = 0.f;
+      CU(h, k_probe_roundtrip(mode, h->d_u + lo, h->d_v + lo, h->d_r + lo, hi - lo, h->k, h->n, h->d_P, h->row0,
+                              h->d_Q, warps ? warps : auto_warps(h, items), reps, &t, h->stream));
+      sum += t;
+    }
+    *ms = sum;
+    return finish(h);
+  }
   const int64_t w = warps ? warps : auto_warps(h, h->n);
   float t = 0.f;
   CU(h, k_probe_roundtrip(mode, h->d_u, h->d_v, h->d_r, h->local_nnz, h->k, h->n, h->d_P, h->row0, h->d_Q, w, reps, &t,
