@@ -811,3 +811,23 @@ def test_det_wavefront_degenerate_grids(pkg, orc, m, n, nnz, B, k):
     assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
     Po, Qo = prob.factors()
     assert max(np.abs(outs[0][0] - Po).max(), np.abs(outs[0][1] - Qo).max()) <= 1e-4
+
+
+@pytest.mark.parametrize("Bc", [1, 3])
+def test_probe_roundtrip_leaves_the_model_alone(pkg, Bc):
+    # the in-run ceiling probes (bench.py binding_frac): every mode returns a positive time, on a
+    # (1, Bc) grid phase by phase, and none of them changes the model's factors (the reductions go
+    # to a scratch Q; the p_u stream mode stores back the rows it loaded)
+    cfg = synth.CONFIGS["c1"]
+    (u, v, r), _ = synth.make(cfg)
+    mdl = pkg.Model(cfg.m, cfg.n, 128, 0.005, 0.01)
+    mdl.load(u, v, r)
+    mdl.partition(1, (1, Bc), seed=2)
+    mdl.init(3)
+    P0, Q0 = mdl.factors()
+    for mode in ("red_f32", "ldred_f16", "ldred_f32", "q_stream", "p_stream", "bulkred_f32", "bulkldred_f32",
+                 "ldbulkred_f32"):
+        assert mdl.probe_roundtrip(mode, reps=1) > 0.0, mode
+    P1, Q1 = mdl.factors()
+    mdl.close()
+    assert np.array_equal(P0, P1) and np.array_equal(Q0, Q1)
