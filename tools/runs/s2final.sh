@@ -1,8 +1,8 @@
-timeout 1500 python bench.py > gpurun_out/bench_s2f.json 2> gpurun_out/bench_s2f.err
-echo "bench rc=$?"; tail -2 gpurun_out/bench_s2f.err
+timeout 1500 python bench.py > gpurun_out/bench_s2g.json 2> gpurun_out/bench_s2g.err
+echo "bench rc=$?"; tail -2 gpurun_out/bench_s2g.err
 python - <<'PY'
 import json
-d=json.load(open('gpurun_out/bench_s2f.json'))
+d=json.load(open('gpurun_out/bench_s2g.json'))
 r=d['roofline']
 print('C5', round(d['value']/1e9,3), round(d['ms_per_step'],1), d['clocks'], 'frac', round(r['frac'],4), 'bfrac', round(r['binding_frac'],3), 'rtfrac', round(r.get('roundtrip_frac',0),3))
 print('fp16', round(d['storage_fp16']['value']/1e9,3), d['storage_fp16']['roofline']['binding_frac'])
